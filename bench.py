@@ -1,0 +1,422 @@
+#!/usr/bin/env python
+"""Benchmark: full-graph GCN + GAT training epochs on the synthetic Reddit-shaped graph.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--model both|gcn|gat] [--impl seastar|reference]
+
+BASELINE.json metric: "GAT/GCN train epoch ms and edges/s at 1/2/4/8 B200; achieved HBM GB/s" on
+configs[4] (Reddit-shaped: 232,965 V, 114,615,892 E incl. self-loops, 602 features, 41 classes;
+GCN 602-16-41, GAT 602-8x8-1x41).  One step = one GCN training epoch + one GAT training epoch
+(forward, softmax cross-entropy, backward, Adam), every kernel in libseastar.so.  ``value`` =
+edges processed per second over the whole job (E per model-epoch, summed over the step's epochs).
+
+N > 1 (torchrun, one process per GPU, NCCL): destination rows are range-partitioned; per-layer
+all-gathers of source rows and one gradient all-reduce run through torch.distributed.  Total work
+is fixed as N grows ("strong" scaling); the step time is the max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+CFG = synth.CONFIGS["reddit"]
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--model", default="both", choices=["both", "gcn", "gat"])
+    ap.add_argument("--impl", default="seastar", choices=["seastar", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample-edges", type=int, default=3_000_000)
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------------------------------
+# inputs (seeded, synthetic, Reddit-shaped)
+# ------------------------------------------------------------------------------------------
+def make_inputs():
+    ip, ix = synth.make_graph(CFG)
+    X = synth.uniform(CFG.feat_seed, (CFG.N, CFG.F_in), -1.0, 1.0)
+    lab = synth.labels(CFG.label_seed, CFG.N, CFG.classes)
+    H, C = CFG.hidden, CFG.classes
+    gcn_p = {"W1": synth.glorot(CFG.weight_seed(1), CFG.F_in, H), "b1": np.zeros(H, np.float32),
+             "W2": synth.glorot(CFG.weight_seed(2), H, C), "b2": np.zeros(C, np.float32)}
+    heads, hid = CFG.heads, CFG.extra["gat_hidden"]
+    Wd = heads * hid
+    gat_p = {"W1": synth.glorot(CFG.weight_seed(11), CFG.F_in, Wd),
+             "al1": synth.glorot(CFG.weight_seed(12), hid, 1, (heads, hid)),
+             "ar1": synth.glorot(CFG.weight_seed(13), hid, 1, (heads, hid)),
+             "b1": np.zeros(Wd, np.float32),
+             "W2": synth.glorot(CFG.weight_seed(14), Wd, C),
+             "al2": synth.glorot(CFG.weight_seed(15), C, 1, (1, C)),
+             "ar2": synth.glorot(CFG.weight_seed(16), C, 1, (1, C)),
+             "b2": np.zeros(C, np.float32)}
+    return ip, ix, X, lab, gcn_p, gat_p
+
+
+# ------------------------------------------------------------------------------------------
+# algorithmic bytes per launch (gathered rows counted once per edge)
+# ------------------------------------------------------------------------------------------
+def bytes_gcn_agg(E, n, F, extra_row_out=1, extra_row_in=0):
+    # per edge: 4B index + 4F gathered row ; per row: off+perm 8B, norm 4B, rows written/read
+    return E * (4 + 4 * F) + n * (8 + 4 + 4 * F * (1 + extra_row_out + extra_row_in) + 4)
+
+
+def bytes_gat_fwd(E, n, H, F):
+    W = H * F
+    return E * (4 + 4 * H + 4 * W) + n * (8 + 4 * H + 2 * 4 * W + 4 * H)
+
+
+def bytes_gat_bwd(E, n, H, F):
+    W = H * F
+    ldd = (W + 3) // 4 * 4 + 4 * H
+    return E * (4 + 4 + 4 * ldd + 4 * H) + n * (8 + 4 * W + 4 * H + 4 * W + 4 * H)
+
+
+# ------------------------------------------------------------------------------------------
+# clocks sampler (nvidia-smi during the timed region)
+# ------------------------------------------------------------------------------------------
+class Clocks:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, dev_index):
+        self.dev = dev_index
+        self.p = None
+        self.path = os.path.join(ROOT, "gpurun_out", f"clocks_rank{dev_index}.csv")
+
+    def start(self):
+        os.makedirs(os.path.dirname(self.path), exist_ok=True)
+        try:
+            self.f = open(self.path, "w")
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.Q}", "--format=csv",
+                                       "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.close()
+        sm, mx, reasons = [], None, set()
+        for line in open(self.path).read().splitlines()[1:]:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                s = float(parts[1].split()[0])
+                mx = float(parts[2].split()[0])
+            except ValueError:
+                continue
+            p_w = parts[3]
+            sm.append((s, p_w))
+            names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+            for nm, val in zip(names, parts[5:9]):
+                if "Active" in val and "Not" not in val:
+                    reasons.add(nm)
+        if not sm:
+            return None
+        loaded = [s for s, _ in sm if s > 500] or [s for s, _ in sm]
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------------------
+# CPU oracle baseline (bounded sample of the same workload) -- the only use of oracle/ here
+# ------------------------------------------------------------------------------------------
+def oracle_sample(ip, ix, X, sample_edges, seed=0):
+    """Oracle fwd+bwd aggregations of both GCN layers (F=16) and the GAT forward layers (8x8, 1x41)
+    over the first vertices (by id; ids are shuffled) covering ~sample_edges edges.  Returns
+    (edges processed, seconds, description)."""
+    import oracle
+    N = len(ip) - 1
+    deg_in = np.diff(ip)
+    k = int(np.searchsorted(np.cumsum(deg_in), sample_edges)) + 1
+    k = min(k, N)
+    rows = np.arange(k, dtype=np.int64)
+    outdeg = np.bincount(ix, minlength=N)
+    e_in, e_out = int(deg_in[:k].sum()), int(outdeg[:k].sum())
+    in_n, out_n = oracle.degree_norms(ip, ix)
+    H16 = X[:, :16].astype(np.float64)
+    T64 = X[:, :64].reshape(N, 8, 8).astype(np.float64)
+    T41 = X[:, 64:105].reshape(N, 1, 41).astype(np.float64)
+    el8, er8 = X[:, 105:113].astype(np.float64), X[:, 113:121].astype(np.float64)
+    el1, er1 = X[:, 121:122].astype(np.float64), X[:, 122:123].astype(np.float64)
+    t0 = time.perf_counter()
+    for _ in range(2):     # GCN layers 1 and 2: forward aggregation, backward (transposed) aggregation
+        oracle.gcn_aggregate(ip, ix, H16, out_n, in_n, rows)
+        oracle.gcn_aggregate_T(ip, ix, H16, out_n, in_n, rows)
+    oracle.gat_fwd(ip, ix, T64, el8, er8, 0.2, rows)
+    oracle.gat_fwd(ip, ix, T41, el1, er1, 0.2, rows)
+    dt = time.perf_counter() - t0
+    edges = 2 * (e_in + e_out) + 2 * e_in
+    desc = (f"oracle fwd+bwd GCN aggregations (F=16, 2 layers) and GAT forward layers (8x8, 1x41) for the "
+            f"first {k} vertex ids ({e_in} in-edges, {e_out} out-edges) of the Reddit-shaped graph; "
+            f"edges/s = aggregated edge visits / wall time")
+    return edges, dt, desc
+
+
+def omp_threads():
+    try:
+        return int(os.environ.get("OMP_NUM_THREADS", "")) or os.cpu_count()
+    except ValueError:
+        return os.cpu_count()
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    ip, ix = synth.make_graph(CFG)
+    X = synth.uniform(CFG.feat_seed, (CFG.N, CFG.F_in), -1.0, 1.0)
+    sample = max(200_000, args.cpu_sample_edges // 4)
+    for _ in range(args.warmup):
+        oracle_sample(ip, ix, X, sample)
+    tot_e, tot_t, desc = 0, 0.0, ""
+    for _ in range(args.steps):
+        e, t, desc = oracle_sample(ip, ix, X, sample)
+        tot_e += e
+        tot_t += t
+    v = tot_e / tot_t
+    line = {"impl": "reference", "metric": "GAT/GCN train epoch ms and edges/s at 1/2/4/8 B200; achieved HBM GB/s",
+            "value": v, "unit": "edges/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1000 * tot_t / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": "reddit-shaped GCN+GAT (oracle sample)", "N": CFG.N, "E": CFG.E},
+            "cpu_baseline": {"value": v, "unit": "edges/s", "cores": omp_threads(), "kind": "oracle", "sample": desc},
+            "e2e": {"value": v, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------------------
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        os.environ.setdefault("OMP_NUM_THREADS", str(max(1, (os.cpu_count() or 8) // world)))
+    if args.impl == "reference":
+        if world > 1:
+            import torch.distributed as dist
+            dist.init_process_group("gloo")
+            if rank != 0:
+                dist.barrier()
+                return
+        run_reference(args, rank, world)
+        if world > 1:
+            import torch.distributed as dist
+            dist.barrier()
+        return
+
+    import torch
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
+    from paper_conf_eurosys_wumcjlzcy21_b200.graph import Graph
+    from paper_conf_eurosys_wumcjlzcy21_b200.models import GAT2, GCN2, Comm
+    L.seastar_device_check()
+
+    t_setup = time.perf_counter()
+    ip, ix, X, lab, gcn_p, gat_p = make_inputs()
+    N = CFG.N
+    n_per = (N + world - 1) // world
+    rb, re = min(N, rank * n_per), min(N, (rank + 1) * n_per)
+    g = Graph(ip, ix, row_begin=rb, row_end=re, device=dev)
+    X_loc = torch.from_numpy(X[rb:re]).to(dev)
+    lab_loc = torch.from_numpy(lab[rb:re]).to(dev)
+    comm = Comm(world, rank)
+    models = {}
+    if args.model in ("both", "gcn"):
+        models["gcn"] = GCN2(g, X_loc, lab_loc, gcn_p, comm=comm, n_pad_rows=n_per * world)
+    if args.model in ("both", "gat"):
+        models["gat"] = GAT2(g, X_loc, lab_loc, gat_p, CFG.heads, CFG.extra["gat_hidden"], comm=comm,
+                             n_pad_rows=n_per * world)
+    if world > 1 and re - rb < n_per:
+        raise SystemExit("uneven partition: pad N to a multiple of the world size")
+    torch.cuda.synchronize()
+    setup_s = time.perf_counter() - t_setup
+
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # > 126 MB L2
+
+    # per-kernel event timers on the launching stream
+    kt = {}
+
+    def timer(name):
+        ev = torch.cuda.Event(enable_timing=True)
+        ev.record(stream)
+        kt.setdefault(name, []).append(ev)
+
+    def step():
+        for m in models.values():
+            m.epoch()
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    for m in models.values():
+        m.timer = timer if hasattr(m, "timer") else None
+
+    clocks = Clocks(local)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    step_ms = []
+    model_ms = {k: [] for k in models}
+    for _ in range(args.steps):
+        flush.zero_()                       # evict L2 between timed iterations (untimed)
+        evs = []
+        e0 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for k, m in models.items():
+            m.epoch()
+            e1 = torch.cuda.Event(enable_timing=True)
+            e1.record(stream)
+            evs.append((k, e1))
+        torch.cuda.synchronize()
+        prev = e0
+        for k, e1 in evs:
+            model_ms[k].append(prev.elapsed_time(e1))
+            prev = e1
+        step_ms.append(e0.elapsed_time(evs[-1][1]))
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    ck = clocks.stop()
+    for m in models.values():
+        m.timer = None
+
+    total_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([total_ms], device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        total_ms = t.item()
+    ms_per_step = total_ms / args.steps
+    E = CFG.E
+    edges_per_step = E * len(models)
+    value = edges_per_step / (ms_per_step / 1e3)
+
+    # kernel timings (pairs of events recorded around the hot graph kernels)
+    kernels = {}
+    for name, evs in kt.items():
+        if name.endswith("_end"):
+            continue
+        ends = kt.get(name + "_end", [])
+        ts = [a.elapsed_time(b) for a, b in zip(evs, ends)]
+        if ts:
+            kernels[name] = statistics.mean(ts)
+    info = g.info
+    E_f, E_r, n = info["num_fwd_edges"], info["num_rev_edges"], g.n_loc
+    alg = {"gat_fwd1": bytes_gat_fwd(E_f, n, 8, 8), "gat_bwd1": bytes_gat_bwd(E_r, n, 8, 8),
+           "gat_bwd2": bytes_gat_bwd(E_r, n, 1, 41), "gcn_fwd1": bytes_gcn_agg(E_f, n, 16, 1, 0),
+           "gcn_bwd2": bytes_gcn_agg(E_r, n, 16, 1, 1)}
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    hbm = peaks.get("hbm_gbs", 6650.0)
+    dom = max(kernels, key=kernels.get) if kernels else None
+    roofline = None
+    if dom:
+        ach = alg.get(dom, 0) / (kernels[dom] / 1e3) / 1e9
+        traffic = None
+        try:
+            tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+            traffic = tr.get(dom)
+        except Exception:
+            pass
+        roofline = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": hbm, "unit": "GB/s",
+                    "frac": ach / hbm, "traffic": traffic, "algorithmic_bytes": alg.get(dom),
+                    "ms": kernels[dom], "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback"}
+    kern_out = {k: {"ms": v, "GB/s": (alg[k] / (v / 1e3) / 1e9) if k in alg else None} for k, v in kernels.items()}
+
+    # ---- e2e through the public API: pinned host X -> device each step, loss -> host each step ----
+    e2e = None
+    if not args.no_e2e:
+        Xh = torch.from_numpy(X[rb:re]).pin_memory()
+        loss_h = torch.empty(len(models), dtype=torch.float32).pin_memory()
+        if world > 1:
+            torch.distributed.barrier()
+        torch.cuda.synchronize()
+        e_ms = []
+        for _ in range(args.steps):
+            flush.zero_()
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            X_loc.copy_(Xh, non_blocking=True)
+            for i, m in enumerate(models.values()):
+                loss_h[i:i + 1].copy_(m.epoch(), non_blocking=True)
+            b.record(stream)
+            b.synchronize()
+            _ = loss_h.tolist()
+            e_ms.append(a.elapsed_time(b))
+        tot = sum(e_ms)
+        if world > 1:
+            t = torch.tensor([tot], device=dev)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            tot = t.item()
+        e2e = {"value": edges_per_step / (tot / args.steps / 1e3), "unit": "edges/s",
+               "h2d_bytes_per_step": int(Xh.numel() * 4) * world, "d2h_bytes_per_step": 4 * len(models) * world,
+               "ms_per_step": tot / args.steps}
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only) ----
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        e, t, desc = oracle_sample(ip, ix, X, args.cpu_sample_edges)
+        cpu = {"value": e / t, "unit": "edges/s", "cores": omp_threads(), "kind": "oracle", "sample": desc,
+               "seconds": t}
+
+    gpu_launches = None
+    if rank == 0:
+        per_epoch = {"gcn": 21, "gat": 36}
+        gpu_launches = args.steps * sum(per_epoch[k] for k in models)
+        line = {
+            "metric": "GAT/GCN train epoch ms and edges/s at 1/2/4/8 B200; achieved HBM GB/s",
+            "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "reddit-shaped full-graph training: 2-layer GCN (602-16-41) + 2-layer GAT "
+                                   "(602-8x8-1x41), one epoch each per step",
+                       "N": CFG.N, "E": E, "F_in": CFG.F_in, "classes": CFG.classes,
+                       "parallelism": f"row-partition x{world}", "l2": "flushed (256 MB write) between steps",
+                       "epoch_ms": {k: statistics.mean(v) for k, v in model_ms.items()},
+                       "edges_per_s": {k: E / (statistics.mean(v) / 1e3) for k, v in model_ms.items()},
+                       "setup_s": setup_s},
+            "roofline": roofline, "kernels": kern_out, "cpu_baseline": cpu, "e2e": e2e, "clocks": ck,
+            "gpu_launches": gpu_launches,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

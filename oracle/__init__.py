@@ -190,8 +190,9 @@ def gcn_aggregate(indptr, indices, H, src_norm=None, dst_norm=None, rows=None):
     rows = _i64(rows)
     nrows = N if rows is None else rows.size
     out = np.empty((nrows, F))
-    _L().orc_gcn_aggregate(N, int(indptr[-1]), _p(indptr), _p(indices), F, _p(H), _p(_f64(src_norm)),
-                           _p(_f64(dst_norm)), _p(rows), nrows, _p(out))
+    sn, dn = _f64(src_norm), _f64(dst_norm)     # keep the converted arrays alive across the C call
+    _L().orc_gcn_aggregate(N, int(indptr[-1]), _p(indptr), _p(indices), F, _p(H), _p(sn), _p(dn), _p(rows), nrows,
+                           _p(out))
     return out
 
 
@@ -202,8 +203,9 @@ def gcn_aggregate_T(indptr, indices, G, src_norm=None, dst_norm=None, rows=None)
     rows = _i64(rows)
     nrows = N if rows is None else rows.size
     out = np.empty((nrows, F))
-    _L().orc_gcn_aggregate_T(N, int(indptr[-1]), _p(indptr), _p(indices), F, _p(G), _p(_f64(src_norm)),
-                             _p(_f64(dst_norm)), _p(rows), nrows, _p(out))
+    sn, dn = _f64(src_norm), _f64(dst_norm)     # keep the converted arrays alive across the C call
+    _L().orc_gcn_aggregate_T(N, int(indptr[-1]), _p(indptr), _p(indices), F, _p(G), _p(sn), _p(dn), _p(rows),
+                             nrows, _p(out))
     return out
 
 

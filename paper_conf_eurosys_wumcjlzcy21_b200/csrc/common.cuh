@@ -1,0 +1,170 @@
+// common.cuh -- shared internals of libseastar.so (sm_100a).  Not part of the ABI.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string>
+
+#include "seastar.h"
+
+namespace seastar {
+
+// ----------------------------------------------------------------------------------------------
+// error plumbing: thread-local message + status codes, no exceptions across the ABI
+// ----------------------------------------------------------------------------------------------
+void set_error(const char* fmt, ...);
+seastar_status cuda_status(cudaError_t err, const char* where);
+seastar_status check_launch(const char* where);
+seastar_status check_device();   // sm_100 or UNSUPPORTED (cached per device)
+
+#define SS_ARG(cond, ...)                                   \
+    do {                                                    \
+        if (!(cond)) {                                      \
+            ::seastar::set_error(__VA_ARGS__);              \
+            return SEASTAR_ERR_INVALID_ARGUMENT;            \
+        }                                                   \
+    } while (0)
+
+#define SS_CUDA(call)                                                     \
+    do {                                                                  \
+        cudaError_t _e = (call);                                          \
+        if (_e != cudaSuccess) return ::seastar::cuda_status(_e, #call);  \
+    } while (0)
+
+#define SS_TRY(expr)                          \
+    do {                                      \
+        seastar_status _s = (expr);           \
+        if (_s != SEASTAR_OK) return _s;      \
+    } while (0)
+
+inline cudaStream_t to_stream(seastar_stream s) { return reinterpret_cast<cudaStream_t>(s); }
+
+// ----------------------------------------------------------------------------------------------
+// the graph handle (all index arrays are int32 on the device; E < 2^31 is validated at create)
+// ----------------------------------------------------------------------------------------------
+struct IndexSet {
+    int32_t* perm = nullptr;   // row -> vertex id            [n_rows]   (nullptr for LSF: identity)
+    int32_t* off = nullptr;    // row offsets                 [n_rows+1]
+    int32_t* nbr = nullptr;    // FWD: src id, REV: dst id     [n_edges]
+    int32_t* eid = nullptr;    // user edge id                 [n_edges]
+    int32_t* pos = nullptr;    // REV only: position in FWD (or LSF)
+    int32_t* type = nullptr;   // edge type or nullptr
+    float* norm = nullptr;     // R-GCN 1/c_{v,r} or nullptr
+    int64_t n_rows = 0;
+    int64_t n_edges = 0;
+    int64_t bucket_rows[SEASTAR_NUM_BUCKETS] = {0, 0, 0, 0};
+    int64_t max_deg = 0;
+};
+
+// Type-major view of the FWD edges for the R-GCN weight gradient: edges sorted by (type, dst row,
+// eid) and cut into (type, dst) runs; runs are grouped into tasks that never cross a type, so one
+// warp can own dW_r partials in registers (deterministic, no atomics).
+struct TypeMajor {
+    int32_t* src = nullptr;       // [Ef] source id per edge
+    int32_t* eid = nullptr;       // [Ef]
+    float* norm = nullptr;        // [Ef] or nullptr
+    int32_t* run_off = nullptr;   // [n_runs+1]
+    int32_t* run_dst = nullptr;   // [n_runs] destination vertex id
+    int32_t* task_run = nullptr;  // [n_tasks+1]
+    int32_t* task_type = nullptr; // [n_tasks]
+    int32_t* type_task = nullptr; // [R+1]
+    int64_t n_runs = 0, n_tasks = 0;
+};
+constexpr int kTaskEdges = 512;   // edges per dW task (a task may exceed it only inside one run)
+
+}  // namespace seastar
+
+struct seastar_graph_s {
+    int device = 0;
+    int64_t N = 0, E = 0, row_begin = 0, row_end = 0;
+    int32_t R = 1;
+    uint32_t flags = 0;
+    bool partitioned = false;
+    seastar::IndexSet fwd, rev, lsf;
+    seastar::TypeMajor tm;
+    int32_t* indeg_loc = nullptr;    // [n_loc]
+    int32_t* outdeg_loc = nullptr;   // [n_loc]
+    void* pool = nullptr;            // single device allocation backing every array above
+    size_t pool_bytes = 0;
+    int64_t n_loc() const { return row_end - row_begin; }
+};
+
+namespace seastar {
+
+constexpr int kBucketThreshold[SEASTAR_NUM_BUCKETS] = {1024, 32, 1, 0};
+
+// ----------------------------------------------------------------------------------------------
+// device helpers
+// ----------------------------------------------------------------------------------------------
+template <int VEC>
+struct Vec;
+template <>
+struct Vec<4> {
+    using T = float4;
+};
+template <>
+struct Vec<1> {
+    using T = float;
+};
+
+// read-only 128-bit / 32-bit loads through the non-coherent path
+__device__ __forceinline__ float4 ldg4(const float* p) { return __ldg(reinterpret_cast<const float4*>(p)); }
+__device__ __forceinline__ float ldg1(const float* p) { return __ldg(p); }
+
+template <int VEC>
+__device__ __forceinline__ void load_vec(const float* p, float (&v)[VEC]) {
+    if constexpr (VEC == 4) {
+        float4 t = ldg4(p);
+        v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+    } else {
+        v[0] = ldg1(p);
+    }
+}
+template <int VEC>
+__device__ __forceinline__ void store_vec(float* p, const float (&v)[VEC]) {
+    if constexpr (VEC == 4) {
+        *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+    } else {
+        p[0] = v[0];
+    }
+}
+
+// activation and its derivative expressed through the activation's output y
+__device__ __forceinline__ float act_apply(int act, float x) {
+    switch (act) {
+        case SEASTAR_ACT_RELU: return x > 0.f ? x : 0.f;
+        case SEASTAR_ACT_ELU: return x > 0.f ? x : expm1f(x);
+        case SEASTAR_ACT_SIGMOID: return 1.f / (1.f + expf(-x));
+        default: return x;
+    }
+}
+__device__ __forceinline__ float act_grad_from_y(int act, float y) {
+    switch (act) {
+        case SEASTAR_ACT_RELU: return y > 0.f ? 1.f : 0.f;
+        case SEASTAR_ACT_ELU: return y > 0.f ? 1.f : y + 1.f;
+        case SEASTAR_ACT_SIGMOID: return y * (1.f - y);
+        default: return 1.f;
+    }
+}
+
+inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+inline int num_sms() {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    return sms;
+}
+
+inline int pow2_ceil(int x) {
+    int p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+
+}  // namespace seastar

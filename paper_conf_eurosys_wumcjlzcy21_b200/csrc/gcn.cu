@@ -1,0 +1,244 @@
+// gcn.cu -- a5 / a8: fused GCN / APPNP aggregation, forward on the degree-sorted CSR and backward
+// on the degree-sorted reverse CSR (Fig. 1 L85-L93, Fig. 3, Alg. 1,
+// §6.3.2 "vertex-parallel edge-sequential", §6.3.4).
+//
+// B200 mapping (prior art: the paper's FAT groups, §6.3.1; not copied):
+//   * a row's features are split into L "chunk lanes" of VEC floats (128-bit loads when VEC = 4);
+//   * a row group of RL lanes (RL = 32: one warp per row; RL = L: several rows per warp for the
+//     low-degree bucket) owns one destination row; its S = RL / L edge slots walk the row's edges,
+//     RL edge ids at a time (one coalesced 32-bit load per lane, broadcast by shuffles), with UB
+//     gathers in flight per lane;
+//   * partial sums stay in registers and are merged by a fixed xor-shuffle tree: no atomics, no
+//     shared memory, bitwise deterministic;
+//   * rows are degree-sorted (hubs first, similar degrees share a warp), the grid is oversubscribed
+//     and the block scheduler's id order provides the dynamic load balance of §6.3.3 (L437-L453);
+//   * the epilogue (norm, APPNP mix, bias, activation, next-layer pre-scaling / activation
+//     derivative) is fused so each output row is written once.
+#include "common.cuh"
+
+namespace seastar {
+
+struct AggArgs {
+    const int32_t* perm;   // row -> vertex id
+    const int32_t* off;    // row offsets
+    const int32_t* nbr;    // neighbour ids per edge
+    int64_t row_begin;     // first row of this launch (bucket)
+    int64_t row_end;       // one past the last row of this launch
+    int64_t vbase;         // owned vertex base (row_begin of the partition)
+    const float* table;    // gathered rows [N, ld]
+    int64_t ld;
+    int F;
+    int bwd;               // 0: forward epilogue, 1: backward epilogue
+    const float* rscale;   // per-vertex scale [n_loc] (dst_norm fwd / src_norm bwd) or null
+    float gscale;          // global scale (1 fwd, APPNP (1-alpha) bwd)
+    // forward
+    const float* H0; float alpha; const float* bias; int act; float* Y; const float* out_scale; float* Ys;
+    // backward
+    const float* Yact; float* dA; const float* post_scale; float* dP;
+};
+
+template <int VEC, int L, int RL>
+__global__ void __launch_bounds__(256) k_aggregate(const AggArgs a) {
+    constexpr int S = RL / L;                    // edge slots per row group
+    constexpr int UB = (L < 4 ? L : 4);          // gathers in flight per lane per batch
+    const int lane = threadIdx.x & 31;
+    const int gl = lane % RL;                    // lane within the row group
+    const int slot = gl / L;
+    const int c = gl % L;
+    const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t row = a.row_begin + warp * (32 / RL) + lane / RL;
+    const bool valid = row < a.row_end;
+    const int beg = valid ? __ldg(a.off + row) : 0;
+    const int end = valid ? __ldg(a.off + row + 1) : 0;
+    const int64_t v = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;
+    const int C = (a.F + VEC - 1) / VEC;
+
+    for (int cb = 0; cb < C; cb += L) {
+        const int chunk = cb + c;
+        const bool active = chunk < C;
+        const int64_t col = (int64_t)chunk * VEC;
+        float acc[VEC];
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) acc[i] = 0.f;
+
+        for (int base = beg; base < end; base += RL) {
+            const int n = min(RL, end - base);
+            const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+#pragma unroll
+            for (int j0 = 0; j0 < L; j0 += UB) {
+                if (j0 * S >= n) break;
+                float val[UB][VEC];
+#pragma unroll
+                for (int jj = 0; jj < UB; ++jj) {
+                    const int k = (j0 + jj) * S + slot;
+                    const int u = __shfl_sync(gmask, my, k & (RL - 1), RL);
+                    if (k < n && active) {
+                        load_vec<VEC>(a.table + (int64_t)u * a.ld + col, val[jj]);
+                    } else {
+#pragma unroll
+                        for (int i = 0; i < VEC; ++i) val[jj][i] = 0.f;
+                    }
+                }
+#pragma unroll
+                for (int jj = 0; jj < UB; ++jj)
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) acc[i] += val[jj][i];
+            }
+        }
+        // merge the S edge slots (fixed tree)
+#pragma unroll
+        for (int o = L; o < RL; o <<= 1)
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) acc[i] += __shfl_xor_sync(gmask, acc[i], o, RL);
+
+        if (!valid || slot != 0 || !active) continue;
+        const float rs = (a.rscale ? __ldg(a.rscale + v) : 1.f) * a.gscale;
+        float out[VEC], out2[VEC];
+        if (!a.bwd) {
+            const float os = a.out_scale ? __ldg(a.out_scale + v) : 1.f;
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) {
+                float z = acc[i] * rs;
+                const int64_t cc = col + i;
+                if (cc < a.F) {
+                    if (a.H0) z = (1.f - a.alpha) * z + a.alpha * __ldg(a.H0 + v * a.ld + cc);
+                    if (a.bias) z += __ldg(a.bias + cc);
+                }
+                z = act_apply(a.act, z);
+                out[i] = z;
+                out2[i] = os * z;
+            }
+            float* y = a.Y + v * a.ld + col;
+            float* ys = a.Ys ? a.Ys + v * a.ld + col : nullptr;
+            if (col + VEC <= a.F) {
+                store_vec<VEC>(y, out);
+                if (ys) store_vec<VEC>(ys, out2);
+            } else {
+                for (int i = 0; i < VEC && col + i < a.F; ++i) {
+                    y[i] = out[i];
+                    if (ys) ys[i] = out2[i];
+                }
+            }
+        } else {
+            const float ps = a.post_scale ? __ldg(a.post_scale + v) : 1.f;
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) {
+                float g = acc[i] * rs;
+                if (a.Yact && col + i < a.F) g *= act_grad_from_y(a.act, __ldg(a.Yact + v * a.ld + col + i));
+                out[i] = g;
+                out2[i] = ps * g;
+            }
+            float* da = a.dA ? a.dA + v * a.ld + col : nullptr;
+            float* dp = a.dP ? a.dP + v * a.ld + col : nullptr;
+            if (col + VEC <= a.F) {
+                if (da) store_vec<VEC>(da, out);
+                if (dp) store_vec<VEC>(dp, out2);
+            } else {
+                for (int i = 0; i < VEC && col + i < a.F; ++i) {
+                    if (da) da[i] = out[i];
+                    if (dp) dp[i] = out2[i];
+                }
+            }
+        }
+    }
+}
+
+template <int VEC, int L>
+static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s) {
+    const int64_t rows = a.row_end - a.row_begin;
+    if (rows <= 0) return;
+    constexpr int threads = 256;
+    if (warp_rows) {
+        const int64_t blocks = (rows + (threads / 32) - 1) / (threads / 32);
+        k_aggregate<VEC, L, 32><<<(unsigned)blocks, threads, 0, s>>>(a);
+    } else {
+        constexpr int RL = L < 4 ? 4 : L;   // at least 4 lanes per row group keeps index loads useful
+        const int64_t per_block = threads / RL;
+        const int64_t blocks = (rows + per_block - 1) / per_block;
+        k_aggregate<VEC, L, RL><<<(unsigned)blocks, threads, 0, s>>>(a);
+    }
+}
+
+template <int VEC>
+static void launch_vec(AggArgs a, int L, bool warp_rows, cudaStream_t s) {
+    switch (L) {
+        case 1: launch_rl<VEC, 1>(a, warp_rows, s); break;
+        case 2: launch_rl<VEC, 2>(a, warp_rows, s); break;
+        case 4: launch_rl<VEC, 4>(a, warp_rows, s); break;
+        case 8: launch_rl<VEC, 8>(a, warp_rows, s); break;
+        case 16: launch_rl<VEC, 16>(a, warp_rows, s); break;
+        default: launch_rl<VEC, 32>(a, warp_rows, s); break;
+    }
+}
+
+// launch over the two degree classes of an index set: rows with degree >= 32 get a warp each,
+// the rest (incl. empty rows, which still need their epilogue) get sub-warp row groups
+seastar_status launch_aggregate(const IndexSet& x, AggArgs a, bool vec4, cudaStream_t s) {
+    const int VEC = vec4 ? 4 : 1;
+    const int C = (a.F + VEC - 1) / VEC;
+    const int L = C >= 32 ? 32 : pow2_ceil(C);
+    const int64_t split = x.bucket_rows[1];   // # rows with degree >= 32
+    a.perm = x.perm;
+    a.off = x.off;
+    a.nbr = x.nbr;
+    AggArgs hi = a, lo = a;
+    hi.row_begin = 0; hi.row_end = split;
+    lo.row_begin = split; lo.row_end = x.n_rows;
+    if (vec4) {
+        launch_vec<4>(hi, L, true, s);
+        launch_vec<4>(lo, L, L >= 32, s);
+    } else {
+        launch_vec<1>(hi, L, true, s);
+        launch_vec<1>(lo, L, L >= 32, s);
+    }
+    return check_launch("k_aggregate");
+}
+
+}  // namespace seastar
+
+using namespace seastar;
+
+extern "C" {
+
+seastar_status seastar_gcn_fwd(seastar_graph g, const float* T_all, int64_t F, int64_t ld, const float* dst_norm,
+                               const float* bias, seastar_act act, float alpha, const float* H0_loc, float* Y_loc,
+                               const float* out_scale, float* Ys_loc, seastar_stream stream) {
+    SS_ARG(g != nullptr, "gcn_fwd: graph is NULL");
+    SS_ARG(F >= 1 && ld >= F, "gcn_fwd: need 1 <= F <= ld (F=%lld, ld=%lld)", (long long)F, (long long)ld);
+    SS_ARG(T_all != nullptr && Y_loc != nullptr, "gcn_fwd: T_all and Y_loc are required");
+    SS_ARG(!Ys_loc || out_scale, "gcn_fwd: Ys_loc requires out_scale");
+    SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "gcn_fwd: bad activation %d", (int)act);
+    SS_ARG((void*)T_all != (void*)Y_loc, "gcn_fwd: output aliases the gathered table");
+    SS_TRY(check_device());
+    AggArgs a{};
+    a.vbase = g->row_begin;
+    a.table = T_all; a.ld = ld; a.F = (int)F; a.bwd = 0;
+    a.rscale = dst_norm; a.gscale = 1.f;
+    a.H0 = H0_loc; a.alpha = alpha; a.bias = bias; a.act = act; a.Y = Y_loc; a.out_scale = out_scale; a.Ys = Ys_loc;
+    bool vec4 = (ld % 4 == 0) && aligned16(T_all) && aligned16(Y_loc) && (!H0_loc || aligned16(H0_loc)) &&
+                (!Ys_loc || aligned16(Ys_loc));
+    return launch_aggregate(g->fwd, a, vec4, to_stream(stream));
+}
+
+seastar_status seastar_gcn_bwd(seastar_graph g, const float* dP_all, int64_t F, int64_t ld, const float* src_norm,
+                               float scale, const float* Yact_loc, seastar_act act, const float* post_scale,
+                               float* dA_loc, float* dP_loc, seastar_stream stream) {
+    SS_ARG(g != nullptr, "gcn_bwd: graph is NULL");
+    SS_ARG(F >= 1 && ld >= F, "gcn_bwd: need 1 <= F <= ld");
+    SS_ARG(dP_all != nullptr, "gcn_bwd: dP_all is NULL");
+    SS_ARG(dA_loc || dP_loc, "gcn_bwd: need dA_loc and/or dP_loc");
+    SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "gcn_bwd: bad activation %d", (int)act);
+    SS_ARG((void*)dP_all != (void*)dA_loc && (void*)dP_all != (void*)dP_loc, "gcn_bwd: output aliases the input");
+    SS_TRY(check_device());
+    AggArgs a{};
+    a.vbase = g->row_begin;
+    a.table = dP_all; a.ld = ld; a.F = (int)F; a.bwd = 1;
+    a.rscale = src_norm; a.gscale = scale;
+    a.Yact = Yact_loc; a.act = act; a.dA = dA_loc; a.post_scale = post_scale; a.dP = dP_loc;
+    bool vec4 = (ld % 4 == 0) && aligned16(dP_all) && (!dA_loc || aligned16(dA_loc)) && (!dP_loc || aligned16(dP_loc)) &&
+                (!Yact_loc || aligned16(Yact_loc));
+    return launch_aggregate(g->rev, a, vec4, to_stream(stream));
+}
+
+}  // extern "C"

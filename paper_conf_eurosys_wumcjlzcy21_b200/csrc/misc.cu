@@ -1,0 +1,189 @@
+// misc.cu -- training-step glue kept on the GPU so the whole epoch runs in this library:
+// softmax cross-entropy (mean over rows), deterministic column sums (bias gradients), axpby,
+// and a flat-buffer Adam step (DGL's default training loop).
+#include <math.h>
+
+#include "common.cuh"
+
+namespace seastar {
+
+static int64_t colsum_blocks(int64_t M) {
+    int64_t b = 2 * num_sms();
+    if (M < b * 32) b = (M + 31) / 32;
+    return b < 1 ? 1 : b;
+}
+
+size_t colsum_ws(int64_t M, int64_t F) { return (size_t)colsum_blocks(M) * (size_t)F * sizeof(float) + 256; }
+
+// stage 1: block b sums rows [b*rpb, (b+1)*rpb) of each column (8 row lanes x 32 columns, fixed order)
+__global__ void __launch_bounds__(256) k_colsum1(const float* __restrict__ X, int64_t M, int64_t F, int64_t ld,
+                                                 int64_t rpb, float* __restrict__ part) {
+    __shared__ float red[8][33];
+    const int64_t r0 = blockIdx.x * rpb, r1 = min(M, r0 + rpb);
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    for (int64_t cb = 0; cb < F; cb += 32) {
+        const int64_t j = cb + tx;
+        float s = 0.f;
+        if (j < F)
+            for (int64_t r = r0 + ty; r < r1; r += 8) s += __ldg(X + r * ld + j);
+        red[ty][tx] = s;
+        __syncthreads();
+        if (ty == 0 && j < F) {
+            float x = 0.f;
+            for (int k = 0; k < 8; ++k) x += red[k][tx];
+            part[blockIdx.x * F + j] = x;
+        }
+        __syncthreads();
+    }
+}
+
+__global__ void k_colsum2(const float* __restrict__ part, int64_t nblk, int64_t F, float* __restrict__ out) {
+    const int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (j >= F) return;
+    float x = 0.f;
+    for (int64_t b = 0; b < nblk; ++b) x += part[b * F + j];
+    out[j] = x;
+}
+
+seastar_status colsum_impl(const float* X, int64_t M, int64_t F, int64_t ld, float* out, void* ws, size_t ws_bytes,
+                           cudaStream_t s) {
+    if (ws_bytes < colsum_ws(M, F)) {
+        set_error("colsum: workspace too small");
+        return SEASTAR_ERR_INVALID_ARGUMENT;
+    }
+    if (F == 0) return SEASTAR_OK;
+    const int64_t nblk = colsum_blocks(M);
+    const int64_t rpb = M > 0 ? (M + nblk - 1) / nblk : 1;
+    float* part = static_cast<float*>(ws);
+    k_colsum1<<<(unsigned)nblk, 256, 0, s>>>(X, M, F, ld, rpb, part);
+    k_colsum2<<<(unsigned)((F + 255) / 256), 256, 0, s>>>(part, nblk, F, out);
+    return check_launch("k_colsum");
+}
+
+// warp per row: loss_r = lse(z_r) - z_r[label]; dZ = (softmax - onehot) / M; per-block loss partials
+__global__ void __launch_bounds__(256) k_softmax_xent(const float* __restrict__ Z, int64_t M, int C, int64_t ldz,
+                                                      const int64_t* __restrict__ labels, float* __restrict__ dZ,
+                                                      int64_t lddz, float* __restrict__ part) {
+    __shared__ float wl[8];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t r = blockIdx.x * 8 + w;
+    float loss = 0.f;
+    if (r < M) {
+        const float* z = Z + r * ldz;
+        float m = -INFINITY;
+        for (int c = lane; c < C; c += 32) m = fmaxf(m, __ldg(z + c));
+        for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        float sum = 0.f;
+        for (int c = lane; c < C; c += 32) sum += expf(__ldg(z + c) - m);
+        for (int o = 16; o; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+        const float lse = m + logf(sum);
+        const int64_t lab = labels[r];
+        const float inv = 1.f / (float)M;
+        if (dZ)
+            for (int c = lane; c < C; c += 32)
+                dZ[r * lddz + c] = (expf(__ldg(z + c) - lse) - (c == lab ? 1.f : 0.f)) * inv;
+        loss = lse - __ldg(z + lab);
+    }
+    if (lane == 0) wl[w] = loss;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        float x = 0.f;
+        for (int k = 0; k < 8; ++k) x += wl[k];
+        part[blockIdx.x] = x;
+    }
+}
+
+__global__ void k_loss_final(const float* __restrict__ part, int64_t n, int64_t M, float* __restrict__ loss) {
+    __shared__ double red[256];
+    double x = 0.0;
+    for (int64_t i = threadIdx.x; i < n; i += 256) x += (double)part[i];
+    red[threadIdx.x] = x;
+    __syncthreads();
+    for (int o = 128; o; o >>= 1) {
+        if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) *loss = (float)(red[0] / (double)M);
+}
+
+__global__ void k_axpby(int64_t n, float a, const float* __restrict__ x, float b, float* __restrict__ y) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < n) y[i] = a * x[i] + (b == 0.f ? 0.f : b * y[i]);
+}
+
+__global__ void k_adam(float* __restrict__ p, const float* __restrict__ g, float* __restrict__ m,
+                       float* __restrict__ v, int64_t n, float lr, float b1, float b2, float eps,
+                       const int32_t* __restrict__ step) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const int t = *step;
+    const float c1 = 1.f - powf(b1, (float)t), c2 = 1.f - powf(b2, (float)t);
+    const float gi = g[i];
+    const float mi = b1 * m[i] + (1.f - b1) * gi;
+    const float vi = b2 * v[i] + (1.f - b2) * gi * gi;
+    m[i] = mi;
+    v[i] = vi;
+    p[i] -= lr * (mi / c1) / (sqrtf(vi / c2) + eps);
+}
+
+__global__ void k_step_inc(int32_t* c) { *c += 1; }
+
+}  // namespace seastar
+
+using namespace seastar;
+
+extern "C" {
+
+size_t seastar_colsum_workspace(int64_t M, int64_t F) { return colsum_ws(M, F); }
+
+seastar_status seastar_colsum(const float* X, int64_t M, int64_t F, int64_t ld, float* out, void* workspace,
+                              size_t ws_bytes, seastar_stream stream) {
+    SS_ARG(X && out && workspace, "colsum: NULL argument");
+    SS_ARG(M >= 0 && F >= 1 && ld >= F, "colsum: bad sizes");
+    SS_TRY(check_device());
+    return colsum_impl(X, M, F, ld, out, workspace, ws_bytes, to_stream(stream));
+}
+
+size_t seastar_softmax_xent_workspace(int64_t M) { return (size_t)((M + 7) / 8 + 1) * sizeof(float) + 256; }
+
+seastar_status seastar_softmax_xent(const float* Z, int64_t M, int32_t C, int64_t ldz, const int64_t* labels,
+                                    float* loss, float* dZ, int64_t lddz, void* workspace, size_t ws_bytes,
+                                    seastar_stream stream) {
+    SS_ARG(Z && labels && loss && workspace, "softmax_xent: NULL argument");
+    SS_ARG(M >= 1 && C >= 1 && ldz >= C && (!dZ || lddz >= C), "softmax_xent: bad sizes");
+    SS_ARG(ws_bytes >= seastar_softmax_xent_workspace(M), "softmax_xent: workspace too small");
+    SS_TRY(check_device());
+    cudaStream_t s = to_stream(stream);
+    const int64_t nblk = (M + 7) / 8;
+    float* part = static_cast<float*>(workspace);
+    k_softmax_xent<<<(unsigned)nblk, 256, 0, s>>>(Z, M, C, ldz, labels, dZ, lddz, part);
+    k_loss_final<<<1, 256, 0, s>>>(part, nblk, M, loss);
+    return check_launch("k_softmax_xent");
+}
+
+seastar_status seastar_axpby(int64_t n, float a, const float* x, float b, float* y, seastar_stream stream) {
+    SS_ARG(x && y && n >= 0, "axpby: bad argument");
+    SS_TRY(check_device());
+    if (n == 0) return SEASTAR_OK;
+    k_axpby<<<(unsigned)((n + 255) / 256), 256, 0, to_stream(stream)>>>(n, a, x, b, y);
+    return check_launch("k_axpby");
+}
+
+seastar_status seastar_adam(float* param, const float* grad, float* m, float* v, int64_t n, float lr, float beta1,
+                            float beta2, float eps, const int32_t* step, seastar_stream stream) {
+    SS_ARG(param && grad && m && v && step && n >= 0, "adam: bad argument");
+    SS_TRY(check_device());
+    if (n == 0) return SEASTAR_OK;
+    k_adam<<<(unsigned)((n + 255) / 256), 256, 0, to_stream(stream)>>>(param, grad, m, v, n, lr, beta1, beta2, eps,
+                                                                        step);
+    return check_launch("k_adam");
+}
+
+seastar_status seastar_step_inc(int32_t* counter, seastar_stream stream) {
+    SS_ARG(counter, "step_inc: NULL");
+    SS_TRY(check_device());
+    k_step_inc<<<1, 1, 0, to_stream(stream)>>>(counter);
+    return check_launch("k_step_inc");
+}
+
+}  // extern "C"

@@ -1,0 +1,387 @@
+"""Whole training epochs of the paper's models, every step in libseastar.so kernels.
+
+PAPER.md §7 (L477-L481) trains GCN [37], GAT [58], APPNP [38] and R-GCN [53] with DGL's default
+configurations.  Each class below owns its buffers (allocated once, so an epoch launches kernels
+only -- capturable in a CUDA graph) and exposes ``epoch()`` = forward + softmax cross-entropy +
+backward + Adam, all through the C ABI.  PyTorch only allocates memory and, when the graph is
+row-partitioned over several GPUs, moves rows between ranks with NCCL collectives
+(``torch.distributed``): all-gather of the per-layer source rows, all-gather of the packed
+backward records, reduce-scatter of GAT's partial ``der``, and one all-reduce of the flat gradient
+buffer.
+
+Readings of the paper used here: dropout p = 0; ReLU hidden / identity output for
+GCN; ELU hidden (heads concatenated) / 1-head identity output for GAT; LeakyReLU slope 0.2; bias
+inside the activation; DGL "both" degree normalisation for GCN, in-degree^-1/2 for APPNP.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import _lib as L
+from .graph import Graph
+
+
+def _ld(F: int) -> int:
+    return (F + 3) // 4 * 4
+
+
+class Comm:
+    """Row-partition plumbing.  P = 1: every gather is the identity (no copies)."""
+
+    def __init__(self, world: int = 1, rank: int = 0, group=None):
+        self.world, self.rank, self.group = world, rank, group
+
+    def all_gather(self, out_all: torch.Tensor, loc: torch.Tensor):
+        if self.world == 1:
+            return loc
+        torch.distributed.all_gather_into_tensor(out_all, loc, group=self.group)
+        return out_all
+
+    def reduce_scatter(self, out_loc: torch.Tensor, part_all: torch.Tensor):
+        if self.world == 1:
+            return part_all
+        torch.distributed.reduce_scatter_tensor(out_loc, part_all, group=self.group)
+        return out_loc
+
+    def all_reduce(self, flat: torch.Tensor):
+        if self.world > 1:
+            torch.distributed.all_reduce(flat, group=self.group)
+
+
+class _Params:
+    """One flat fp32 buffer for parameters, gradients and Adam moments (one all-reduce, one Adam launch)."""
+
+    def __init__(self, shapes: dict, init: dict, device):
+        self.offsets = {}
+        n = 0
+        for k, s in shapes.items():
+            self.offsets[k] = (n, s)
+            n += int(np.prod(s))
+        self.n = n
+        self.flat = torch.zeros(n, device=device)
+        self.grad = torch.zeros(n, device=device)
+        self.m = torch.zeros(n, device=device)
+        self.v = torch.zeros(n, device=device)
+        self.step = torch.zeros(1, dtype=torch.int32, device=device)
+        for k, a in init.items():
+            self.p(k).copy_(torch.from_numpy(np.ascontiguousarray(a, np.float32)).reshape(self.offsets[k][1]))
+
+    def _view(self, buf, k):
+        o, s = self.offsets[k]
+        return buf[o:o + int(np.prod(s))].view(*s)
+
+    def p(self, k):
+        return self._view(self.flat, k)
+
+    def g(self, k):
+        return self._view(self.grad, k)
+
+    def adam(self, lr, b1=0.9, b2=0.999, eps=1e-8):
+        L.seastar_step_inc(self.step)
+        L.seastar_adam(self.flat, self.grad, self.m, self.v, self.n, lr, b1, b2, eps, self.step)
+
+
+class _Ws:
+    """Grow-only byte workspace shared by the deterministic reductions."""
+
+    def __init__(self, device):
+        self.device = device
+        self.buf = torch.empty(256, dtype=torch.uint8, device=device)
+
+    def need(self, nbytes: int) -> torch.Tensor:
+        if nbytes > self.buf.numel():
+            self.buf = torch.empty(nbytes, dtype=torch.uint8, device=self.device)
+        return self.buf
+
+
+class GCN2:
+    """2-layer GCN (Fig. 1 / Fig. 3): F_in -> hidden (ReLU) -> C (identity), softmax-xent.
+
+    Layer 1 transforms first (F_in > hidden), layer 2 aggregates first (hidden < C)
+    (reading #20).  The src-side norm is folded into the producing kernel's epilogue, the dst-side
+    norm, bias and activation into the aggregation's epilogue, and the activation derivative and
+    next-layer norm into the backward aggregation's epilogue."""
+
+    def __init__(self, g: Graph, X_loc: torch.Tensor, labels_loc: torch.Tensor, params: dict, lr=0.01,
+                 comm: Comm | None = None, n_pad_rows: int | None = None):
+        self.g, self.X, self.lab, self.lr = g, X_loc, labels_loc, lr
+        self.comm = comm or Comm()
+        dev = X_loc.device
+        self.n = g.n_loc
+        self.N = g.N
+        self.rows_all = n_pad_rows if n_pad_rows is not None else g.N      # all-gather height (P * n_per)
+        self.Fin = X_loc.shape[1]
+        self.H = params["W1"].shape[1]
+        self.C = params["W2"].shape[1]
+        self.P = _Params({"W1": params["W1"].shape, "b1": (self.H,), "W2": params["W2"].shape, "b2": (self.C,)},
+                         params, dev)
+        self.src_n, self.dst_n = g.degree_norms("both")
+        H, C, n = self.H, self.C, self.n
+        e = lambda r, c: torch.zeros((r, c), device=dev)
+        self.T1 = e(n, H)          # src_norm * (X W1), local rows
+        self.H1 = e(n, H)          # relu(dst_norm * sum T1 + b1)
+        self.H1s = e(n, H)         # src_norm * H1 (layer-2 table)
+        self.P2 = e(n, H)          # dst_norm * sum H1s
+        self.ldc = _ld(C)
+        self.logits = e(n, self.ldc)
+        self.dlogits = e(n, self.ldc)
+        self.dP2 = e(n, H)         # dst_norm * (dlogits W2^T)
+        self.dA1 = e(n, H)
+        self.dP1 = e(n, H)
+        self.dT1 = e(n, H)
+        self.loss = torch.zeros(1, device=dev)
+        self.ws = _Ws(dev)
+        P = self.comm.world
+        self.T1_all = e(self.rows_all, H) if P > 1 else None
+        self.H1s_all = e(self.rows_all, H) if P > 1 else None
+        self.dP2_all = e(self.rows_all, H) if P > 1 else None
+        self.dP1_all = e(self.rows_all, H) if P > 1 else None
+        self.timer = None
+
+    def _t(self, name):
+        if self.timer is not None:
+            self.timer(name)
+
+    def forward(self):
+        g, p, H, C, n = self.g, self.P, self.H, self.C, self.n
+        L.seastar_linear_fwd(self.X, n, self.Fin, self.X.stride(0), p.p("W1"), H, None, self.src_n, "none",
+                             self.T1, H)
+        T1_all = self.comm.all_gather(self.T1_all, self.T1)
+        self._t("gcn_fwd1")
+        L.seastar_gcn_fwd(g.handle, T1_all, H, H, self.dst_n, p.p("b1"), "relu", 0.0, None, self.H1, self.src_n,
+                          self.H1s)
+        self._t("gcn_fwd1_end")
+        H1s_all = self.comm.all_gather(self.H1s_all, self.H1s)
+        L.seastar_gcn_fwd(g.handle, H1s_all, H, H, self.dst_n, None, "none", 0.0, None, self.P2)
+        L.seastar_linear_fwd(self.P2, n, H, H, p.p("W2"), C, p.p("b2"), None, "none", self.logits, self.ldc)
+        ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
+        L.seastar_softmax_xent(self.logits, n, C, self.ldc, self.lab, self.loss, self.dlogits, self.ldc, ws,
+                               ws.numel())
+        return self.loss
+
+    def backward(self):
+        g, p, H, C, n = self.g, self.P, self.H, self.C, self.n
+        ws = self.ws.need(max(L.seastar_linear_bwd_weight_workspace(n, H, C),
+                              L.seastar_linear_bwd_weight_workspace(n, self.Fin, H),
+                              L.seastar_colsum_workspace(n, H)))
+        L.seastar_linear_bwd_weight(self.P2, n, H, H, self.dlogits, C, self.ldc, p.g("W2"), p.g("b2"), ws,
+                                    ws.numel())
+        L.seastar_linear_bwd_data(self.dlogits, n, C, self.ldc, p.p("W2"), H, self.dst_n, None, "none", self.dP2, H)
+        dP2_all = self.comm.all_gather(self.dP2_all, self.dP2)
+        self._t("gcn_bwd2")
+        L.seastar_gcn_bwd(g.handle, dP2_all, H, H, self.src_n, 1.0, self.H1, "relu", self.dst_n, self.dA1, self.dP1)
+        self._t("gcn_bwd2_end")
+        L.seastar_colsum(self.dA1, n, H, H, p.g("b1"), ws, ws.numel())
+        dP1_all = self.comm.all_gather(self.dP1_all, self.dP1)
+        L.seastar_gcn_bwd(g.handle, dP1_all, H, H, self.src_n, 1.0, None, "none", None, self.dT1, None)
+        L.seastar_linear_bwd_weight(self.X, n, self.Fin, self.X.stride(0), self.dT1, H, H, p.g("W1"), None, ws,
+                                    ws.numel())
+        self.comm.all_reduce(self.P.grad)
+
+    def epoch(self):
+        loss = self.forward()
+        self.backward()
+        self.P.adam(self.lr)
+        return loss
+
+
+class GAT2:
+    """2-layer GAT (Fig. 2 / Fig. 3): F_in -> heads x hidden (ELU, concat) -> 1 x C, softmax-xent.
+    LeakyReLU slope 0.2, attention vectors a_l (source) / a_r (destination) per head."""
+
+    def __init__(self, g: Graph, X_loc: torch.Tensor, labels_loc: torch.Tensor, params: dict, heads: int,
+                 hidden: int, lr=0.005, slope=0.2, comm: Comm | None = None, n_pad_rows: int | None = None):
+        self.g, self.X, self.lab, self.lr, self.slope = g, X_loc, labels_loc, lr, slope
+        self.comm = comm or Comm()
+        dev = X_loc.device
+        self.n, self.N = g.n_loc, g.N
+        self.rows_all = n_pad_rows if n_pad_rows is not None else g.N
+        self.Fin = X_loc.shape[1]
+        self.H1, self.F1 = heads, hidden
+        self.W1w = heads * hidden
+        self.C = params["W2"].shape[1]
+        shapes = {"W1": (self.Fin, self.W1w), "al1": (heads, hidden), "ar1": (heads, hidden), "b1": (self.W1w,),
+                  "W2": (self.W1w, self.C), "al2": (1, self.C), "ar2": (1, self.C), "b2": (self.C,)}
+        self.P = _Params(shapes, params, dev)
+        n, W1w, C = self.n, self.W1w, self.C
+        self.ld1, self.ld2 = _ld(W1w), _ld(C)
+        e = lambda r, c: torch.zeros((r, c), device=dev)
+        self.T1, self.A1, self.Y1 = e(n, self.ld1), e(n, self.ld1), e(n, self.ld1)
+        self.el1, self.er1, self.lse1 = e(n, heads), e(n, heads), e(n, heads)
+        self.T2, self.A2, self.Y2 = e(n, self.ld2), e(n, self.ld2), e(n, self.ld2)
+        self.el2, self.er2, self.lse2 = e(n, 1), e(n, 1), e(n, 1)
+        self.dY2 = e(n, self.ld2)
+        self.ldd1, self.ldd2 = L.seastar_gat_record_ld(heads, hidden), L.seastar_gat_record_ld(1, C)
+        self.D1, self.D2 = e(n, self.ldd1), e(n, self.ldd2)
+        self.dT1, self.dT2 = e(n, self.ld1), e(n, self.ld2)
+        self.del1, self.del2 = e(n, heads), e(n, 1)
+        self.der1, self.der2 = e(self.rows_all if self.comm.world > 1 else n, heads), \
+            e(self.rows_all if self.comm.world > 1 else n, 1)
+        self.der1_loc, self.der2_loc = (e(n, heads), e(n, 1)) if self.comm.world > 1 else (self.der1, self.der2)
+        n_ds = g.info["num_rev_edges"]
+        self.ds1 = torch.zeros((max(n_ds, 1), heads), device=dev)
+        self.ds2 = torch.zeros((max(n_ds, 1), 1), device=dev)
+        self.dY1 = e(n, self.ld1)
+        self.loss = torch.zeros(1, device=dev)
+        self.ws = _Ws(dev)
+        P = self.comm.world
+        R = self.rows_all
+        self.T1_all = e(R, self.ld1) if P > 1 else None
+        self.el1_all = e(R, heads) if P > 1 else None
+        self.T2_all = e(R, self.ld2) if P > 1 else None
+        self.el2_all = e(R, 1) if P > 1 else None
+        self.D1_all = e(R, self.ldd1) if P > 1 else None
+        self.D2_all = e(R, self.ldd2) if P > 1 else None
+        self.timer = None
+
+    def _t(self, name):
+        if self.timer is not None:
+            self.timer(name)
+
+    def forward(self):
+        g, p, n = self.g, self.P, self.n
+        H, F, W, C = self.H1, self.F1, self.W1w, self.C
+        L.seastar_linear_fwd(self.X, n, self.Fin, self.X.stride(0), p.p("W1"), W, None, None, "none", self.T1,
+                             self.ld1)
+        L.seastar_gat_attn_proj(self.T1, n, H, F, self.ld1, p.p("al1"), p.p("ar1"), self.el1, self.er1)
+        T1_all = self.comm.all_gather(self.T1_all, self.T1)
+        el1_all = self.comm.all_gather(self.el1_all, self.el1)
+        self._t("gat_fwd1")
+        L.seastar_gat_fwd(g.handle, T1_all, el1_all, self.er1, H, F, self.ld1, self.slope, p.p("b1"), "elu", self.A1,
+                          self.Y1, self.lse1)
+        self._t("gat_fwd1_end")
+        L.seastar_linear_fwd(self.Y1, n, W, self.ld1, p.p("W2"), C, None, None, "none", self.T2, self.ld2)
+        L.seastar_gat_attn_proj(self.T2, n, 1, C, self.ld2, p.p("al2"), p.p("ar2"), self.el2, self.er2)
+        T2_all = self.comm.all_gather(self.T2_all, self.T2)
+        el2_all = self.comm.all_gather(self.el2_all, self.el2)
+        L.seastar_gat_fwd(g.handle, T2_all, el2_all, self.er2, 1, C, self.ld2, self.slope, p.p("b2"), "none", self.A2,
+                          self.Y2, self.lse2)
+        ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
+        L.seastar_softmax_xent(self.Y2, n, C, self.ld2, self.lab, self.loss, self.dY2, self.ld2, ws, ws.numel())
+        return self.loss
+
+    def _layer_bwd(self, T, T_loc_ld, el, er, A, Y, lse, dY, act, H, F, D, D_all_buf, dT, del_, der, der_loc, ds,
+                   al, ar, dal, dar, db, tag):
+        g, n = self.g, self.n
+        L.seastar_gat_bwd_prep(g.handle, dY, Y, act, A, er, lse, H, F, T_loc_ld, D)
+        ldd = L.seastar_gat_record_ld(H, F)
+        ws = self.ws.need(max(L.seastar_colsum_workspace(n, H * F), L.seastar_gat_attn_proj_bwd_workspace(n, H, F)))
+        L.seastar_colsum(D, n, H * F, ldd, db, ws, ws.numel())       # db = sum_v dA[v] (dA = first H*F columns)
+        D_all = self.comm.all_gather(D_all_buf, D)
+        self._t(f"gat_bwd{tag}")
+        L.seastar_gat_bwd(g.handle, T, el, D_all, H, F, T_loc_ld, self.slope, dT, del_, ds)
+        self._t(f"gat_bwd{tag}_end")
+        L.seastar_gat_der(g.handle, ds, H, der)
+        der_l = self.comm.reduce_scatter(der_loc, der)
+        L.seastar_gat_attn_proj_bwd(T, n, H, F, T_loc_ld, al, ar, del_, der_l, dT, dal, dar, ws, ws.numel())
+
+    def backward(self):
+        p, n = self.P, self.n
+        H, F, W, C = self.H1, self.F1, self.W1w, self.C
+        self._layer_bwd(self.T2, self.ld2, self.el2, self.er2, self.A2, self.Y2, self.lse2, self.dY2, "none", 1, C,
+                        self.D2, self.D2_all, self.dT2, self.del2, self.der2, self.der2_loc, self.ds2, p.p("al2"),
+                        p.p("ar2"), p.g("al2"), p.g("ar2"), p.g("b2"), "2")
+        ws = self.ws.need(max(L.seastar_linear_bwd_weight_workspace(n, W, C),
+                              L.seastar_linear_bwd_weight_workspace(n, self.Fin, W)))
+        L.seastar_linear_bwd_weight(self.Y1, n, W, self.ld1, self.dT2, C, self.ld2, p.g("W2"), None, ws, ws.numel())
+        L.seastar_linear_bwd_data(self.dT2, n, C, self.ld2, p.p("W2"), W, None, None, "none", self.dY1, self.ld1)
+        self._layer_bwd(self.T1, self.ld1, self.el1, self.er1, self.A1, self.Y1, self.lse1, self.dY1, "elu", H, F,
+                        self.D1, self.D1_all, self.dT1, self.del1, self.der1, self.der1_loc, self.ds1, p.p("al1"),
+                        p.p("ar1"), p.g("al1"), p.g("ar1"), p.g("b1"), "1")
+        ws = self.ws.need(L.seastar_linear_bwd_weight_workspace(n, self.Fin, W))
+        L.seastar_linear_bwd_weight(self.X, n, self.Fin, self.X.stride(0), self.dT1, W, self.ld1, p.g("W1"), None, ws,
+                                    ws.numel())
+        self.comm.all_reduce(self.P.grad)
+
+    def epoch(self):
+        loss = self.forward()
+        self.backward()
+        self.P.adam(self.lr)
+        return loss
+
+
+class APPNPNet:
+    """APPNP [38]: H0 = MLP(X) (Linear -> ReLU -> Linear), K steps Z <- (1-a) n A n Z + a H0, softmax-xent.
+    Each propagation step is one fused gcn_fwd (APPNP epilogue, writes Z and n*Z for the next step)."""
+
+    def __init__(self, g: Graph, X_loc, labels_loc, params: dict, K=10, alpha=0.1, lr=0.01, comm: Comm | None = None,
+                 n_pad_rows: int | None = None):
+        self.g, self.X, self.lab, self.K, self.alpha, self.lr = g, X_loc, labels_loc, K, alpha, lr
+        self.comm = comm or Comm()
+        dev = X_loc.device
+        self.n = g.n_loc
+        self.rows_all = n_pad_rows if n_pad_rows is not None else g.N
+        self.Fin = X_loc.shape[1]
+        self.Hd = params["W1"].shape[1]
+        self.C = params["W2"].shape[1]
+        self.P = _Params({"W1": params["W1"].shape, "b1": (self.Hd,), "W2": params["W2"].shape, "b2": (self.C,)},
+                         params, dev)
+        _, self.nrm = g.degree_norms("in")
+        n, Hd, C = self.n, self.Hd, self.C
+        self.ldc = _ld(C)
+        e = lambda r, c: torch.zeros((r, c), device=dev)
+        self.Hh = e(n, Hd)
+        self.H0 = e(n, self.ldc)
+        self.Z = [e(n, self.ldc) for _ in range(K + 1)]       # Z[0] aliases H0's values (copied by linear)
+        self.Zs = [e(n, self.ldc) for _ in range(K + 1)]      # n * Z[k]
+        self.G = e(n, self.ldc)
+        self.Gs = [e(n, self.ldc), e(n, self.ldc)]
+        self.Gtmp = e(n, self.ldc)
+        self.dH0 = e(n, self.ldc)
+        self.dHh = e(n, Hd)
+        self.loss = torch.zeros(1, device=dev)
+        self.ws = _Ws(dev)
+        P = self.comm.world
+        self.Zs_all = e(self.rows_all, self.ldc) if P > 1 else None
+        self.Gs_all = e(self.rows_all, self.ldc) if P > 1 else None
+
+    def forward(self):
+        g, p, n, Hd, C, ld = self.g, self.P, self.n, self.Hd, self.C, self.ldc
+        L.seastar_linear_fwd(self.X, n, self.Fin, self.X.stride(0), p.p("W1"), Hd, p.p("b1"), None, "relu", self.Hh,
+                             Hd)
+        L.seastar_linear_fwd(self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), None, "none", self.H0, ld)
+        L.seastar_linear_fwd(self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), self.nrm, "none", self.Zs[0], ld)
+        for k in range(self.K):
+            Zs_all = self.comm.all_gather(self.Zs_all, self.Zs[k])
+            L.seastar_gcn_fwd(g.handle, Zs_all, C, ld, self.nrm, None, "none", self.alpha, self.H0, self.Z[k + 1],
+                              self.nrm, self.Zs[k + 1])
+        out = self.Z[self.K] if self.K > 0 else self.H0
+        ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
+        L.seastar_softmax_xent(out, n, C, ld, self.lab, self.loss, self.G, ld, ws, ws.numel())
+        return self.loss
+
+    def backward(self):
+        g, p, n, Hd, C, ld, a = self.g, self.P, self.n, self.Hd, self.C, self.ldc, self.alpha
+        # G = dL/dZ^K ; for k = K-1..0: dH0 += a G ; G <- (1-a) n sum_out n G
+        self.dH0.zero_()
+        L.seastar_linear_fwd(self.G, n, C, ld, self._eye(C), C, None, self.nrm, "none", self.Gs[0], ld) \
+            if self.K > 0 else None
+        cur = 0
+        G = self.G
+        for k in range(self.K):
+            L.seastar_axpby(n * ld, a, G, 1.0, self.dH0)
+            Gs_all = self.comm.all_gather(self.Gs_all, self.Gs[cur])
+            nxt = self.Gtmp if G is self.G else self.G
+            L.seastar_gcn_bwd(g.handle, Gs_all, C, ld, self.nrm, 1.0 - a, None, "none", self.nrm, nxt, self.Gs[1 - cur])
+            G = nxt
+            cur = 1 - cur
+        L.seastar_axpby(n * ld, 1.0, G, 1.0, self.dH0)
+        ws = self.ws.need(max(L.seastar_linear_bwd_weight_workspace(n, Hd, C),
+                              L.seastar_linear_bwd_weight_workspace(n, self.Fin, Hd)))
+        L.seastar_linear_bwd_weight(self.Hh, n, Hd, Hd, self.dH0, C, ld, p.g("W2"), p.g("b2"), ws, ws.numel())
+        L.seastar_linear_bwd_data(self.dH0, n, C, ld, p.p("W2"), Hd, None, self.Hh, "relu", self.dHh, Hd)
+        L.seastar_linear_bwd_weight(self.X, n, self.Fin, self.X.stride(0), self.dHh, Hd, Hd, p.g("W1"), p.g("b1"), ws,
+                                    ws.numel())
+        self.comm.all_reduce(self.P.grad)
+
+    def _eye(self, C):
+        if not hasattr(self, "_I") or self._I.shape[0] != C:
+            self._I = torch.eye(C, device=self.X.device)
+        return self._I
+
+    def epoch(self):
+        loss = self.forward()
+        self.backward()
+        self.P.adam(self.lr)
+        return loss

@@ -1,0 +1,104 @@
+"""a4 / a11 and the training glue on the GPU vs the oracle: dense transform fwd/bwd, softmax
+cross-entropy, column sums, Adam."""
+import numpy as np
+import pytest
+
+import oracle
+from conftest import rel_err
+from helpers import padded, rnd
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-5
+
+
+@pytest.fixture(scope="module")
+def env():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
+    return dict(torch=torch, L=L)
+
+
+def dev(env, a):
+    return env["torch"].from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+SHAPES = [(1, 1, 1), (5, 3, 7), (1000, 602, 16), (3001, 64, 41), (777, 1433, 16), (2000, 70, 64), (513, 16, 70),
+          (300, 8710, 8)]
+
+
+@pytest.mark.parametrize("M,K,N", SHAPES)
+def test_linear_fwd(env, M, K, N):
+    torch, L = env["torch"], env["L"]
+    X, W, b = rnd(1, (M, K)), rnd(2, (K, N)), rnd(3, (N,))
+    rs = rnd(4, (M,), 0.5, 2.0)
+    ldx = K + 3
+    ldy = N + 5
+    Y = torch.full((M, ldy), float("nan"), device="cuda")
+    L.seastar_linear_fwd(dev(env, padded(X, ldx)), M, K, ldx, dev(env, W), N, dev(env, b), dev(env, rs), "relu",
+                         Y, ldy)
+    ref = oracle.act_fwd("relu", oracle.linear_fwd(X, W, b)) * rs.astype(np.float64)[:, None]
+    assert rel_err(Y.cpu().numpy()[:, :N], ref) <= TOL
+    assert np.isnan(Y.cpu().numpy()[:, N:]).all()
+
+
+@pytest.mark.parametrize("M,K,N", SHAPES)
+def test_linear_bwd(env, M, K, N):
+    torch, L = env["torch"], env["L"]
+    if N > 64:
+        pytest.skip("bwd_weight supports Nout <= 64")
+    X, W, dY = rnd(5, (M, K)), rnd(6, (K, N)), rnd(7, (M, N))
+    rs = rnd(8, (M,), 0.5, 2.0)
+    dX = torch.empty((M, K), device="cuda")
+    Z = rnd(9, (M, K)).astype(np.float64)
+    Yact = oracle.act_fwd("elu", Z).astype(np.float32)
+    L.seastar_linear_bwd_data(dev(env, dY), M, N, N, dev(env, W), K, dev(env, rs), dev(env, Yact), "elu", dX, K)
+    rdX, rdW, rdb = oracle.linear_bwd(X, W, dY)
+    assert rel_err(dX.cpu().numpy(), oracle.act_bwd("elu", Z, rdX * rs.astype(np.float64)[:, None])) <= TOL
+    ws_b = L.seastar_linear_bwd_weight_workspace(M, K, N)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dW = torch.empty((K, N), device="cuda")
+    db = torch.empty((N,), device="cuda")
+    L.seastar_linear_bwd_weight(dev(env, X), M, K, K, dev(env, dY), N, N, dW, db, ws, ws_b)
+    assert rel_err(dW.cpu().numpy(), rdW) <= TOL
+    assert rel_err(db.cpu().numpy(), rdb) <= TOL
+
+
+@pytest.mark.parametrize("M,C", [(1, 1), (100, 7), (5000, 41), (3000, 70)])
+def test_softmax_xent(env, M, C):
+    torch, L = env["torch"], env["L"]
+    Z = rnd(9, (M, C), -3, 3)
+    lab = (rnd(10, (M,), 0, 1).astype(np.float64) * C).astype(np.int64).clip(0, C - 1)
+    ws_b = L.seastar_softmax_xent_workspace(M)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    loss = torch.empty((1,), device="cuda")
+    dZ = torch.empty((M, C), device="cuda")
+    L.seastar_softmax_xent(dev(env, Z), M, C, C, dev(env, lab), loss, dZ, C, ws, ws_b)
+    rl, rd = oracle.softmax_xent(Z, lab)
+    assert abs(loss.item() - rl) <= TOL * abs(rl)
+    assert rel_err(dZ.cpu().numpy(), rd) <= TOL
+
+
+def test_colsum_axpby_adam(env):
+    torch, L = env["torch"], env["L"]
+    M, F = 12345, 37
+    X = rnd(11, (M, F))
+    ws_b = L.seastar_colsum_workspace(M, F)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    out = torch.empty((F,), device="cuda")
+    L.seastar_colsum(dev(env, padded(X, 40)), M, F, 40, out, ws, ws_b)
+    assert rel_err(out.cpu().numpy(), X.astype(np.float64).sum(0)) <= TOL
+    x, y = rnd(12, (1000,)), rnd(13, (1000,))
+    yd = dev(env, y.copy())
+    L.seastar_axpby(1000, 0.5, dev(env, x), -2.0, yd)
+    assert rel_err(yd.cpu().numpy(), 0.5 * x.astype(np.float64) - 2.0 * y) <= TOL
+    n = 4097
+    p, g = rnd(14, (n,)), rnd(15, (n,))
+    pd, md, vd = dev(env, p.copy()), torch.zeros(n, device="cuda"), torch.zeros(n, device="cuda")
+    step = torch.zeros(1, dtype=torch.int32, device="cuda")
+    pr, mr, vr = p.astype(np.float64), np.zeros(n), np.zeros(n)
+    for t in (1, 2, 3):
+        L.seastar_step_inc(step)
+        L.seastar_adam(pd, dev(env, g), md, vd, n, 0.01, 0.9, 0.999, 1e-8, step)
+        oracle.adam(pr, g, mr, vr, 0.01, t)
+    assert rel_err(pd.cpu().numpy() - p, pr - p) <= 1e-4   # update magnitude ~lr; compare the deltas

@@ -346,3 +346,26 @@ def test_adam_closed_form():
     # second step with the same gradient: m_hat = g, v_hat = g^2 again
     oracle.adam(p, g, m, v, lr=0.01, t=2)
     np.testing.assert_allclose(p, -0.02 * g / (np.abs(g) + 1e-8), rtol=1e-12)
+
+
+def test_marshalling_independent_of_input_dtype():
+    """fp32 / int32 inputs are converted by the wrapper; results must equal the fp64 inputs' (guards
+    against passing pointers to temporaries across the C call)."""
+    indptr, indices = small_graph(4, N=40, E=300)
+    H = rnd(1, 40, 6)
+    sn, dn = rnd(2, 40), rnd(3, 40)
+    ref = oracle.gcn_aggregate(indptr, indices, H, sn, dn)
+    import gc
+    for _ in range(3):
+        got = oracle.gcn_aggregate(indptr.astype(np.int32), indices.astype(np.int32), H.astype(np.float32),
+                                   sn.astype(np.float32), dn.astype(np.float32))
+        gc.collect()
+        ref32 = np.diag(dn.astype(np.float32).astype(np.float64)) @ dense_adj(indptr, indices) @ \
+            np.diag(sn.astype(np.float32).astype(np.float64)) @ H.astype(np.float32).astype(np.float64)
+        assert rel_err(got, ref32) < 1e-13
+        gotT = oracle.gcn_aggregate_T(indptr, indices, H.astype(np.float32), sn.astype(np.float32),
+                                      dn.astype(np.float32))
+        assert rel_err(gotT, oracle.gcn_aggregate_T(indptr, indices, H.astype(np.float32).astype(np.float64),
+                                                    sn.astype(np.float32).astype(np.float64),
+                                                    dn.astype(np.float32).astype(np.float64))) == 0.0
+    assert rel_err(ref, ref) == 0.0
