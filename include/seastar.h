@@ -265,13 +265,18 @@ seastar_status seastar_rgcn_fwd(seastar_graph g, const float* X_all, int64_t F_i
                                 int64_t F_out, const float* norm_user, const float* bias, seastar_act act,
                                 float* Y_loc, int64_t ldy, seastar_stream stream);
 /*
- * Backward on the type-sorted reverse CSR, for owned sources u and each type run r of out(u):
- *   q = sum_{e in run} norm_e dA_all[dst(e),:];  dX_loc[u] += q W[r]^T ;  dW[r] += X_loc[u]^T q.
- *   dA_all [N,F_out] ld ldd ; X_loc [n_loc,F_in] ld ldx ; dX_loc [n_loc,F_in] ld ldx or NULL ;
- *   dW [R,F_in,F_out] or NULL (overwritten; this rank's partial when partitioned).
+ * Backward of seastar_rgcn_fwd's pre-activation output given dA = dL/d(pre-activation):
+ *   dX_loc[u] = sum_{type runs r of out(u)} (sum_{e in run} norm_e dA_all[dst(e),:]) W[r]^T
+ *     -- source-major over the type-sorted reverse CSR (§6.3.4 L461 + §6.3.5);
+ *   dW[r] = sum_{owned v} g_{v,r}^T dA_all[v,:],  g_{v,r} = sum_{e in in(v), type r} norm_e X_all[src(e),:]
+ *     -- over a type-major view of the forward edges built at graph_create; one warp owns a dW_r
+ *     partial in registers per task, partials are reduced per type in task order (deterministic).
+ *   X_all [N,F_in] ld ldx (the forward's gathered input) ; dA_all [N,F_out] ld ldd (gathered) ;
+ *   dX_loc [n_loc,F_in] ld ldx or NULL ; dW [R,F_in,F_out] or NULL (overwritten; this rank's partial
+ *   when partitioned).  ldx, ldd multiples of 4; F_in*F_out <= 1024.
  *   workspace: seastar_rgcn_bwd_workspace() bytes (dev).
  */
-seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_loc, int64_t F_in, int64_t ldx,
+seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_in, int64_t ldx,
                                 const float* dA_all, int64_t F_out, int64_t ldd, const float* W,
                                 const float* norm_user, float* dX_loc, float* dW, void* workspace,
                                 size_t ws_bytes, seastar_stream stream);

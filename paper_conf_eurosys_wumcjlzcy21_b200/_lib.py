@@ -283,9 +283,9 @@ def seastar_rgcn_bwd_workspace(g, F_in, F_out) -> int:
     return int(load().seastar_rgcn_bwd_workspace(g, F_in, F_out))
 
 
-def seastar_rgcn_bwd(g, X_loc, F_in, ldx, dA_all, F_out, ldd, W, norm_user, dX_loc, dW, workspace, ws_bytes,
+def seastar_rgcn_bwd(g, X_all, F_in, ldx, dA_all, F_out, ldd, W, norm_user, dX_loc, dW, workspace, ws_bytes,
                      stream=None) -> None:
-    _call("seastar_rgcn_bwd", g, _dptr(X_loc, "X"), F_in, ldx, _dptr(dA_all, "dA"), F_out, ldd, _dptr(W, "W"),
+    _call("seastar_rgcn_bwd", g, _dptr(X_all, "X"), F_in, ldx, _dptr(dA_all, "dA"), F_out, ldd, _dptr(W, "W"),
           _dptr(norm_user, "norm"), _dptr(dX_loc, "dX"), _dptr(dW, "dW"), _dptr(workspace, "workspace"), ws_bytes,
           _stream(stream))
 

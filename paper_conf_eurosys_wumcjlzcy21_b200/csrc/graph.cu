@@ -248,6 +248,78 @@ __global__ void k_degree_norms(int64_t n, const int32_t* __restrict__ indeg, con
     if (src_norm) src_norm[i] = mode == SEASTAR_NORM_IN ? ni : 1.0f / sqrtf((float)dout);
 }
 
+// ---- type-major view (R-GCN dW): edges by (type, fwd row, eid), cut into runs and tasks --------
+__global__ void k_row_index(int64_t n, const int32_t* __restrict__ off, int32_t* __restrict__ rowidx) {
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    for (int64_t k = warp; k < n; k += ((int64_t)gridDim.x * blockDim.x) >> 5)
+        for (int64_t p = off[k] + lane; p < off[k + 1]; p += 32) rowidx[p] = (int32_t)k;
+}
+__global__ void k_tm_keys(int64_t n, const int32_t* __restrict__ rowidx, const int32_t* __restrict__ typ, int rbits,
+                          uint64_t* __restrict__ key) {
+    const int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (p < n) key[p] = ((uint64_t)typ[p] << rbits) | (uint64_t)rowidx[p];
+}
+__global__ void k_tm_fill(int64_t n, const int32_t* __restrict__ pos, const int32_t* __restrict__ src,
+                          const int32_t* __restrict__ eid, const float* __restrict__ norm, int32_t* __restrict__ tsrc,
+                          int32_t* __restrict__ teid, float* __restrict__ tnorm) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const int32_t p = pos[i];
+    tsrc[i] = src[p];
+    teid[i] = eid[p];
+    if (tnorm) tnorm[i] = norm[p];
+}
+__global__ void k_tm_run_heads(int64_t n, const uint64_t* __restrict__ key, int32_t* __restrict__ head) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < n) head[i] = (i == 0 || key[i] != key[i - 1]) ? 1 : 0;
+}
+// runs: run r starts at the r-th head; meta[0] = #runs
+__global__ void k_tm_runs(int64_t n, const uint64_t* __restrict__ key, const int32_t* __restrict__ head,
+                          const int32_t* __restrict__ rid, int rbits, const int32_t* __restrict__ perm,
+                          int32_t* __restrict__ run_off, int32_t* __restrict__ run_dst, int32_t* __restrict__ run_type,
+                          long long* __restrict__ meta) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    if (head[i]) {
+        const int32_t r = rid[i] - 1;
+        const uint64_t k = key[i];
+        run_off[r] = (int32_t)i;
+        run_dst[r] = perm[k & ((1ull << rbits) - 1)];
+        run_type[r] = (int32_t)(k >> rbits);
+    }
+    if (i == n - 1) {
+        run_off[rid[i]] = (int32_t)n;
+        meta[0] = rid[i];
+    }
+}
+// a task starts at run 0, at every type change, and whenever a run starts in a new kTaskEdges block
+__global__ void k_tm_task_heads(int64_t bound, const long long* __restrict__ meta, const int32_t* __restrict__ run_off,
+                                const int32_t* __restrict__ run_type, int ke, int32_t* __restrict__ thead) {
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (r >= bound) return;
+    const int64_t nr = meta[0];
+    if (r >= nr) { thead[r] = 0; return; }
+    thead[r] = (r == 0 || run_type[r] != run_type[r - 1] || run_off[r] / ke != run_off[r - 1] / ke) ? 1 : 0;
+}
+__global__ void k_tm_tasks(int64_t bound, long long* __restrict__ meta, const int32_t* __restrict__ thead,
+                           const int32_t* __restrict__ tid, const int32_t* __restrict__ run_type,
+                           int32_t* __restrict__ task_run, int32_t* __restrict__ task_type, int32_t* __restrict__ cnt) {
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t nr = meta[0];
+    if (r >= bound || r >= nr) return;
+    if (thead[r]) {
+        const int32_t t = tid[r] - 1;
+        task_run[t] = (int32_t)r;
+        task_type[t] = run_type[r];
+        atomicAdd(&cnt[run_type[r]], 1);   // integer count per type: order-independent
+    }
+    if (r == nr - 1) {
+        task_run[tid[r]] = (int32_t)nr;
+        meta[1] = tid[r];
+    }
+}
+
 // ----------------------------------------------------------------------------------------------
 // host helpers
 // ----------------------------------------------------------------------------------------------
@@ -294,6 +366,15 @@ static seastar_status exclusive_sum(Temps& t, const int32_t* in, int32_t* out, i
     void* tmp = nullptr;
     SS_CUDA(t.alloc(reinterpret_cast<char**>(&tmp), bytes));
     SS_CUDA(cub::DeviceScan::ExclusiveSum(tmp, bytes, in, out, (int)n, t.s));
+    return SEASTAR_OK;
+}
+
+static seastar_status inclusive_sum(Temps& t, const int32_t* in, int32_t* out, int64_t n) {
+    size_t bytes = 0;
+    SS_CUDA(cub::DeviceScan::InclusiveSum(nullptr, bytes, in, out, (int)n, t.s));
+    void* tmp = nullptr;
+    SS_CUDA(t.alloc(reinterpret_cast<char**>(&tmp), bytes));
+    SS_CUDA(cub::DeviceScan::InclusiveSum(tmp, bytes, in, out, (int)n, t.s));
     return SEASTAR_OK;
 }
 

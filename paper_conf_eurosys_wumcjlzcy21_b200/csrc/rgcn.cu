@@ -1,5 +1,289 @@
-// rgcn.cu -- a7 / a10: R-GCN (§6.3.5).  Placeholder until the fused kernels land.
+// rgcn.cu -- a7 / a10: fused R-GCN layer (§6.3.5, layer of [53]).
+//
+// "Heterogeneous Seastar": the aggregation is hierarchical -- sum over the edges of one type, then
+// over types -- and the paper runs it sequentially by sorting each vertex's edges by type and
+// "detecting changes of edge types" (L473-L475).  On B200:
+//   forward (dst-major, FWD CSR, type-sorted rows): every edge slot keeps a run-sum g of
+//     norm_e * X[src_e] in registers; when its type changes, g is pushed through W_r, which is staged
+//     once per CTA in shared memory (R x F_in x F_out fp32, <= 200 KB), and accumulated into the
+//     row's output; the slots are merged by a fixed shuffle tree; no atomics.
+//   dX (src-major, REV CSR, type-sorted rows): the same skeleton gathering dA[dst] with W_r^T staged.
+//   dW (type-major view built at graph_create): dW_r = sum_v g_{v,r} (x) dA[v], where g_{v,r} is the
+//     forward run-sum.  Runs are grouped into tasks that never cross a type, so each warp keeps its
+//     dW_r partial in registers; per-task partials are reduced per type in task order
+//     (deterministic; no shared- or global-memory atomics).
 #include "common.cuh"
+
+namespace seastar {
+
+struct RgcnRowArgs {
+    const int32_t* perm; const int32_t* off; const int32_t* nbr; const int32_t* typ;
+    const float* norm; const int32_t* eid; const float* norm_user;
+    int64_t row_begin, row_end, vbase;
+    const float* table; int64_t ldt;   // gathered rows (X_all forward, dA_all for dX)
+    const float* W;                     // [R, F_in, F_out]
+    int R, Fg, Fo;                      // gathered width, output width
+    int transpose;                      // 0: forward (g W_r), 1: dX (q W_r^T)
+    float* out; int64_t ldo;
+    const float* bias; int act;
+};
+
+// stage W (or W^T) as [R][Fg][Fop] with Fop = round4(Fo), zero padded
+__device__ void stage_w(const RgcnRowArgs& a, float* Ws) {
+    const int Fop = (a.Fo + 3) & ~3;
+    const int64_t n = (int64_t)a.R * a.Fg * Fop;
+    for (int64_t idx = threadIdx.x; idx < n; idx += blockDim.x) {
+        const int j = (int)(idx % Fop);
+        const int64_t ri = idx / Fop;
+        const int i = (int)(ri % a.Fg);
+        const int r = (int)(ri / a.Fg);
+        float w = 0.f;
+        if (j < a.Fo) {
+            // forward: Ws[r][i][j] = W[r][i][j] (i in F_in, j in F_out)
+            // dX     : Ws[r][j'][i'] = W[r][i'][j'] with gathered index = j' (F_out), output = i' (F_in)
+            w = a.transpose ? __ldg(a.W + ((int64_t)r * a.Fo + j) * a.Fg + i)
+                            : __ldg(a.W + ((int64_t)r * a.Fg + i) * a.Fo + j);
+        }
+        Ws[idx] = w;
+    }
+}
+
+template <int L, int RL>
+__global__ void __launch_bounds__(512) k_rgcn_rows(const RgcnRowArgs a) {
+    extern __shared__ float4 smem4[];
+    float* Ws = reinterpret_cast<float*>(smem4);
+    stage_w(a, Ws);
+    __syncthreads();
+    constexpr int S = RL / L;
+    constexpr int UB = (L < 4 ? L : 4);
+    const int lane = threadIdx.x & 31;
+    const int gl = lane % RL;
+    const int slot = gl / L;
+    const int c = gl % L;
+    const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
+    const unsigned smask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << ((lane / L) * L));
+    const int Fop = (a.Fo + 3) & ~3;
+    const int Cg = (a.Fg + 3) / 4, Co = (a.Fo + 3) / 4;
+    const int gpb = blockDim.x / RL;
+    const int64_t ngroups = (int64_t)gridDim.x * gpb;
+
+    for (int64_t row = a.row_begin + (int64_t)blockIdx.x * gpb + threadIdx.x / RL; row < a.row_end; row += ngroups) {
+        const int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+        const int64_t v = (int64_t)__ldg(a.perm + row) - a.vbase;
+        float out[4] = {0.f, 0.f, 0.f, 0.f};
+        float g[4] = {0.f, 0.f, 0.f, 0.f};
+        int cur = -1;
+        auto flush = [&](int r) {
+            const float* wr = Ws + (int64_t)r * a.Fg * Fop;
+#pragma unroll
+            for (int cl = 0; cl < L; ++cl) {
+                if (cl >= Cg) break;
+                float gv[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) gv[q] = __shfl_sync(smask, g[q], cl, L);
+                if (c < Co) {
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const int i = 4 * cl + q;
+                        if (i < a.Fg) {
+                            const float4 w4 = *reinterpret_cast<const float4*>(wr + (int64_t)i * Fop + 4 * c);
+                            out[0] = fmaf(gv[q], w4.x, out[0]);
+                            out[1] = fmaf(gv[q], w4.y, out[1]);
+                            out[2] = fmaf(gv[q], w4.z, out[2]);
+                            out[3] = fmaf(gv[q], w4.w, out[3]);
+                        }
+                    }
+                }
+            }
+        };
+        for (int base = beg; base < end; base += RL) {
+            const int n = min(RL, end - base);
+            int my_u = 0, my_t = 0;
+            float my_w = 0.f;
+            if (gl < n) {
+                my_u = __ldg(a.nbr + base + gl);
+                my_t = __ldg(a.typ + base + gl);
+                my_w = a.norm_user ? __ldg(a.norm_user + __ldg(a.eid + base + gl)) : __ldg(a.norm + base + gl);
+            }
+#pragma unroll
+            for (int j0 = 0; j0 < L; j0 += UB) {
+                if (j0 * S >= n) break;
+                float x[UB][4];
+                int tt[UB];
+                float ww[UB];
+#pragma unroll
+                for (int jj = 0; jj < UB; ++jj) {
+                    const int k = (j0 + jj) * S + slot;
+                    const int u = __shfl_sync(gmask, my_u, k & (RL - 1), RL);
+                    tt[jj] = __shfl_sync(gmask, my_t, k & (RL - 1), RL);
+                    ww[jj] = __shfl_sync(gmask, my_w, k & (RL - 1), RL);
+                    if (k < n && c < Cg) {
+                        const float4 t4 = ldg4(a.table + (int64_t)u * a.ldt + 4 * c);
+                        x[jj][0] = t4.x; x[jj][1] = t4.y; x[jj][2] = t4.z; x[jj][3] = t4.w;
+#pragma unroll
+                        for (int q = 0; q < 4; ++q)
+                            if (4 * c + q >= a.Fg) x[jj][q] = 0.f;
+                    } else {
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) x[jj][q] = 0.f;
+                    }
+                }
+#pragma unroll
+                for (int jj = 0; jj < UB; ++jj) {
+                    const int k = (j0 + jj) * S + slot;
+                    if (k < n) {                     // slot-uniform
+                        if (tt[jj] != cur) {
+                            if (cur >= 0) flush(cur);
+                            g[0] = g[1] = g[2] = g[3] = 0.f;
+                            cur = tt[jj];
+                        }
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) g[q] = fmaf(ww[jj], x[jj][q], g[q]);
+                    }
+                }
+            }
+        }
+        if (cur >= 0) flush(cur);
+#pragma unroll
+        for (int o = L; o < RL; o <<= 1)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) out[q] += __shfl_xor_sync(gmask, out[q], o, RL);
+        if (slot == 0 && c < Co) {
+            float* po = a.out + v * a.ldo + 4 * c;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int j = 4 * c + q;
+                if (j < a.Fo) {
+                    float z = out[q];
+                    if (!a.transpose) z = act_apply(a.act, z + (a.bias ? __ldg(a.bias + j) : 0.f));
+                    po[q] = z;
+                }
+            }
+        }
+    }
+}
+
+struct RgcnDwArgs {
+    const int32_t* src; const int32_t* eid; const float* norm; const float* norm_user;
+    const int32_t* run_off; const int32_t* run_dst; const int32_t* task_run;
+    int64_t n_tasks;
+    const float* X; int64_t ldx; const float* dA; int64_t ldd;
+    int Fin, Fout;
+    float* part;
+};
+
+// warp per task: dW_r partial (Fin x Fout entries, NPL per lane) in registers
+template <int L, int NPL>
+__global__ void __launch_bounds__(256) k_rgcn_dw(const RgcnDwArgs a) {
+    constexpr int S = 32 / L;
+    __shared__ float sg[8][64];
+    __shared__ float sd[8][64];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int slot = lane / L, c = lane % L;
+    const int Cg = (a.Fin + 3) / 4;
+    const int FF = a.Fin * a.Fout;
+    const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t t = blockIdx.x * (int64_t)(blockDim.x >> 5) + w; t < a.n_tasks; t += nwarps) {
+        float acc[NPL];
+#pragma unroll
+        for (int i = 0; i < NPL; ++i) acc[i] = 0.f;
+        const int r0 = __ldg(a.task_run + t), r1 = __ldg(a.task_run + t + 1);
+        for (int run = r0; run < r1; ++run) {
+            const int es = __ldg(a.run_off + run), ee = __ldg(a.run_off + run + 1);
+            const int64_t v = __ldg(a.run_dst + run);
+            float g[4] = {0.f, 0.f, 0.f, 0.f};
+            for (int k = es + slot; k < ee; k += S) {
+                if (c < Cg) {
+                    const int u = __ldg(a.src + k);
+                    const float wgt = a.norm_user ? __ldg(a.norm_user + __ldg(a.eid + k)) : __ldg(a.norm + k);
+                    const float4 x = ldg4(a.X + (int64_t)u * a.ldx + 4 * c);
+                    g[0] = fmaf(wgt, x.x, g[0]); g[1] = fmaf(wgt, x.y, g[1]);
+                    g[2] = fmaf(wgt, x.z, g[2]); g[3] = fmaf(wgt, x.w, g[3]);
+                }
+            }
+#pragma unroll
+            for (int o = L; o < 32; o <<= 1)
+#pragma unroll
+                for (int q = 0; q < 4; ++q) g[q] += __shfl_xor_sync(0xffffffffu, g[q], o);
+            if (slot == 0 && c < Cg)
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    if (4 * c + q < a.Fin) sg[w][4 * c + q] = g[q];
+            for (int j = lane; j < a.Fout; j += 32) sd[w][j] = __ldg(a.dA + v * a.ldd + j);
+            __syncwarp();
+#pragma unroll
+            for (int i = 0; i < NPL; ++i) {
+                const int e = lane + 32 * i;
+                if (e < FF) acc[i] = fmaf(sg[w][e / a.Fout], sd[w][e % a.Fout], acc[i]);
+            }
+            __syncwarp();
+        }
+        float* p = a.part + t * FF;
+#pragma unroll
+        for (int i = 0; i < NPL; ++i) {
+            const int e = lane + 32 * i;
+            if (e < FF) p[e] = acc[i];
+        }
+    }
+}
+
+// dW[r][e] = sum over the tasks of type r (task order) of part[task][e]
+__global__ void k_rgcn_dw_reduce(const float* __restrict__ part, const int32_t* __restrict__ type_task, int R, int FF,
+                                 float* __restrict__ dW) {
+    const int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (idx >= (int64_t)R * FF) return;
+    const int r = (int)(idx / FF), e = (int)(idx % FF);
+    float x = 0.f;
+    for (int t = type_task[r]; t < type_task[r + 1]; ++t) x += part[(int64_t)t * FF + e];
+    dW[idx] = x;
+}
+
+template <int L, int RL>
+static seastar_status launch_rows(const RgcnRowArgs& a, size_t smem, cudaStream_t s) {
+    if (a.row_end <= a.row_begin) return SEASTAR_OK;
+    static bool attr_set = false;
+    if (!attr_set) {
+        SS_CUDA(cudaFuncSetAttribute(k_rgcn_rows<L, RL>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+        attr_set = true;
+    }
+    int per_sm = 0;
+    SS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rgcn_rows<L, RL>, 512, smem));
+    if (per_sm < 1) {
+        set_error("rgcn: W (%zu bytes) does not fit in shared memory", smem);
+        return SEASTAR_ERR_UNSUPPORTED;
+    }
+    const int64_t groups = a.row_end - a.row_begin;
+    int64_t blocks = (int64_t)per_sm * num_sms();
+    const int64_t need = (groups + (512 / RL) - 1) / (512 / RL);
+    if (blocks > need) blocks = need;
+    k_rgcn_rows<L, RL><<<(unsigned)blocks, 512, smem, s>>>(a);
+    return check_launch("k_rgcn_rows");
+}
+
+template <int L>
+static seastar_status launch_buckets(const IndexSet& x, RgcnRowArgs a, size_t smem, cudaStream_t s) {
+    const int64_t split = x.bucket_rows[1];   // rows with degree >= 32 get a warp with 32/L slots
+    RgcnRowArgs hi = a, lo = a;
+    hi.row_begin = 0; hi.row_end = split;
+    lo.row_begin = split; lo.row_end = x.n_rows;
+    SS_TRY((launch_rows<L, 32>(hi, smem, s)));
+    constexpr int RLo = L < 4 ? 4 : L;
+    return launch_rows<L, RLo>(lo, smem, s);
+}
+
+static seastar_status launch_rows_L(const IndexSet& x, const RgcnRowArgs& a, cudaStream_t s) {
+    const int Cm = ((a.Fg > a.Fo ? a.Fg : a.Fo) + 3) / 4;
+    const size_t smem = (size_t)a.R * a.Fg * ((a.Fo + 3) & ~3) * sizeof(float);
+    switch (pow2_ceil(Cm)) {
+        case 1: return launch_buckets<1>(x, a, smem, s);
+        case 2: return launch_buckets<2>(x, a, smem, s);
+        case 4: return launch_buckets<4>(x, a, smem, s);
+        case 8: return launch_buckets<8>(x, a, smem, s);
+        default: return launch_buckets<16>(x, a, smem, s);
+    }
+}
+
+}  // namespace seastar
 
 using namespace seastar;
 
@@ -8,17 +292,97 @@ extern "C" {
 seastar_status seastar_rgcn_fwd(seastar_graph g, const float* X_all, int64_t F_in, int64_t ldx, const float* W,
                                 int64_t F_out, const float* norm_user, const float* bias, seastar_act act,
                                 float* Y_loc, int64_t ldy, seastar_stream stream) {
-    set_error("rgcn_fwd: not implemented yet");
-    return SEASTAR_ERR_UNSUPPORTED;
+    SS_ARG(g && X_all && W && Y_loc, "rgcn_fwd: NULL argument");
+    SS_ARG(F_in >= 1 && F_in <= 64 && F_out >= 1 && F_out <= 64, "rgcn_fwd: need 1 <= F_in, F_out <= 64");
+    SS_ARG(ldx >= F_in && ldx % 4 == 0 && aligned16(X_all), "rgcn_fwd: X_all needs ldx %% 4 == 0 and 16B alignment");
+    SS_ARG(ldy >= F_out, "rgcn_fwd: bad ldy");
+    SS_ARG(g->fwd.type != nullptr || g->R == 1, "rgcn_fwd: graph has no edge types");
+    SS_ARG(norm_user || g->fwd.norm, "rgcn_fwd: pass norm_user or create the graph with SEASTAR_GRAPH_RGCN_NORM");
+    SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "rgcn_fwd: bad activation");
+    SS_ARG(g->fwd.type != nullptr, "rgcn_fwd: graph was created without etypes");
+    SS_TRY(check_device());
+    RgcnRowArgs a{};
+    a.perm = g->fwd.perm; a.off = g->fwd.off; a.nbr = g->fwd.nbr; a.typ = g->fwd.type;
+    a.norm = g->fwd.norm; a.eid = g->fwd.eid; a.norm_user = norm_user;
+    a.vbase = g->row_begin;
+    a.table = X_all; a.ldt = ldx; a.W = W; a.R = g->R; a.Fg = (int)F_in; a.Fo = (int)F_out; a.transpose = 0;
+    a.out = Y_loc; a.ldo = ldy; a.bias = bias; a.act = act;
+    return launch_rows_L(g->fwd, a, to_stream(stream));
 }
 
-size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out) { return 0; }
+size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out) {
+    if (!g) return 0;
+    return (size_t)(g->tm.n_tasks + 1) * (size_t)(F_in * F_out) * sizeof(float) + 256;
+}
 
-seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_loc, int64_t F_in, int64_t ldx, const float* dA_all,
+seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_in, int64_t ldx, const float* dA_all,
                                 int64_t F_out, int64_t ldd, const float* W, const float* norm_user, float* dX_loc,
                                 float* dW, void* workspace, size_t ws_bytes, seastar_stream stream) {
-    set_error("rgcn_bwd: not implemented yet");
-    return SEASTAR_ERR_UNSUPPORTED;
+    SS_ARG(g && X_all && dA_all && W, "rgcn_bwd: NULL argument");
+    SS_ARG(dX_loc || dW, "rgcn_bwd: nothing to compute");
+    SS_ARG(F_in >= 1 && F_in <= 64 && F_out >= 1 && F_out <= 64, "rgcn_bwd: need 1 <= F_in, F_out <= 64");
+    SS_ARG(F_in * F_out <= 32 * 32, "rgcn_bwd: F_in * F_out <= 1024 required for the register dW path");
+    SS_ARG(ldx >= F_in && ldx % 4 == 0 && aligned16(X_all), "rgcn_bwd: X_all needs ldx %% 4 == 0, 16B alignment");
+    SS_ARG(ldd >= F_out && ldd % 4 == 0 && aligned16(dA_all), "rgcn_bwd: dA_all needs ldd %% 4 == 0, 16B alignment");
+    SS_ARG(g->fwd.type != nullptr, "rgcn_bwd: graph was created without etypes");
+    SS_ARG(norm_user || g->fwd.norm, "rgcn_bwd: pass norm_user or create the graph with SEASTAR_GRAPH_RGCN_NORM");
+    SS_ARG(!dW || (workspace && ws_bytes >= seastar_rgcn_bwd_workspace(g, F_in, F_out)),
+           "rgcn_bwd: workspace too small");
+    SS_TRY(check_device());
+    cudaStream_t s = to_stream(stream);
+    if (dX_loc) {
+        RgcnRowArgs a{};
+        a.perm = g->rev.perm; a.off = g->rev.off; a.nbr = g->rev.nbr; a.typ = g->rev.type;
+        a.norm = g->rev.norm; a.eid = g->rev.eid; a.norm_user = norm_user;
+        a.vbase = g->row_begin;
+        a.table = dA_all; a.ldt = ldd; a.W = W; a.R = g->R; a.Fg = (int)F_out; a.Fo = (int)F_in; a.transpose = 1;
+        a.out = dX_loc; a.ldo = ldx; a.bias = nullptr; a.act = SEASTAR_ACT_NONE;
+        SS_TRY(launch_rows_L(g->rev, a, s));
+    }
+    if (dW) {
+        const int FF = (int)(F_in * F_out);
+        if (g->tm.n_tasks > 0) {
+            RgcnDwArgs d{};
+            d.src = g->tm.src; d.eid = g->tm.eid; d.norm = g->tm.norm; d.norm_user = norm_user;
+            d.run_off = g->tm.run_off; d.run_dst = g->tm.run_dst; d.task_run = g->tm.task_run;
+            d.n_tasks = g->tm.n_tasks;
+            d.X = X_all; d.ldx = ldx; d.dA = dA_all; d.ldd = ldd; d.Fin = (int)F_in; d.Fout = (int)F_out;
+            d.part = static_cast<float*>(workspace);
+            int64_t blocks = (g->tm.n_tasks + 7) / 8;
+            const int64_t cap = 16 * (int64_t)num_sms();
+            if (blocks > cap) blocks = cap;
+            const int Cg = (int)((F_in + 3) / 4);
+            const int L = pow2_ceil(Cg);
+            const int npl = pow2_ceil((FF + 31) / 32);
+#define RGCN_DW(LL, NN) k_rgcn_dw<LL, NN><<<(unsigned)blocks, 256, 0, s>>>(d)
+#define RGCN_DW_L(LL)                                                   \
+    switch (npl) {                                                      \
+        case 1: RGCN_DW(LL, 1); break;                                  \
+        case 2: RGCN_DW(LL, 2); break;                                  \
+        case 4: RGCN_DW(LL, 4); break;                                  \
+        case 8: RGCN_DW(LL, 8); break;                                  \
+        case 16: RGCN_DW(LL, 16); break;                                \
+        default: RGCN_DW(LL, 32); break;                                \
+    }
+            switch (L) {
+                case 1: RGCN_DW_L(1); break;
+                case 2: RGCN_DW_L(2); break;
+                case 4: RGCN_DW_L(4); break;
+                case 8: RGCN_DW_L(8); break;
+                default: RGCN_DW_L(16); break;
+            }
+#undef RGCN_DW_L
+#undef RGCN_DW
+            SS_TRY(check_launch("k_rgcn_dw"));
+            const int64_t n = (int64_t)g->R * FF;
+            k_rgcn_dw_reduce<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(static_cast<float*>(workspace),
+                                                                          g->tm.type_task, g->R, FF, dW);
+            SS_TRY(check_launch("k_rgcn_dw_reduce"));
+        } else {
+            SS_CUDA(cudaMemsetAsync(dW, 0, sizeof(float) * (size_t)g->R * FF, s));
+        }
+    }
+    return SEASTAR_OK;
 }
 
 }  // extern "C"
