@@ -83,9 +83,17 @@ def bytes_gat_fwd(E, n, H, F):
 
 
 def bytes_gat_bwd(E, n, H, F):
+    # src-major: per edge 4B dst id + the gathered record D[v] (dA | er, lse, c); per row T, el in, dT, del out
     W = H * F
     ldd = (W + 3) // 4 * 4 + 4 * H
-    return E * (4 + 4 + 4 * ldd + 4 * H) + n * (8 + 4 * W + 4 * H + 4 * W + 4 * H)
+    return E * (4 + 4 * ldd) + n * (8 + 4 * W + 4 * H + 4 * W + 4 * H)
+
+
+def bytes_gat_der(E, n, H, F):
+    # dst-major: per edge 4B src id + el[u] (H floats) + T[u] row; per row the record D[v] in, der out
+    W = H * F
+    ldd = (W + 3) // 4 * 4 + 4 * H
+    return E * (4 + 4 * H + 4 * W) + n * (8 + 4 * ldd + 4 * H)
 
 
 # ------------------------------------------------------------------------------------------
@@ -334,7 +342,8 @@ def main():
     E_f, E_r, n = info["num_fwd_edges"], info["num_rev_edges"], g.n_loc
     alg = {"gat_fwd1": bytes_gat_fwd(E_f, n, 8, 8), "gat_bwd1": bytes_gat_bwd(E_r, n, 8, 8),
            "gat_bwd2": bytes_gat_bwd(E_r, n, 1, 41), "gcn_fwd1": bytes_gcn_agg(E_f, n, 16, 1, 0),
-           "gcn_bwd2": bytes_gcn_agg(E_r, n, 16, 1, 1)}
+           "gcn_bwd2": bytes_gcn_agg(E_r, n, 16, 1, 1), "gat_der1": bytes_gat_der(E_f, n, 8, 8),
+           "gat_der2": bytes_gat_der(E_f, n, 1, 41)}
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))

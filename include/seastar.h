@@ -227,19 +227,21 @@ seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const 
  * Fused source-major backward over the reverse CSR, for every owned u and out-edge e = (u -> v):
  *   a_e = exp(LeakyReLU(el[u,h] + er[v,h]) - lse[v,h]);  g_e = <dA[v,h,:], T[u,h,:]>;
  *   ds_e = a_e (g_e - c[v,h]) LeakyReLU'(s_e);
- *   dT_loc[u,h,:] = sum_e a_e dA[v,h,:];  del_loc[u,h] = sum_e ds_e;  ds_work[pos(e)*H + h] = ds_e.
- * T_loc [n_loc,H*F] ld ldt; el_loc [n_loc,H]; D_all [N, gat_record_ld] (gathered);
- * ds_work [num_lsf_edges, H] where pos(e) is the FWD position (or LSF position when partitioned).
+ *   dT_loc[u,h,:] = sum_e a_e dA[v,h,:];  del_loc[u,h] = sum_e ds_e   (registers, no atomics).
+ * T_loc [n_loc,H*F] ld ldt; el_loc [n_loc,H]; D_all [N, gat_record_ld] (gathered records).
  */
 seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float* el_loc, const float* D_all,
                                int32_t H, int32_t F, int64_t ldt, float slope, float* dT_loc, float* del_loc,
-                               float* ds_work, seastar_stream stream);
+                               seastar_stream stream);
 /*
- * der[v,h] = sum_{e in in(v)} ds_work[pos(e)*H + h] as a dst-major, coalesced segment sum.
- * Unpartitioned: der is [N,H] (all rows are owned).  Partitioned: der is the partial [N,H] over
- * local-source edges (reduce-scatter it across ranks).
+ * Fused destination-major pass over the forward CSR: der_loc[v,h] = sum_{e in in(v)} ds_e with ds_e
+ * recomputed from the gathered T_all / el_all rows and v's own record D_loc[v] (no E x H array is
+ * materialised; when partitioned each rank computes its owned rows, no reduction is needed).
+ * T_all [N,H*F] ld ldt, el_all [N,H] (the forward's gathered tables); D_loc [n_loc, gat_record_ld];
+ * der_loc [n_loc,H].
  */
-seastar_status seastar_gat_der(seastar_graph g, const float* ds_work, int32_t H, float* der, seastar_stream stream);
+seastar_status seastar_gat_der(seastar_graph g, const float* T_all, const float* el_all, const float* D_loc,
+                               int32_t H, int32_t F, int64_t ldt, float slope, float* der_loc, seastar_stream stream);
 /*
  * Backward of seastar_gat_attn_proj over M rows:  dT[u,h,:] += del[u,h] a_l[h,:] + der[u,h] a_r[h,:];
  * da_l = sum_u del[u,h] T[u,h,:];  da_r = sum_u der[u,h] T[u,h,:]   (deterministic, via workspace of

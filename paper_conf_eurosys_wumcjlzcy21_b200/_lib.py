@@ -69,8 +69,8 @@ _SIGS = {
     "seastar_gat_fwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _I32, _P, _P, _P, _P], _ST),
     "seastar_gat_record_ld": ([_I32, _I32], _I64),
     "seastar_gat_bwd_prep": ([_P, _P, _P, _I32, _P, _P, _P, _I32, _I32, _I64, _P, _P], _ST),
-    "seastar_gat_bwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P, _P, _P], _ST),
-    "seastar_gat_der": ([_P, _P, _I32, _P, _P], _ST),
+    "seastar_gat_bwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P, _P], _ST),
+    "seastar_gat_der": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P], _ST),
     "seastar_gat_attn_proj_bwd": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P, _P, _P, _P, _SZ, _P], _ST),
     "seastar_gat_attn_proj_bwd_workspace": ([_I64, _I32, _I32], _SZ),
     "seastar_rgcn_fwd": ([_P, _P, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
@@ -253,13 +253,14 @@ def seastar_gat_bwd_prep(g, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, H, F, ld
           _dptr(er_loc, "er"), _dptr(lse_loc, "lse"), H, F, ldt, _dptr(D_loc, "D"), _stream(stream))
 
 
-def seastar_gat_bwd(g, T_loc, el_loc, D_all, H, F, ldt, slope, dT_loc, del_loc, ds_work, stream=None) -> None:
+def seastar_gat_bwd(g, T_loc, el_loc, D_all, H, F, ldt, slope, dT_loc, del_loc, stream=None) -> None:
     _call("seastar_gat_bwd", g, _dptr(T_loc, "T"), _dptr(el_loc, "el"), _dptr(D_all, "D"), H, F, ldt, float(slope),
-          _dptr(dT_loc, "dT"), _dptr(del_loc, "del"), _dptr(ds_work, "ds"), _stream(stream))
+          _dptr(dT_loc, "dT"), _dptr(del_loc, "del"), _stream(stream))
 
 
-def seastar_gat_der(g, ds_work, H, der, stream=None) -> None:
-    _call("seastar_gat_der", g, _dptr(ds_work, "ds"), H, _dptr(der, "der"), _stream(stream))
+def seastar_gat_der(g, T_all, el_all, D_loc, H, F, ldt, slope, der_loc, stream=None) -> None:
+    _call("seastar_gat_der", g, _dptr(T_all, "T"), _dptr(el_all, "el"), _dptr(D_loc, "D"), H, F, ldt, float(slope),
+          _dptr(der_loc, "der"), _stream(stream))
 
 
 def seastar_gat_attn_proj_bwd_workspace(M, H, F) -> int:

@@ -2,17 +2,24 @@
 //
 // Forward: the paper's FSM splits the GAT forward into 2 fused units at the Div (L391-L393:
 // AggSum of exp, then Div -> Mul -> AggSum).  On B200 it is ONE pass over in(v): an online
-// softmax keeps (running max m, running sum S, running weighted row acc) per head in registers, so
-// no E-sized intermediate and no second gather of T are needed.  lse = m + log S is saved for the
+// softmax keeps (running max m, running sum S, running weighted row acc) in registers, so no
+// E-sized intermediate and no second gather of T are needed.  lse = m + log S is saved for the
 // backward.
 //
 // Backward (§6.3.4: the Aggregation stage becomes the Source stage on the reverse CSR):
 //   row pass (gat_bwd_prep): dA = dY act'(Y), c[v,h] = <dA[v,h], A[v,h]> (= sum_e a_e <dA_v, T_u>,
 //     which removes the softmax-Jacobian pass), packed with er and lse into one record D[v];
-//   source-major pass (gat_bwd): per u, per out-edge (u->v): a_e from lse, g_e = <dA_v, T_u> with
-//     T_u held in registers, ds_e = a_e (g_e - c_v) LReLU'(s_e); dT_u += a_e dA_v and del_u += ds_e
-//     accumulate in registers (no atomics); ds_e is stored at the edge's forward position;
-//   der (gat_der): dst-major coalesced segment sum of ds over each forward row.
+//   source-major pass (gat_bwd, REV CSR): per u, per out-edge (u->v): a_e = exp(LReLU(s_e) - lse_v),
+//     g_e = <dA_v, T_u>, ds_e = a_e (g_e - c_v) LReLU'(s_e); dT_u += a_e dA_v, del_u += ds_e in
+//     registers (no atomics);
+//   destination-major pass (gat_der, FWD CSR): der_v = sum_{e in in(v)} ds_e, recomputing ds_e from
+//     the L2-resident T / el tables instead of materialising an E x H array.
+//
+// Two lane mappings:
+//   * head-per-lane ("hpl", H | 32, F % 4 == 0, F <= 32): lane = (edge slot, head), each lane owns a
+//     whole head row of F floats: one exp per (edge, head), dot products stay inside a lane;
+//   * chunked (any H, F): a row is split into float4 (or float) chunks over L lanes per edge,
+//     head dot products by a segmented shuffle reduction.
 #include <math.h>
 
 #include "common.cuh"
@@ -30,13 +37,16 @@ struct GatFwdArgs {
     float* A; float* Y; float* lse;
 };
 
-// lane geometry shared by the GAT kernels: chunk `chunk` covers floats [chunk*VEC, chunk*VEC+VEC)
+// lane geometry of the chunked kernels: chunk `chunk` covers floats [chunk*VEC, chunk*VEC+VEC)
 // of a row of W = H*F floats; with VEC = 4 every chunk lies inside one head (F % 4 == 0 or H == 1)
 template <int VEC>
 __device__ __forceinline__ int head_of(int chunk, int F, int H) {
     return H == 1 ? 0 : (chunk * VEC) / F;
 }
 
+// ============================================================================================
+// forward
+// ============================================================================================
 template <int VEC, int L, int RL>
 __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
     constexpr int S = RL / L;
@@ -139,14 +149,111 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
         a.lse[v * a.H + h] = ssum > 0.f ? m + logf(ssum) : -INFINITY;
 }
 
+// head-per-lane forward: warp per destination row; lane = (slot, head), S = 32/H edge slots.
+template <int F4>
+__global__ void __launch_bounds__(256) k_gat_fwd_hpl(const GatFwdArgs a) {
+    constexpr int F = 4 * F4;
+    constexpr int UB = F4 <= 2 ? 4 : (F4 <= 4 ? 2 : 1);
+    const int H = a.H;
+    const int S = 32 / H;
+    const int lane = threadIdx.x & 31;
+    const int h = lane % H, slot = lane / H;
+    const int64_t row = a.row_begin + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    if (row >= a.row_end) return;                      // warp-uniform
+    const int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+    const int64_t v = (int64_t)__ldg(a.perm + row) - a.vbase;
+    const float erv = __ldg(a.er + v * H + h);
+    const int64_t hoff = (int64_t)h * F;
+    float m = -INFINITY, ssum = 0.f, acc[F];
+#pragma unroll
+    for (int i = 0; i < F; ++i) acc[i] = 0.f;
+    for (int base = beg; base < end; base += 32) {
+        const int n = min(32, end - base);
+        const int my = (lane < n) ? __ldg(a.nbr + base + lane) : 0;
+        for (int i0 = 0; i0 < H; i0 += UB) {             // this slot's edges: k = slot + S * i
+            if (i0 * S >= n) break;
+            float z[UB], x[UB][F];
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const int k = slot + S * (i0 + jj);
+                const int u = __shfl_sync(0xffffffffu, my, k & 31);
+                if (k < n && i0 + jj < H) {
+                    z[jj] = lrelu(__ldg(a.el + (int64_t)u * H + h) + erv, a.slope);
+                    const float* tp = a.T + (int64_t)u * a.ld + hoff;
+#pragma unroll
+                    for (int q = 0; q < F4; ++q) {
+                        const float4 t4 = ldg4(tp + 4 * q);
+                        x[jj][4 * q] = t4.x; x[jj][4 * q + 1] = t4.y; x[jj][4 * q + 2] = t4.z; x[jj][4 * q + 3] = t4.w;
+                    }
+                } else {
+                    z[jj] = -INFINITY;
+#pragma unroll
+                    for (int i = 0; i < F; ++i) x[jj][i] = 0.f;
+                }
+            }
+            float mb = m;
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) mb = fmaxf(mb, z[jj]);
+            const float corr = (m == -INFINITY) ? 0.f : expf(m - mb);
+            ssum *= corr;
+#pragma unroll
+            for (int i = 0; i < F; ++i) acc[i] *= corr;
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const float p = (z[jj] == -INFINITY) ? 0.f : expf(z[jj] - mb);
+                ssum += p;
+#pragma unroll
+                for (int i = 0; i < F; ++i) acc[i] = fmaf(p, x[jj][i], acc[i]);
+            }
+            m = mb;
+        }
+    }
+    for (int o = H; o < 32; o <<= 1) {
+        const float mo = __shfl_xor_sync(0xffffffffu, m, o);
+        const float so = __shfl_xor_sync(0xffffffffu, ssum, o);
+        const float mn = fmaxf(m, mo);
+        const float ca = (m == -INFINITY) ? 0.f : expf(m - mn);
+        const float cb = (mo == -INFINITY) ? 0.f : expf(mo - mn);
+        ssum = ssum * ca + so * cb;
+#pragma unroll
+        for (int i = 0; i < F; ++i) acc[i] = acc[i] * ca + __shfl_xor_sync(0xffffffffu, acc[i], o) * cb;
+        m = mn;
+    }
+    if (slot != 0) return;
+    const float inv = ssum > 0.f ? 1.f / ssum : 0.f;
+    float* pa = a.A + v * a.ld + hoff;
+    float* py = a.Y + v * a.ld + hoff;
+#pragma unroll
+    for (int q = 0; q < F4; ++q) {
+        float o4[4], y4[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            o4[i] = acc[4 * q + i] * inv;
+            y4[i] = act_apply(a.act, o4[i] + (a.bias ? __ldg(a.bias + hoff + 4 * q + i) : 0.f));
+        }
+        *reinterpret_cast<float4*>(pa + 4 * q) = make_float4(o4[0], o4[1], o4[2], o4[3]);
+        *reinterpret_cast<float4*>(py + 4 * q) = make_float4(y4[0], y4[1], y4[2], y4[3]);
+    }
+    a.lse[v * H + h] = ssum > 0.f ? m + logf(ssum) : -INFINITY;
+}
+
+// ============================================================================================
+// backward
+// ============================================================================================
 struct GatBwdArgs {
-    const int32_t* perm; const int32_t* off; const int32_t* nbr; const int32_t* pos;
+    const int32_t* perm; const int32_t* off; const int32_t* nbr;
     int64_t row_begin, row_end, vbase;
-    const float* T; const float* el; const float* D;
+    const float* T;      // gathered (der) or owned (src-major) rows
+    const float* el;     // gathered (der) or owned (src-major)
+    const float* D;      // packed records: gathered (src-major) or owned (der)
     int H, F; int64_t ldt, ldd; float slope;
-    float* dT; float* del; float* ds;
+    float* dT; float* del;   // src-major outputs
+    float* der;              // der output
 };
 
+__device__ __forceinline__ int rec_aux_offset(int W) { return (W + 3) & ~3; }
+
+// chunked source-major backward (REV CSR): dT_u, del_u
 template <int VEC, int L, int RL>
 __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
     constexpr int S = RL / L;
@@ -168,10 +275,10 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
     const bool active = chunk < C;
     const int h = active ? head_of<VEC>(chunk, a.F, a.H) : (a.H - 1);
     const int64_t col = (int64_t)chunk * VEC;
-    // lanes of head h inside the edge group: [hs, hs + lph)
-    const int lph = (a.H == 1) ? C : (a.F / VEC);
+    const int lph = (a.H == 1) ? C : (a.F / VEC);      // lanes of head h inside the edge group
     const int hc = active ? (a.H == 1 ? chunk : chunk - h * lph) : 0;
     const int hs = c - hc;
+    const int aux0 = rec_aux_offset(W);
 
     float t[VEC];
     if (valid && active) load_vec<VEC>(a.T + u * a.ldt + col, t);
@@ -186,34 +293,22 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
         const int myv = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
-        const int myp = (gl < n) ? __ldg(a.pos + base + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
             float dA[UB][VEC], er[UB], lse[UB], cv[UB];
-            int pe[UB];
 #pragma unroll
             for (int jj = 0; jj < UB; ++jj) {
                 const int k = (j0 + jj) * S + slot;
                 const int v = __shfl_sync(gmask, myv, k & (RL - 1), RL);
-                pe[jj] = __shfl_sync(gmask, myp, k & (RL - 1), RL);
                 if (k < n && active) {
                     const float* rec = a.D + (int64_t)v * a.ldd;
                     load_vec<VEC>(rec + col, dA[jj]);
 #pragma unroll
                     for (int i = 0; i < VEC; ++i)
                         if (col + i >= W) dA[jj][i] = 0.f;
-                    const float* aux = rec + ((W + 3) & ~3) + 4 * h;
-                    if constexpr (VEC == 4) {
-                        if ((a.ldd & 3) == 0) {
-                            const float4 x = ldg4(aux);
-                            er[jj] = x.x; lse[jj] = x.y; cv[jj] = x.z;
-                        } else {
-                            er[jj] = __ldg(aux); lse[jj] = __ldg(aux + 1); cv[jj] = __ldg(aux + 2);
-                        }
-                    } else {
-                        er[jj] = __ldg(aux); lse[jj] = __ldg(aux + 1); cv[jj] = __ldg(aux + 2);
-                    }
+                    const float* aux = rec + aux0 + 4 * h;
+                    er[jj] = __ldg(aux); lse[jj] = __ldg(aux + 1); cv[jj] = __ldg(aux + 2);
                 } else {
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) dA[jj][i] = 0.f;
@@ -223,7 +318,6 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
 #pragma unroll
             for (int jj = 0; jj < UB; ++jj) {
                 const int k = (j0 + jj) * S + slot;
-                // g = <dA_v[h], T_u[h]> : segmented reduction over the lanes of head h, then broadcast
                 float gp = 0.f;
 #pragma unroll
                 for (int i = 0; i < VEC; ++i) gp = fmaf(dA[jj][i], t[i], gp);
@@ -236,11 +330,9 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
                 if (k < n && active) {
                     const float s = elu + er[jj];
                     const float al = expf(lrelu(s, a.slope) - lse[jj]);
-                    const float ds = al * (g - cv[jj]) * (s > 0.f ? 1.f : a.slope);
+                    dl += al * (g - cv[jj]) * (s > 0.f ? 1.f : a.slope);
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) acc[i] = fmaf(al, dA[jj][i], acc[i]);
-                    dl += ds;
-                    if (hc == 0) a.ds[(int64_t)pe[jj] * a.H + h] = ds;
                 }
             }
         }
@@ -259,36 +351,462 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
     if (hc == 0) a.del[u * a.H + h] = dl;
 }
 
-// der[v,h] = sum over row of ds[j*H + h]; warp per row, rows given by (perm or identity, off)
-__global__ void __launch_bounds__(256) k_gat_der(const int32_t* __restrict__ perm, const int32_t* __restrict__ off,
-                                                 int64_t n_rows, int64_t vbase, const float* __restrict__ ds, int H,
-                                                 float* __restrict__ der) {
+// chunked destination-major der pass (FWD CSR): der_v = sum_{e in in(v)} ds_e
+template <int VEC, int L, int RL>
+__global__ void __launch_bounds__(256) k_gat_der(const GatBwdArgs a) {
+    constexpr int S = RL / L;
+    constexpr int UB = (L < 4 ? L : 4);
     const int lane = threadIdx.x & 31;
-    const int64_t row = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    if (row >= n_rows) return;
-    const int64_t beg = (int64_t)__ldg(off + row) * H, end = (int64_t)__ldg(off + row + 1) * H;
-    const int64_t v = (perm ? (int64_t)__ldg(perm + row) : row) - vbase;
-    if ((32 % H) == 0) {
-        float x0 = 0.f, x1 = 0.f;
-        int64_t i = beg + lane;
-        for (; i + 32 < end; i += 64) {   // two loads in flight
-            x0 += __ldg(ds + i);
-            x1 += __ldg(ds + i + 32);
+    const int gl = lane % RL;
+    const int slot = gl / L;
+    const int c = gl % L;
+    const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t row = a.row_begin + warp * (32 / RL) + lane / RL;
+    const bool valid = row < a.row_end;
+    const int beg = valid ? __ldg(a.off + row) : 0;
+    const int end = valid ? __ldg(a.off + row + 1) : 0;
+    const int64_t v = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;
+    const int W = a.H * a.F;
+    const int C = (W + VEC - 1) / VEC;
+    const int chunk = c;
+    const bool active = chunk < C;
+    const int h = active ? head_of<VEC>(chunk, a.F, a.H) : (a.H - 1);
+    const int64_t col = (int64_t)chunk * VEC;
+    const int lph = (a.H == 1) ? C : (a.F / VEC);
+    const int hc = active ? (a.H == 1 ? chunk : chunk - h * lph) : 0;
+    const int hs = c - hc;
+
+    float d[VEC];
+    float erv = 0.f, lsev = 0.f, cvv = 0.f;
+    if (valid && active) {
+        const float* rec = a.D + v * a.ldd;
+        load_vec<VEC>(rec + col, d);
+        const float* aux = rec + rec_aux_offset(W) + 4 * h;
+        erv = __ldg(aux); lsev = __ldg(aux + 1); cvv = __ldg(aux + 2);
+    }
+#pragma unroll
+    for (int i = 0; i < VEC; ++i)
+        if (!(valid && active) || col + i >= W) d[i] = 0.f;
+    float dr = 0.f;
+    for (int base = beg; base < end; base += RL) {
+        const int n = min(RL, end - base);
+        const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+#pragma unroll
+        for (int j0 = 0; j0 < L; j0 += UB) {
+            if (j0 * S >= n) break;
+            float t[UB][VEC], elu[UB];
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const int k = (j0 + jj) * S + slot;
+                const int u = __shfl_sync(gmask, my, k & (RL - 1), RL);
+                if (k < n && active) {
+                    load_vec<VEC>(a.T + (int64_t)u * a.ldt + col, t[jj]);
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i)
+                        if (col + i >= W) t[jj][i] = 0.f;
+                    elu[jj] = __ldg(a.el + (int64_t)u * a.H + h);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) t[jj][i] = 0.f;
+                    elu[jj] = 0.f;
+                }
+            }
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const int k = (j0 + jj) * S + slot;
+                float gp = 0.f;
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) gp = fmaf(d[i], t[jj][i], gp);
+#pragma unroll
+                for (int o = 1; o < L; o <<= 1) {
+                    const float x = __shfl_down_sync(gmask, gp, o, L);
+                    if (hc + o < lph) gp += x;
+                }
+                const float g = __shfl_sync(gmask, gp, hs, L);
+                if (k < n && active) {
+                    const float s = elu[jj] + erv;
+                    const float al = expf(lrelu(s, a.slope) - lsev);
+                    dr += al * (g - cvv) * (s > 0.f ? 1.f : a.slope);
+                }
+            }
         }
-        if (i < end) x0 += __ldg(ds + i);
-        float x = x0 + x1;
-        // lanes l and l' share a head iff l = l' (mod H); the row block starts at a multiple of H
-        for (int o = H; o < 32; o <<= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
-        if (lane < H) der[v * H + lane] = x;
-    } else {
-        for (int hh = lane; hh < H; hh += 32) {
-            float x = 0.f;
-            for (int64_t i = beg + hh; i < end; i += H) x += __ldg(ds + i);
-            der[v * H + hh] = x;
+    }
+#pragma unroll
+    for (int o = L; o < RL; o <<= 1) dr += __shfl_xor_sync(gmask, dr, o, RL);
+    if (!valid || slot != 0 || !active) return;
+    if (hc == 0) a.der[v * a.H + h] = dr;
+}
+
+// head-per-lane source-major backward (REV CSR)
+template <int F4>
+__global__ void __launch_bounds__(256) k_gat_bwd_hpl(const GatBwdArgs a) {
+    constexpr int F = 4 * F4;
+    constexpr int UB = F4 <= 2 ? 4 : (F4 <= 4 ? 2 : 1);
+    const int H = a.H, S = 32 / H;
+    const int lane = threadIdx.x & 31;
+    const int h = lane % H, slot = lane / H;
+    const int64_t row = a.row_begin + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    if (row >= a.row_end) return;
+    const int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+    const int64_t u = (int64_t)__ldg(a.perm + row) - a.vbase;
+    const int64_t hoff = (int64_t)h * F;
+    const int aux0 = rec_aux_offset(H * F) + 4 * h;
+    float t[F], acc[F];
+#pragma unroll
+    for (int q = 0; q < F4; ++q) {
+        const float4 t4 = ldg4(a.T + u * a.ldt + hoff + 4 * q);
+        t[4 * q] = t4.x; t[4 * q + 1] = t4.y; t[4 * q + 2] = t4.z; t[4 * q + 3] = t4.w;
+    }
+#pragma unroll
+    for (int i = 0; i < F; ++i) acc[i] = 0.f;
+    const float elu = __ldg(a.el + u * H + h);
+    float dl = 0.f;
+    for (int base = beg; base < end; base += 32) {
+        const int n = min(32, end - base);
+        const int my = (lane < n) ? __ldg(a.nbr + base + lane) : 0;
+        for (int i0 = 0; i0 < H; i0 += UB) {
+            if (i0 * S >= n) break;
+            float d[UB][F], ax[UB][3];
+            bool ok[UB];
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const int k = slot + S * (i0 + jj);
+                const int v = __shfl_sync(0xffffffffu, my, k & 31);
+                ok[jj] = k < n && i0 + jj < H;
+                if (ok[jj]) {
+                    const float* rec = a.D + (int64_t)v * a.ldd;
+#pragma unroll
+                    for (int q = 0; q < F4; ++q) {
+                        const float4 d4 = ldg4(rec + hoff + 4 * q);
+                        d[jj][4 * q] = d4.x; d[jj][4 * q + 1] = d4.y; d[jj][4 * q + 2] = d4.z; d[jj][4 * q + 3] = d4.w;
+                    }
+                    const float4 x4 = ldg4(rec + aux0);
+                    ax[jj][0] = x4.x; ax[jj][1] = x4.y; ax[jj][2] = x4.z;
+                } else {
+#pragma unroll
+                    for (int i = 0; i < F; ++i) d[jj][i] = 0.f;
+                    ax[jj][0] = 0.f; ax[jj][1] = INFINITY; ax[jj][2] = 0.f;
+                }
+            }
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                if (!ok[jj]) continue;
+                float g = 0.f;
+#pragma unroll
+                for (int i = 0; i < F; ++i) g = fmaf(d[jj][i], t[i], g);
+                const float s = elu + ax[jj][0];
+                const float al = expf(lrelu(s, a.slope) - ax[jj][1]);
+                dl += al * (g - ax[jj][2]) * (s > 0.f ? 1.f : a.slope);
+#pragma unroll
+                for (int i = 0; i < F; ++i) acc[i] = fmaf(al, d[jj][i], acc[i]);
+            }
+        }
+    }
+    for (int o = H; o < 32; o <<= 1) {
+#pragma unroll
+        for (int i = 0; i < F; ++i) acc[i] += __shfl_xor_sync(0xffffffffu, acc[i], o);
+        dl += __shfl_xor_sync(0xffffffffu, dl, o);
+    }
+    if (slot != 0) return;
+    float* pd = a.dT + u * a.ldt + hoff;
+#pragma unroll
+    for (int q = 0; q < F4; ++q)
+        *reinterpret_cast<float4*>(pd + 4 * q) = make_float4(acc[4 * q], acc[4 * q + 1], acc[4 * q + 2], acc[4 * q + 3]);
+    a.del[u * H + h] = dl;
+}
+
+// head-per-lane destination-major der pass (FWD CSR)
+template <int F4>
+__global__ void __launch_bounds__(256) k_gat_der_hpl(const GatBwdArgs a) {
+    constexpr int F = 4 * F4;
+    constexpr int UB = F4 <= 2 ? 4 : (F4 <= 4 ? 2 : 1);
+    const int H = a.H, S = 32 / H;
+    const int lane = threadIdx.x & 31;
+    const int h = lane % H, slot = lane / H;
+    const int64_t row = a.row_begin + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    if (row >= a.row_end) return;
+    const int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+    const int64_t v = (int64_t)__ldg(a.perm + row) - a.vbase;
+    const int64_t hoff = (int64_t)h * F;
+    const float* rec = a.D + v * a.ldd;
+    float d[F];
+#pragma unroll
+    for (int q = 0; q < F4; ++q) {
+        const float4 d4 = ldg4(rec + hoff + 4 * q);
+        d[4 * q] = d4.x; d[4 * q + 1] = d4.y; d[4 * q + 2] = d4.z; d[4 * q + 3] = d4.w;
+    }
+    const float4 x4 = ldg4(rec + rec_aux_offset(H * F) + 4 * h);
+    const float erv = x4.x, lsev = x4.y, cvv = x4.z;
+    float dr = 0.f;
+    for (int base = beg; base < end; base += 32) {
+        const int n = min(32, end - base);
+        const int my = (lane < n) ? __ldg(a.nbr + base + lane) : 0;
+        for (int i0 = 0; i0 < H; i0 += UB) {
+            if (i0 * S >= n) break;
+            float t[UB][F], elu[UB];
+            bool ok[UB];
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const int k = slot + S * (i0 + jj);
+                const int u = __shfl_sync(0xffffffffu, my, k & 31);
+                ok[jj] = k < n && i0 + jj < H;
+                if (ok[jj]) {
+                    const float* tp = a.T + (int64_t)u * a.ldt + hoff;
+#pragma unroll
+                    for (int q = 0; q < F4; ++q) {
+                        const float4 t4 = ldg4(tp + 4 * q);
+                        t[jj][4 * q] = t4.x; t[jj][4 * q + 1] = t4.y; t[jj][4 * q + 2] = t4.z; t[jj][4 * q + 3] = t4.w;
+                    }
+                    elu[jj] = __ldg(a.el + (int64_t)u * H + h);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < F; ++i) t[jj][i] = 0.f;
+                    elu[jj] = 0.f;
+                }
+            }
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                if (!ok[jj]) continue;
+                float g = 0.f;
+#pragma unroll
+                for (int i = 0; i < F; ++i) g = fmaf(d[i], t[jj][i], g);
+                const float s = elu[jj] + erv;
+                const float al = expf(lrelu(s, a.slope) - lsev);
+                dr += al * (g - cvv) * (s > 0.f ? 1.f : a.slope);
+            }
+        }
+    }
+    for (int o = H; o < 32; o <<= 1) dr += __shfl_xor_sync(0xffffffffu, dr, o);
+    if (slot == 0) a.der[v * H + h] = dr;
+}
+
+// ============================================================================================
+// single-head kernels: each lane owns VPL consecutive float4 chunks of the row, L lanes per edge
+// (L <= 4), S = RL / L edge slots; g = <dA, T> by an L-lane xor reduction
+// ============================================================================================
+template <int VPL>
+__device__ __forceinline__ void load_chunks(const float* p, int col0, int W, float (&x)[4 * VPL]) {
+#pragma unroll
+    for (int q = 0; q < VPL; ++q) {
+        const int col = col0 + 4 * q;
+        if (col < W) {
+            const float4 t = ldg4(p + col);
+            x[4 * q] = t.x; x[4 * q + 1] = t.y; x[4 * q + 2] = t.z; x[4 * q + 3] = t.w;
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+                if (col + i >= W) x[4 * q + i] = 0.f;
+        } else {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) x[4 * q + i] = 0.f;
         }
     }
 }
 
+template <int VPL, int L, int RL>
+__global__ void __launch_bounds__(256) k_gat_fwd_h1(const GatFwdArgs a) {
+    constexpr int NV = 4 * VPL, S = RL / L, UB = VPL <= 2 ? 4 : 2;
+    const int lane = threadIdx.x & 31;
+    const int gl = lane % RL, slot = gl / L, c = gl % L;
+    const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t row = a.row_begin + warp * (32 / RL) + lane / RL;
+    const bool valid = row < a.row_end;
+    const int beg = valid ? __ldg(a.off + row) : 0;
+    const int end = valid ? __ldg(a.off + row + 1) : 0;
+    const int64_t v = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;
+    const int W = a.F, col0 = c * NV;
+    const float erv = valid ? __ldg(a.er + v) : 0.f;
+    float m = -INFINITY, ssum = 0.f, acc[NV];
+#pragma unroll
+    for (int i = 0; i < NV; ++i) acc[i] = 0.f;
+    for (int base = beg; base < end; base += RL) {
+        const int n = min(RL, end - base);
+        const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+#pragma unroll
+        for (int j0 = 0; j0 < L; j0 += UB) {
+            if (j0 * S >= n) break;
+            float z[UB], x[UB][NV];
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const int k = (j0 + jj) * S + slot;
+                const int u = __shfl_sync(gmask, my, k & (RL - 1), RL);
+                if (k < n && j0 + jj < L) {
+                    z[jj] = lrelu(__ldg(a.el + u) + erv, a.slope);
+                    load_chunks<VPL>(a.T + (int64_t)u * a.ld, col0, W, x[jj]);
+                } else {
+                    z[jj] = -INFINITY;
+#pragma unroll
+                    for (int i = 0; i < NV; ++i) x[jj][i] = 0.f;
+                }
+            }
+            float mb = m;
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) mb = fmaxf(mb, z[jj]);
+            const float corr = (m == -INFINITY) ? 0.f : expf(m - mb);
+            ssum *= corr;
+#pragma unroll
+            for (int i = 0; i < NV; ++i) acc[i] *= corr;
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const float p = (z[jj] == -INFINITY) ? 0.f : expf(z[jj] - mb);
+                ssum += p;
+#pragma unroll
+                for (int i = 0; i < NV; ++i) acc[i] = fmaf(p, x[jj][i], acc[i]);
+            }
+            m = mb;
+        }
+    }
+#pragma unroll
+    for (int o = L; o < RL; o <<= 1) {
+        const float mo = __shfl_xor_sync(gmask, m, o, RL);
+        const float so = __shfl_xor_sync(gmask, ssum, o, RL);
+        const float mn = fmaxf(m, mo);
+        const float ca = (m == -INFINITY) ? 0.f : expf(m - mn);
+        const float cb = (mo == -INFINITY) ? 0.f : expf(mo - mn);
+        ssum = ssum * ca + so * cb;
+#pragma unroll
+        for (int i = 0; i < NV; ++i) acc[i] = acc[i] * ca + __shfl_xor_sync(gmask, acc[i], o, RL) * cb;
+        m = mn;
+    }
+    if (!valid || slot != 0) return;
+    const float inv = ssum > 0.f ? 1.f / ssum : 0.f;
+    float* pa = a.A + v * a.ld;
+    float* py = a.Y + v * a.ld;
+#pragma unroll
+    for (int q = 0; q < VPL; ++q) {
+        const int col = col0 + 4 * q;
+        if (col >= W) continue;
+        float o4[4], y4[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            o4[i] = acc[4 * q + i] * inv;
+            y4[i] = act_apply(a.act, o4[i] + ((a.bias && col + i < W) ? __ldg(a.bias + col + i) : 0.f));
+        }
+        if (col + 4 <= W) {
+            *reinterpret_cast<float4*>(pa + col) = make_float4(o4[0], o4[1], o4[2], o4[3]);
+            *reinterpret_cast<float4*>(py + col) = make_float4(y4[0], y4[1], y4[2], y4[3]);
+        } else {
+            for (int i = 0; i < 4 && col + i < W; ++i) { pa[col + i] = o4[i]; py[col + i] = y4[i]; }
+        }
+    }
+    if (c == 0) a.lse[v] = ssum > 0.f ? m + logf(ssum) : -INFINITY;
+}
+
+// DER = false: source-major dT/del over REV; DER = true: destination-major der over FWD
+template <int VPL, int L, int RL, bool DER>
+__global__ void __launch_bounds__(256) k_gat_bwd_h1(const GatBwdArgs a) {
+    constexpr int NV = 4 * VPL, S = RL / L, UB = VPL <= 2 ? 4 : 2;
+    const int lane = threadIdx.x & 31;
+    const int gl = lane % RL, slot = gl / L, c = gl % L;
+    const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t row = a.row_begin + warp * (32 / RL) + lane / RL;
+    const bool valid = row < a.row_end;
+    const int beg = valid ? __ldg(a.off + row) : 0;
+    const int end = valid ? __ldg(a.off + row + 1) : 0;
+    const int64_t w = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;   // u (src-major) or v (der)
+    const int W = a.F, col0 = c * NV;
+    const int aux0 = rec_aux_offset(W);
+    // per-row constants: src-major holds T_u and el_u; der holds dA_v and (er, lse, c)_v
+    float own[NV];
+    float k0 = 0.f, k1 = 0.f, k2 = 0.f;
+    if (valid) {
+        if (!DER) {
+            load_chunks<VPL>(a.T + w * a.ldt, col0, W, own);
+            k0 = __ldg(a.el + w);
+        } else {
+            const float* rec = a.D + w * a.ldd;
+            load_chunks<VPL>(rec, col0, W, own);
+            k0 = __ldg(rec + aux0); k1 = __ldg(rec + aux0 + 1); k2 = __ldg(rec + aux0 + 2);
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < NV; ++i) own[i] = 0.f;
+    }
+    float acc[NV], dsum = 0.f;
+#pragma unroll
+    for (int i = 0; i < NV; ++i) acc[i] = 0.f;
+    for (int base = beg; base < end; base += RL) {
+        const int n = min(RL, end - base);
+        const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+#pragma unroll
+        for (int j0 = 0; j0 < L; j0 += UB) {
+            if (j0 * S >= n) break;
+            float x[UB][NV], e0[UB], e1[UB], e2[UB];
+            bool ok[UB];
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                const int k = (j0 + jj) * S + slot;
+                const int o = __shfl_sync(gmask, my, k & (RL - 1), RL);
+                ok[jj] = k < n && j0 + jj < L;
+                if (ok[jj]) {
+                    if (!DER) {
+                        const float* rec = a.D + (int64_t)o * a.ldd;
+                        load_chunks<VPL>(rec, col0, W, x[jj]);
+                        const float4 ax = ldg4(rec + aux0);
+                        e0[jj] = ax.x; e1[jj] = ax.y; e2[jj] = ax.z;
+                    } else {
+                        load_chunks<VPL>(a.T + (int64_t)o * a.ldt, col0, W, x[jj]);
+                        e0[jj] = __ldg(a.el + o);
+                        e1[jj] = 0.f; e2[jj] = 0.f;
+                    }
+                } else {
+#pragma unroll
+                    for (int i = 0; i < NV; ++i) x[jj][i] = 0.f;
+                    e0[jj] = 0.f; e1[jj] = INFINITY; e2[jj] = 0.f;
+                }
+            }
+#pragma unroll
+            for (int jj = 0; jj < UB; ++jj) {
+                float g = 0.f;
+#pragma unroll
+                for (int i = 0; i < NV; ++i) g = fmaf(x[jj][i], own[i], g);
+#pragma unroll
+                for (int o = 1; o < L; o <<= 1) g += __shfl_xor_sync(gmask, g, o, RL);
+                if (!ok[jj]) continue;
+                // s = el_u + er_v ; alpha = exp(LReLU(s) - lse_v) ; ds = alpha (g - c_v) LReLU'(s)
+                const float s = DER ? e0[jj] + k0 : k0 + e0[jj];
+                const float lse = DER ? k1 : e1[jj];
+                const float cv = DER ? k2 : e2[jj];
+                const float al = expf(lrelu(s, a.slope) - lse);
+                dsum += al * (g - cv) * (s > 0.f ? 1.f : a.slope);
+                if (!DER) {
+#pragma unroll
+                    for (int i = 0; i < NV; ++i) acc[i] = fmaf(al, x[jj][i], acc[i]);
+                }
+            }
+        }
+    }
+#pragma unroll
+    for (int o = L; o < RL; o <<= 1) {
+        if (!DER) {
+#pragma unroll
+            for (int i = 0; i < NV; ++i) acc[i] += __shfl_xor_sync(gmask, acc[i], o, RL);
+        }
+        dsum += __shfl_xor_sync(gmask, dsum, o, RL);
+    }
+    if (!valid || slot != 0) return;
+    if (DER) {
+        if (c == 0) a.der[w] = dsum;
+        return;
+    }
+    float* pd = a.dT + w * a.ldt;
+#pragma unroll
+    for (int q = 0; q < VPL; ++q) {
+        const int col = col0 + 4 * q;
+        if (col >= W) continue;
+        if (col + 4 <= W)
+            *reinterpret_cast<float4*>(pd + col) = make_float4(acc[4 * q], acc[4 * q + 1], acc[4 * q + 2], acc[4 * q + 3]);
+        else
+            for (int i = 0; i < 4 && col + i < W; ++i) pd[col + i] = acc[4 * q + i];
+    }
+    if (c == 0) a.del[w] = dsum;
+}
+
+// ============================================================================================
+// row kernels
+// ============================================================================================
 // thread per (u,h): el/er projections
 __global__ void k_gat_attn_proj(const float* __restrict__ T, int64_t M, int H, int F, int64_t ldt,
                                 const float* __restrict__ a_l, const float* __restrict__ a_r, float* __restrict__ el,
@@ -326,7 +844,9 @@ __global__ void k_gat_bwd_prep(int64_t M, int H, int F, int64_t ldt, const float
         rec[(int64_t)h * F + f] = d;
         cdot = fmaf(d, __ldg(A + o + f), cdot);
     }
-    float* aux = rec + (((int64_t)H * F + 3) & ~3LL) + 4 * h;
+    if (h == H - 1)   // zero the padding between dA and the aux block so vector loads read zeros
+        for (int64_t f = (int64_t)H * F; f < rec_aux_offset(H * F); ++f) rec[f] = 0.f;
+    float* aux = rec + rec_aux_offset(H * F) + 4 * h;
     aux[0] = __ldg(er + i);
     aux[1] = __ldg(lse + i);
     aux[2] = cdot;
@@ -389,28 +909,96 @@ static int64_t proj_bwd_blocks(int64_t M) {
     return b < 1 ? 1 : b;
 }
 
-template <int VEC, int L>
-static void gat_fwd_launch(GatFwdArgs a, int64_t split, int64_t n_rows, cudaStream_t s) {
-    GatFwdArgs hi = a, lo = a;
+// ============================================================================================
+// launch helpers
+// ============================================================================================
+// head-per-lane applies when every head row is whole float4s held by one lane
+static int hpl_f4(int H, int F, int64_t ldt, bool aligned) {
+    if (H < 2 || (32 % H) != 0 || (F % 4) != 0 || F > 32 || (ldt % 4) != 0 || !aligned) return 0;
+    return F / 4;
+}
+
+
+#define SS_HPL_SWITCH(KERNEL, f4, grid, s, args)                      \
+    switch (f4) {                                                     \
+        case 1: KERNEL<1><<<grid, 256, 0, s>>>(args); break;          \
+        case 2: KERNEL<2><<<grid, 256, 0, s>>>(args); break;          \
+        case 3: KERNEL<3><<<grid, 256, 0, s>>>(args); break;          \
+        case 4: KERNEL<4><<<grid, 256, 0, s>>>(args); break;          \
+        case 5: KERNEL<5><<<grid, 256, 0, s>>>(args); break;          \
+        case 6: KERNEL<6><<<grid, 256, 0, s>>>(args); break;          \
+        case 7: KERNEL<7><<<grid, 256, 0, s>>>(args); break;          \
+        default: KERNEL<8><<<grid, 256, 0, s>>>(args); break;         \
+    }
+
+#define SS_CHUNK_SWITCH(KERNEL, VEC, L, RL, grid, s, args)            \
+    switch (L) {                                                      \
+        case 1: KERNEL<VEC, 1, (RL < 4 ? 4 : RL)><<<grid, 256, 0, s>>>(args); break; \
+        case 2: KERNEL<VEC, 2, (RL < 4 ? 4 : RL)><<<grid, 256, 0, s>>>(args); break; \
+        case 4: KERNEL<VEC, 4, RL><<<grid, 256, 0, s>>>(args); break; \
+        case 8: KERNEL<VEC, 8, RL><<<grid, 256, 0, s>>>(args); break; \
+        case 16: KERNEL<VEC, 16, RL><<<grid, 256, 0, s>>>(args); break; \
+        default: KERNEL<VEC, 32, 32><<<grid, 256, 0, s>>>(args); break; \
+    }
+
+// chunked launches over the two degree classes: warp rows (RL = 32) and sub-warp rows (RL = L)
+template <typename Args, typename LaunchWarp, typename LaunchSub>
+static void two_buckets(Args a, int64_t split, int64_t n_rows, int L, LaunchWarp lw, LaunchSub ls) {
+    Args hi = a, lo = a;
     hi.row_begin = 0; hi.row_end = split;
     lo.row_begin = split; lo.row_end = n_rows;
-    if (split > 0) k_gat_fwd<VEC, L, 32><<<(unsigned)((split + 7) / 8), 256, 0, s>>>(hi);
+    if (split > 0) lw(hi, (unsigned)((split + 7) / 8));
     if (n_rows > split) {
-        constexpr int RL = L < 4 ? 4 : L;
+        const int RL = L < 4 ? 4 : L;
         const int64_t per = 256 / RL;
-        k_gat_fwd<VEC, L, RL><<<(unsigned)((n_rows - split + per - 1) / per), 256, 0, s>>>(lo);
+        ls(lo, (unsigned)((n_rows - split + per - 1) / per));
     }
 }
-template <int VEC, int L>
-static void gat_bwd_launch(GatBwdArgs a, int64_t split, int64_t n_rows, cudaStream_t s) {
-    GatBwdArgs hi = a, lo = a;
-    hi.row_begin = 0; hi.row_end = split;
-    lo.row_begin = split; lo.row_end = n_rows;
-    if (split > 0) k_gat_bwd<VEC, L, 32><<<(unsigned)((split + 7) / 8), 256, 0, s>>>(hi);
-    if (n_rows > split) {
-        constexpr int RL = L < 4 ? 4 : L;
-        const int64_t per = 256 / RL;
-        k_gat_bwd<VEC, L, RL><<<(unsigned)((n_rows - split + per - 1) / per), 256, 0, s>>>(lo);
+
+// single-head path: VPL chunks per lane (from {1,2,3,4,6,8}) and L = pow2 lanes per edge (<= 4)
+static bool h1_geometry(int H, int F, int64_t ldt, bool aligned, int& vpl, int& L) {
+    if (H != 1 || (ldt % 4) != 0 || !aligned || F > 128) return false;
+    const int C = (F + 3) / 4;
+    int v = (C + 3) / 4;
+    v = v <= 4 ? v : (v <= 6 ? 6 : 8);
+    vpl = v;
+    L = pow2_ceil((C + v - 1) / v);
+    return L <= 4;
+}
+
+struct FwdH1 {
+    template <int VPL, int L>
+    static void run(const GatFwdArgs& a, int64_t split, int64_t n, cudaStream_t s) {
+        two_buckets(a, split, n, 4, [&](GatFwdArgs x, unsigned grid) { k_gat_fwd_h1<VPL, L, 32><<<grid, 256, 0, s>>>(x); },
+                    [&](GatFwdArgs x, unsigned grid) { k_gat_fwd_h1<VPL, L, 4><<<grid, 256, 0, s>>>(x); });
+    }
+};
+template <bool DER>
+struct BwdH1 {
+    template <int VPL, int L>
+    static void run(const GatBwdArgs& a, int64_t split, int64_t n, cudaStream_t s) {
+        two_buckets(a, split, n, 4,
+                    [&](GatBwdArgs x, unsigned grid) { k_gat_bwd_h1<VPL, L, 32, DER><<<grid, 256, 0, s>>>(x); },
+                    [&](GatBwdArgs x, unsigned grid) { k_gat_bwd_h1<VPL, L, 4, DER><<<grid, 256, 0, s>>>(x); });
+    }
+};
+template <class K, int VPL, class Args>
+static void dispatch_h1_L(int L, const Args& a, int64_t split, int64_t n, cudaStream_t s) {
+    switch (L) {
+        case 1: K::template run<VPL, 1>(a, split, n, s); break;
+        case 2: K::template run<VPL, 2>(a, split, n, s); break;
+        default: K::template run<VPL, 4>(a, split, n, s); break;
+    }
+}
+template <class K, class Args>
+static void dispatch_h1(int vpl, int L, const Args& a, int64_t split, int64_t n, cudaStream_t s) {
+    switch (vpl) {
+        case 1: dispatch_h1_L<K, 1>(L, a, split, n, s); break;
+        case 2: dispatch_h1_L<K, 2>(L, a, split, n, s); break;
+        case 3: dispatch_h1_L<K, 3>(L, a, split, n, s); break;
+        case 4: dispatch_h1_L<K, 4>(L, a, split, n, s); break;
+        case 6: dispatch_h1_L<K, 6>(L, a, split, n, s); break;
+        default: dispatch_h1_L<K, 8>(L, a, split, n, s); break;
     }
 }
 
@@ -418,15 +1006,35 @@ static void gat_bwd_launch(GatBwdArgs a, int64_t split, int64_t n_rows, cudaStre
 
 using namespace seastar;
 
-#define GAT_DISPATCH(FN, VEC, L, ...)          \
-    switch (L) {                               \
-        case 1: FN<VEC, 1>(__VA_ARGS__); break;  \
-        case 2: FN<VEC, 2>(__VA_ARGS__); break;  \
-        case 4: FN<VEC, 4>(__VA_ARGS__); break;  \
-        case 8: FN<VEC, 8>(__VA_ARGS__); break;  \
-        case 16: FN<VEC, 16>(__VA_ARGS__); break; \
-        default: FN<VEC, 32>(__VA_ARGS__); break; \
-    }
+#define CHUNK_LAUNCH(KERNEL, ARGS, SPLIT, NROWS, L, VEC4, S)                                                     \
+    do {                                                                                                         \
+        auto lw = [&](decltype(ARGS) x, unsigned grid) {                                                         \
+            if (VEC4) { SS_CHUNK_SWITCH(KERNEL, 4, L, 32, grid, S, x); }                                         \
+            else { SS_CHUNK_SWITCH(KERNEL, 1, L, 32, grid, S, x); }                                              \
+        };                                                                                                       \
+        auto ls = [&](decltype(ARGS) x, unsigned grid) {                                                         \
+            if (VEC4) {                                                                                          \
+                switch (L) {                                                                                     \
+                    case 1: KERNEL<4, 1, 4><<<grid, 256, 0, S>>>(x); break;                                      \
+                    case 2: KERNEL<4, 2, 4><<<grid, 256, 0, S>>>(x); break;                                      \
+                    case 4: KERNEL<4, 4, 4><<<grid, 256, 0, S>>>(x); break;                                      \
+                    case 8: KERNEL<4, 8, 8><<<grid, 256, 0, S>>>(x); break;                                      \
+                    case 16: KERNEL<4, 16, 16><<<grid, 256, 0, S>>>(x); break;                                   \
+                    default: KERNEL<4, 32, 32><<<grid, 256, 0, S>>>(x); break;                                   \
+                }                                                                                                \
+            } else {                                                                                             \
+                switch (L) {                                                                                     \
+                    case 1: KERNEL<1, 1, 4><<<grid, 256, 0, S>>>(x); break;                                      \
+                    case 2: KERNEL<1, 2, 4><<<grid, 256, 0, S>>>(x); break;                                      \
+                    case 4: KERNEL<1, 4, 4><<<grid, 256, 0, S>>>(x); break;                                      \
+                    case 8: KERNEL<1, 8, 8><<<grid, 256, 0, S>>>(x); break;                                      \
+                    case 16: KERNEL<1, 16, 16><<<grid, 256, 0, S>>>(x); break;                                   \
+                    default: KERNEL<1, 32, 32><<<grid, 256, 0, S>>>(x); break;                                   \
+                }                                                                                                \
+            }                                                                                                    \
+        };                                                                                                       \
+        two_buckets(ARGS, (L) >= 32 ? (NROWS) : (SPLIT), NROWS, L, lw, ls);                                      \
+    } while (0)
 
 extern "C" {
 
@@ -450,22 +1058,32 @@ seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float*
     SS_ARG(H >= 1 && F >= 1 && ldt >= (int64_t)H * F, "gat_fwd: bad sizes H=%d F=%d ldt=%lld", H, F, (long long)ldt);
     SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "gat_fwd: bad activation");
     SS_TRY(check_device());
-    const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_all) && aligned16(A_loc) &&
-                      aligned16(Y_loc);
-    const int VEC = vec4 ? 4 : 1;
-    const int C = (H * F + VEC - 1) / VEC;
-    SS_ARG(C <= 32, "gat_fwd: row of H*F=%d floats exceeds 32 lanes x %d", H * F, VEC);
-    const int L = pow2_ceil(C);
+    cudaStream_t s = to_stream(stream);
     GatFwdArgs a{};
     a.perm = g->fwd.perm; a.off = g->fwd.off; a.nbr = g->fwd.nbr;
     a.vbase = g->row_begin;
     a.T = T_all; a.el = el_all; a.er = er_loc;
     a.H = H; a.F = F; a.ld = ldt; a.slope = slope; a.bias = bias; a.act = act;
     a.A = A_loc; a.Y = Y_loc; a.lse = lse_loc;
-    const int64_t split = L >= 32 ? g->fwd.n_rows : g->fwd.bucket_rows[1];
-    cudaStream_t s = to_stream(stream);
-    if (vec4) { GAT_DISPATCH(gat_fwd_launch, 4, L, a, split, g->fwd.n_rows, s); }
-    else { GAT_DISPATCH(gat_fwd_launch, 1, L, a, split, g->fwd.n_rows, s); }
+    const int f4 = hpl_f4(H, F, ldt, aligned16(T_all) && aligned16(A_loc) && aligned16(Y_loc));
+    if (f4) {
+        a.row_begin = 0; a.row_end = g->fwd.n_rows;
+        const unsigned grid = (unsigned)((g->fwd.n_rows + 7) / 8);
+        if (grid) SS_HPL_SWITCH(k_gat_fwd_hpl, f4, grid, s, a);
+        return check_launch("k_gat_fwd_hpl");
+    }
+    int vpl = 0, Lh = 0;
+    if (h1_geometry(H, F, ldt, aligned16(T_all) && aligned16(A_loc) && aligned16(Y_loc), vpl, Lh)) {
+        dispatch_h1<FwdH1>(vpl, Lh, a, g->fwd.bucket_rows[1], g->fwd.n_rows, s);
+        return check_launch("k_gat_fwd_h1");
+    }
+    const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_all) && aligned16(A_loc) &&
+                      aligned16(Y_loc);
+    const int VEC = vec4 ? 4 : 1;
+    const int C = (H * F + VEC - 1) / VEC;
+    SS_ARG(C <= 32, "gat_fwd: row of H*F=%d floats exceeds 32 lanes x %d", H * F, VEC);
+    const int L = pow2_ceil(C);
+    CHUNK_LAUNCH(k_gat_fwd, a, g->fwd.bucket_rows[1], g->fwd.n_rows, L, vec4, s);
     return check_launch("k_gat_fwd");
 }
 
@@ -486,42 +1104,69 @@ seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const 
 
 seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float* el_loc, const float* D_all,
                                int32_t H, int32_t F, int64_t ldt, float slope, float* dT_loc, float* del_loc,
-                               float* ds_work, seastar_stream stream) {
-    SS_ARG(g && T_loc && el_loc && D_all && dT_loc && del_loc && ds_work, "gat_bwd: NULL argument");
+                               seastar_stream stream) {
+    SS_ARG(g && T_loc && el_loc && D_all && dT_loc && del_loc, "gat_bwd: NULL argument");
     SS_ARG(H >= 1 && F >= 1 && ldt >= (int64_t)H * F, "gat_bwd: bad sizes");
     SS_TRY(check_device());
-    const int64_t ldd = seastar_gat_record_ld(H, F);
+    cudaStream_t s = to_stream(stream);
+    GatBwdArgs a{};
+    a.perm = g->rev.perm; a.off = g->rev.off; a.nbr = g->rev.nbr;
+    a.vbase = g->row_begin;
+    a.T = T_loc; a.el = el_loc; a.D = D_all;
+    a.H = H; a.F = F; a.ldt = ldt; a.ldd = seastar_gat_record_ld(H, F); a.slope = slope;
+    a.dT = dT_loc; a.del = del_loc;
+    const int f4 = hpl_f4(H, F, ldt, aligned16(T_loc) && aligned16(D_all) && aligned16(dT_loc));
+    if (f4) {
+        a.row_begin = 0; a.row_end = g->rev.n_rows;
+        const unsigned grid = (unsigned)((g->rev.n_rows + 7) / 8);
+        if (grid) SS_HPL_SWITCH(k_gat_bwd_hpl, f4, grid, s, a);
+        return check_launch("k_gat_bwd_hpl");
+    }
+    int vpl = 0, Lh = 0;
+    if (h1_geometry(H, F, ldt, aligned16(T_loc) && aligned16(D_all) && aligned16(dT_loc), vpl, Lh)) {
+        dispatch_h1<BwdH1<false>>(vpl, Lh, a, g->rev.bucket_rows[1], g->rev.n_rows, s);
+        return check_launch("k_gat_bwd_h1");
+    }
     const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_loc) && aligned16(D_all) &&
                       aligned16(dT_loc);
     const int VEC = vec4 ? 4 : 1;
     const int C = (H * F + VEC - 1) / VEC;
     SS_ARG(C <= 32, "gat_bwd: row of H*F=%d floats exceeds 32 lanes x %d", H * F, VEC);
     const int L = pow2_ceil(C);
-    GatBwdArgs a{};
-    a.perm = g->rev.perm; a.off = g->rev.off; a.nbr = g->rev.nbr; a.pos = g->rev.pos;
-    a.vbase = g->row_begin;
-    a.T = T_loc; a.el = el_loc; a.D = D_all;
-    a.H = H; a.F = F; a.ldt = ldt; a.ldd = ldd; a.slope = slope;
-    a.dT = dT_loc; a.del = del_loc; a.ds = ds_work;
-    const int64_t split = L >= 32 ? g->rev.n_rows : g->rev.bucket_rows[1];
-    cudaStream_t s = to_stream(stream);
-    if (vec4) { GAT_DISPATCH(gat_bwd_launch, 4, L, a, split, g->rev.n_rows, s); }
-    else { GAT_DISPATCH(gat_bwd_launch, 1, L, a, split, g->rev.n_rows, s); }
+    CHUNK_LAUNCH(k_gat_bwd, a, g->rev.bucket_rows[1], g->rev.n_rows, L, vec4, s);
     return check_launch("k_gat_bwd");
 }
 
-seastar_status seastar_gat_der(seastar_graph g, const float* ds_work, int32_t H, float* der, seastar_stream stream) {
-    SS_ARG(g && ds_work && der, "gat_der: NULL argument");
-    SS_ARG(H >= 1, "gat_der: bad H");
+seastar_status seastar_gat_der(seastar_graph g, const float* T_all, const float* el_all, const float* D_loc, int32_t H,
+                               int32_t F, int64_t ldt, float slope, float* der_loc, seastar_stream stream) {
+    SS_ARG(g && T_all && el_all && D_loc && der_loc, "gat_der: NULL argument");
+    SS_ARG(H >= 1 && F >= 1 && ldt >= (int64_t)H * F, "gat_der: bad sizes");
     SS_TRY(check_device());
     cudaStream_t s = to_stream(stream);
-    if (!g->partitioned) {
-        const int64_t n = g->fwd.n_rows;
-        if (n) k_gat_der<<<(unsigned)((n + 7) / 8), 256, 0, s>>>(g->fwd.perm, g->fwd.off, n, g->row_begin, ds_work, H, der);
-    } else {
-        const int64_t n = g->lsf.n_rows;
-        if (n) k_gat_der<<<(unsigned)((n + 7) / 8), 256, 0, s>>>(nullptr, g->lsf.off, n, 0, ds_work, H, der);
+    GatBwdArgs a{};
+    a.perm = g->fwd.perm; a.off = g->fwd.off; a.nbr = g->fwd.nbr;
+    a.vbase = g->row_begin;
+    a.T = T_all; a.el = el_all; a.D = D_loc;
+    a.H = H; a.F = F; a.ldt = ldt; a.ldd = seastar_gat_record_ld(H, F); a.slope = slope;
+    a.der = der_loc;
+    const int f4 = hpl_f4(H, F, ldt, aligned16(T_all) && aligned16(D_loc));
+    if (f4) {
+        a.row_begin = 0; a.row_end = g->fwd.n_rows;
+        const unsigned grid = (unsigned)((g->fwd.n_rows + 7) / 8);
+        if (grid) SS_HPL_SWITCH(k_gat_der_hpl, f4, grid, s, a);
+        return check_launch("k_gat_der_hpl");
     }
+    int vpl = 0, Lh = 0;
+    if (h1_geometry(H, F, ldt, aligned16(T_all) && aligned16(D_loc), vpl, Lh)) {
+        dispatch_h1<BwdH1<true>>(vpl, Lh, a, g->fwd.bucket_rows[1], g->fwd.n_rows, s);
+        return check_launch("k_gat_der_h1");
+    }
+    const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_all) && aligned16(D_loc);
+    const int VEC = vec4 ? 4 : 1;
+    const int C = (H * F + VEC - 1) / VEC;
+    SS_ARG(C <= 32, "gat_der: row of H*F=%d floats exceeds 32 lanes x %d", H * F, VEC);
+    const int L = pow2_ceil(C);
+    CHUNK_LAUNCH(k_gat_der, a, g->fwd.bucket_rows[1], g->fwd.n_rows, L, vec4, s);
     return check_launch("k_gat_der");
 }
 

@@ -216,12 +216,7 @@ class GAT2:
         self.D1, self.D2 = e(n, self.ldd1), e(n, self.ldd2)
         self.dT1, self.dT2 = e(n, self.ld1), e(n, self.ld2)
         self.del1, self.del2 = e(n, heads), e(n, 1)
-        self.der1, self.der2 = e(self.rows_all if self.comm.world > 1 else n, heads), \
-            e(self.rows_all if self.comm.world > 1 else n, 1)
-        self.der1_loc, self.der2_loc = (e(n, heads), e(n, 1)) if self.comm.world > 1 else (self.der1, self.der2)
-        n_ds = g.info["num_rev_edges"]
-        self.ds1 = torch.zeros((max(n_ds, 1), heads), device=dev)
-        self.ds2 = torch.zeros((max(n_ds, 1), 1), device=dev)
+        self.der1, self.der2 = e(n, heads), e(n, 1)
         self.dY1 = e(n, self.ld1)
         self.loss = torch.zeros(1, device=dev)
         self.ws = _Ws(dev)
@@ -247,6 +242,7 @@ class GAT2:
         L.seastar_gat_attn_proj(self.T1, n, H, F, self.ld1, p.p("al1"), p.p("ar1"), self.el1, self.er1)
         T1_all = self.comm.all_gather(self.T1_all, self.T1)
         el1_all = self.comm.all_gather(self.el1_all, self.el1)
+        self._gathered1 = (T1_all, el1_all)
         self._t("gat_fwd1")
         L.seastar_gat_fwd(g.handle, T1_all, el1_all, self.er1, H, F, self.ld1, self.slope, p.p("b1"), "elu", self.A1,
                           self.Y1, self.lse1)
@@ -255,13 +251,14 @@ class GAT2:
         L.seastar_gat_attn_proj(self.T2, n, 1, C, self.ld2, p.p("al2"), p.p("ar2"), self.el2, self.er2)
         T2_all = self.comm.all_gather(self.T2_all, self.T2)
         el2_all = self.comm.all_gather(self.el2_all, self.el2)
+        self._gathered2 = (T2_all, el2_all)
         L.seastar_gat_fwd(g.handle, T2_all, el2_all, self.er2, 1, C, self.ld2, self.slope, p.p("b2"), "none", self.A2,
                           self.Y2, self.lse2)
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
         L.seastar_softmax_xent(self.Y2, n, C, self.ld2, self.lab, self.loss, self.dY2, self.ld2, ws, ws.numel())
         return self.loss
 
-    def _layer_bwd(self, T, T_loc_ld, el, er, A, Y, lse, dY, act, H, F, D, D_all_buf, dT, del_, der, der_loc, ds,
+    def _layer_bwd(self, T, T_loc_ld, el, er, A, Y, lse, dY, act, H, F, D, D_all_buf, dT, del_, der, gathered,
                    al, ar, dal, dar, db, tag):
         g, n = self.g, self.n
         L.seastar_gat_bwd_prep(g.handle, dY, Y, act, A, er, lse, H, F, T_loc_ld, D)
@@ -270,24 +267,25 @@ class GAT2:
         L.seastar_colsum(D, n, H * F, ldd, db, ws, ws.numel())       # db = sum_v dA[v] (dA = first H*F columns)
         D_all = self.comm.all_gather(D_all_buf, D)
         self._t(f"gat_bwd{tag}")
-        L.seastar_gat_bwd(g.handle, T, el, D_all, H, F, T_loc_ld, self.slope, dT, del_, ds)
+        L.seastar_gat_bwd(g.handle, T, el, D_all, H, F, T_loc_ld, self.slope, dT, del_)
         self._t(f"gat_bwd{tag}_end")
-        L.seastar_gat_der(g.handle, ds, H, der)
-        der_l = self.comm.reduce_scatter(der_loc, der)
-        L.seastar_gat_attn_proj_bwd(T, n, H, F, T_loc_ld, al, ar, del_, der_l, dT, dal, dar, ws, ws.numel())
+        self._t(f"gat_der{tag}")
+        L.seastar_gat_der(g.handle, gathered[0], gathered[1], D, H, F, T_loc_ld, self.slope, der)
+        self._t(f"gat_der{tag}_end")
+        L.seastar_gat_attn_proj_bwd(T, n, H, F, T_loc_ld, al, ar, del_, der, dT, dal, dar, ws, ws.numel())
 
     def backward(self):
         p, n = self.P, self.n
         H, F, W, C = self.H1, self.F1, self.W1w, self.C
         self._layer_bwd(self.T2, self.ld2, self.el2, self.er2, self.A2, self.Y2, self.lse2, self.dY2, "none", 1, C,
-                        self.D2, self.D2_all, self.dT2, self.del2, self.der2, self.der2_loc, self.ds2, p.p("al2"),
+                        self.D2, self.D2_all, self.dT2, self.del2, self.der2, self._gathered2, p.p("al2"),
                         p.p("ar2"), p.g("al2"), p.g("ar2"), p.g("b2"), "2")
         ws = self.ws.need(max(L.seastar_linear_bwd_weight_workspace(n, W, C),
                               L.seastar_linear_bwd_weight_workspace(n, self.Fin, W)))
         L.seastar_linear_bwd_weight(self.Y1, n, W, self.ld1, self.dT2, C, self.ld2, p.g("W2"), None, ws, ws.numel())
         L.seastar_linear_bwd_data(self.dT2, n, C, self.ld2, p.p("W2"), W, None, None, "none", self.dY1, self.ld1)
         self._layer_bwd(self.T1, self.ld1, self.el1, self.er1, self.A1, self.Y1, self.lse1, self.dY1, "elu", H, F,
-                        self.D1, self.D1_all, self.dT1, self.del1, self.der1, self.der1_loc, self.ds1, p.p("al1"),
+                        self.D1, self.D1_all, self.dT1, self.del1, self.der1, self._gathered1, p.p("al1"),
                         p.p("ar1"), p.g("al1"), p.g("ar1"), p.g("b1"), "1")
         ws = self.ws.need(L.seastar_linear_bwd_weight_workspace(n, self.Fin, W))
         L.seastar_linear_bwd_weight(self.X, n, self.Fin, self.X.stride(0), self.dT1, W, self.ld1, p.g("W1"), None, ws,
