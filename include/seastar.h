@@ -280,8 +280,10 @@ seastar_status seastar_rgcn_fwd(seastar_graph g, const float* X_all, int64_t F_i
  */
 seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_in, int64_t ldx,
                                 const float* dA_all, int64_t F_out, int64_t ldd, const float* W,
-                                const float* norm_user, float* dX_loc, float* dW, void* workspace,
-                                size_t ws_bytes, seastar_stream stream);
+                                const float* norm_user, const float* Yact_loc, seastar_act act, float* dX_loc,
+                                float* dW, void* workspace, size_t ws_bytes, seastar_stream stream);
+/* (Yact_loc [n_loc,F_in] ld ldx or NULL: dX_loc is multiplied by act'(Yact_loc), fusing the input
+ *  layer's activation backward; act is ignored when Yact_loc is NULL.) */
 size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out);
 
 /* ------------------------------------------------------------------------------------------ */

@@ -74,7 +74,7 @@ _SIGS = {
     "seastar_gat_attn_proj_bwd": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P, _P, _P, _P, _SZ, _P], _ST),
     "seastar_gat_attn_proj_bwd_workspace": ([_I64, _I32, _I32], _SZ),
     "seastar_rgcn_fwd": ([_P, _P, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
-    "seastar_rgcn_bwd": ([_P, _P, _I64, _I64, _P, _I64, _I64, _P, _P, _P, _P, _P, _SZ, _P], _ST),
+    "seastar_rgcn_bwd": ([_P, _P, _I64, _I64, _P, _I64, _I64, _P, _P, _P, _I32, _P, _P, _P, _SZ, _P], _ST),
     "seastar_rgcn_bwd_workspace": ([_P, _I64, _I64], _SZ),
     "seastar_softmax_xent": ([_P, _I64, _I32, _I64, _P, _P, _P, _I64, _P, _SZ, _P], _ST),
     "seastar_softmax_xent_workspace": ([_I64], _SZ),
@@ -284,11 +284,11 @@ def seastar_rgcn_bwd_workspace(g, F_in, F_out) -> int:
     return int(load().seastar_rgcn_bwd_workspace(g, F_in, F_out))
 
 
-def seastar_rgcn_bwd(g, X_all, F_in, ldx, dA_all, F_out, ldd, W, norm_user, dX_loc, dW, workspace, ws_bytes,
-                     stream=None) -> None:
+def seastar_rgcn_bwd(g, X_all, F_in, ldx, dA_all, F_out, ldd, W, norm_user, Yact_loc, act, dX_loc, dW, workspace,
+                     ws_bytes, stream=None) -> None:
     _call("seastar_rgcn_bwd", g, _dptr(X_all, "X"), F_in, ldx, _dptr(dA_all, "dA"), F_out, ldd, _dptr(W, "W"),
-          _dptr(norm_user, "norm"), _dptr(dX_loc, "dX"), _dptr(dW, "dW"), _dptr(workspace, "workspace"), ws_bytes,
-          _stream(stream))
+          _dptr(norm_user, "norm"), _dptr(Yact_loc, "Yact"), _act(act), _dptr(dX_loc, "dX"), _dptr(dW, "dW"),
+          _dptr(workspace, "workspace"), ws_bytes, _stream(stream))
 
 
 # ----------------------------------------------------------------------------------- glue

@@ -26,6 +26,7 @@ struct RgcnRowArgs {
     int transpose;                      // 0: forward (g W_r), 1: dX (q W_r^T)
     float* out; int64_t ldo;
     const float* bias; int act;
+    const float* Yact;                  // dX only: fused activation backward, out *= act'(Yact)
 };
 
 // stage W (or W^T) as [R][Fg][Fop] with Fop = round4(Fo), zero padded
@@ -156,6 +157,7 @@ __global__ void __launch_bounds__(512) k_rgcn_rows(const RgcnRowArgs a) {
                 if (j < a.Fo) {
                     float z = out[q];
                     if (!a.transpose) z = act_apply(a.act, z + (a.bias ? __ldg(a.bias + j) : 0.f));
+                    else if (a.Yact) z *= act_grad_from_y(a.act, __ldg(a.Yact + v * a.ldo + j));
                     po[q] = z;
                 }
             }
@@ -316,9 +318,11 @@ size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out) 
 }
 
 seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_in, int64_t ldx, const float* dA_all,
-                                int64_t F_out, int64_t ldd, const float* W, const float* norm_user, float* dX_loc,
-                                float* dW, void* workspace, size_t ws_bytes, seastar_stream stream) {
+                                int64_t F_out, int64_t ldd, const float* W, const float* norm_user,
+                                const float* Yact_loc, seastar_act act, float* dX_loc, float* dW, void* workspace,
+                                size_t ws_bytes, seastar_stream stream) {
     SS_ARG(g && X_all && dA_all && W, "rgcn_bwd: NULL argument");
+    SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "rgcn_bwd: bad activation");
     SS_ARG(dX_loc || dW, "rgcn_bwd: nothing to compute");
     SS_ARG(F_in >= 1 && F_in <= 64 && F_out >= 1 && F_out <= 64, "rgcn_bwd: need 1 <= F_in, F_out <= 64");
     SS_ARG(F_in * F_out <= 32 * 32, "rgcn_bwd: F_in * F_out <= 1024 required for the register dW path");
@@ -336,7 +340,7 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
         a.norm = g->rev.norm; a.eid = g->rev.eid; a.norm_user = norm_user;
         a.vbase = g->row_begin;
         a.table = dA_all; a.ldt = ldd; a.W = W; a.R = g->R; a.Fg = (int)F_out; a.Fo = (int)F_in; a.transpose = 1;
-        a.out = dX_loc; a.ldo = ldx; a.bias = nullptr; a.act = SEASTAR_ACT_NONE;
+        a.out = dX_loc; a.ldo = ldx; a.bias = nullptr; a.act = act; a.Yact = Yact_loc;
         SS_TRY(launch_rows_L(g->rev, a, s));
     }
     if (dW) {

@@ -383,3 +383,68 @@ class APPNPNet:
         self.backward()
         self.P.adam(self.lr)
         return loss
+
+
+class RGCN2:
+    """2-layer R-GCN [53] (§6.3.5): F_in -> hidden (ReLU) -> C, one weight matrix per
+    relation, normaliser 1/c_{v,r} (graph built with rgcn_norm=True), softmax-xent."""
+
+    def __init__(self, g: Graph, X_loc, labels_loc, params: dict, lr=0.01, comm: Comm | None = None,
+                 n_pad_rows: int | None = None):
+        self.g, self.X, self.lab, self.lr = g, X_loc, labels_loc, lr
+        self.comm = comm or Comm()
+        dev = X_loc.device
+        self.n = g.n_loc
+        self.rows_all = n_pad_rows if n_pad_rows is not None else g.N
+        R, self.Fin, self.Hd = params["W1"].shape
+        self.C = params["W2"].shape[2]
+        assert X_loc.stride(0) % 4 == 0, "R-GCN input rows need a leading dimension that is a multiple of 4"
+        self.P = _Params({"W1": params["W1"].shape, "b1": (self.Hd,), "W2": params["W2"].shape, "b2": (self.C,)},
+                         params, dev)
+        n = self.n
+        self.ldh, self.ldc = _ld(self.Hd), _ld(self.C)
+        e = lambda r, c: torch.zeros((r, c), device=dev)
+        self.H1, self.dZ1 = e(n, self.ldh), e(n, self.ldh)
+        self.logits, self.dlog = e(n, self.ldc), e(n, self.ldc)
+        self.loss = torch.zeros(1, device=dev)
+        self.ws = _Ws(dev)
+        P, Ra = self.comm.world, self.rows_all
+        self.X_all = e(Ra, X_loc.stride(0)) if P > 1 else None
+        self.H1_all = e(Ra, self.ldh) if P > 1 else None
+        self.dlog_all = e(Ra, self.ldc) if P > 1 else None
+        self.dZ1_all = e(Ra, self.ldh) if P > 1 else None
+        self.timer = None
+
+    def forward(self):
+        g, p, n = self.g, self.P, self.n
+        self._X_all = self.comm.all_gather(self.X_all, self.X)
+        L.seastar_rgcn_fwd(g.handle, self._X_all, self.Fin, self.X.stride(0), p.p("W1"), self.Hd, None, p.p("b1"),
+                           "relu", self.H1, self.ldh)
+        self._H1_all = self.comm.all_gather(self.H1_all, self.H1)
+        L.seastar_rgcn_fwd(g.handle, self._H1_all, self.Hd, self.ldh, p.p("W2"), self.C, None, p.p("b2"), "none",
+                           self.logits, self.ldc)
+        ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
+        L.seastar_softmax_xent(self.logits, n, self.C, self.ldc, self.lab, self.loss, self.dlog, self.ldc, ws,
+                               ws.numel())
+        return self.loss
+
+    def backward(self):
+        g, p, n = self.g, self.P, self.n
+        ws = self.ws.need(max(L.seastar_rgcn_bwd_workspace(g.handle, self.Hd, self.C),
+                              L.seastar_rgcn_bwd_workspace(g.handle, self.Fin, self.Hd),
+                              L.seastar_colsum_workspace(n, max(self.C, self.Hd))))
+        L.seastar_colsum(self.dlog, n, self.C, self.ldc, p.g("b2"), ws, ws.numel())
+        dlog_all = self.comm.all_gather(self.dlog_all, self.dlog)
+        L.seastar_rgcn_bwd(g.handle, self._H1_all, self.Hd, self.ldh, dlog_all, self.C, self.ldc, p.p("W2"), None,
+                           self.H1, "relu", self.dZ1, p.g("W2"), ws, ws.numel())
+        L.seastar_colsum(self.dZ1, n, self.Hd, self.ldh, p.g("b1"), ws, ws.numel())
+        dZ1_all = self.comm.all_gather(self.dZ1_all, self.dZ1)
+        L.seastar_rgcn_bwd(g.handle, self._X_all, self.Fin, self.X.stride(0), dZ1_all, self.Hd, self.ldh, p.p("W1"),
+                           None, None, "none", None, p.g("W1"), ws, ws.numel())
+        self.comm.all_reduce(self.P.grad)
+
+    def epoch(self):
+        loss = self.forward()
+        self.backward()
+        self.P.adam(self.lr)
+        return loss

@@ -1,0 +1,82 @@
+"""Whole-model references composed from the pinned oracle functions (test infrastructure).
+
+Each function returns (loss, grads) for one forward + backward of the paper's models with the
+readings of DESIGN.md §3; the GPU models in paper_conf_eurosys_wumcjlzcy21_b200.models must match
+them parameter by parameter."""
+import numpy as np
+
+import oracle
+
+
+def gcn2(ip, ix, X, lab, p):
+    in_n, out_n = oracle.degree_norms(ip, ix)
+    T = oracle.linear_fwd(X, p["W1"])
+    Z1 = oracle.gcn_aggregate(ip, ix, T, out_n, in_n) + p["b1"]
+    H1 = oracle.act_fwd("relu", Z1)
+    P2 = oracle.gcn_aggregate(ip, ix, H1, out_n, in_n)
+    logits = oracle.linear_fwd(P2, p["W2"], p["b2"])
+    loss, dlog = oracle.softmax_xent(logits, lab)
+    dP2, dW2, db2 = oracle.linear_bwd(P2, p["W2"], dlog)
+    dH1 = oracle.gcn_aggregate_T(ip, ix, dP2, out_n, in_n)
+    dZ1 = oracle.act_bwd("relu", Z1, dH1)
+    db1 = dZ1.sum(0)
+    dT = oracle.gcn_aggregate_T(ip, ix, dZ1, out_n, in_n)
+    _, dW1, _ = oracle.linear_bwd(X, p["W1"], dT, need_dX=False, need_db=False)
+    return loss, {"W1": dW1, "b1": db1, "W2": dW2, "b2": db2}
+
+
+def _gat_layer_fwd(ip, ix, Xin, W, al, ar, b, act, H, F):
+    N = Xin.shape[0]
+    T = oracle.linear_fwd(Xin, W).reshape(N, H, F)
+    el, er = oracle.gat_attn_proj(T, al, ar)
+    A, _, _ = oracle.gat_fwd(ip, ix, T, el, er, 0.2)
+    Z = A.reshape(N, H * F) + b
+    return T, el, er, Z, oracle.act_fwd(act, Z)
+
+
+def _gat_layer_bwd(ip, ix, Xin, W, al, ar, T, el, er, Z, act, dY, H, F, need_dX):
+    N = Xin.shape[0]
+    dZ = oracle.act_bwd(act, Z, dY)
+    db = dZ.sum(0)
+    dT, dl, dr = oracle.gat_bwd(ip, ix, T, el, er, dZ.reshape(N, H, F), 0.2)
+    dTp, dal, dar = oracle.gat_attn_proj_bwd(T, al, ar, dl, dr)
+    dTt = (dT + dTp).reshape(N, H * F)
+    dX, dW, _ = oracle.linear_bwd(Xin, W, dTt, need_dX=need_dX, need_db=False)
+    return dX, dW, dal, dar, db
+
+
+def gat2(ip, ix, X, lab, p, heads, hidden):
+    C = p["W2"].shape[1]
+    T1, el1, er1, Z1, Y1 = _gat_layer_fwd(ip, ix, X, p["W1"], p["al1"], p["ar1"], p["b1"], "elu", heads, hidden)
+    T2, el2, er2, Z2, Y2 = _gat_layer_fwd(ip, ix, Y1, p["W2"], p["al2"], p["ar2"], p["b2"], "none", 1, C)
+    loss, dY2 = oracle.softmax_xent(Y2, lab)
+    dY1, dW2, dal2, dar2, db2 = _gat_layer_bwd(ip, ix, Y1, p["W2"], p["al2"], p["ar2"], T2, el2, er2, Z2, "none",
+                                               dY2, 1, C, True)
+    _, dW1, dal1, dar1, db1 = _gat_layer_bwd(ip, ix, X, p["W1"], p["al1"], p["ar1"], T1, el1, er1, Z1, "elu", dY1,
+                                             heads, hidden, False)
+    return loss, {"W1": dW1, "al1": dal1, "ar1": dar1, "b1": db1, "W2": dW2, "al2": dal2, "ar2": dar2, "b2": db2}
+
+
+def appnp(ip, ix, X, lab, p, K, alpha):
+    Z1 = oracle.linear_fwd(X, p["W1"], p["b1"])
+    Hh = oracle.act_fwd("relu", Z1)
+    H0 = oracle.linear_fwd(Hh, p["W2"], p["b2"])
+    Z = oracle.appnp_fwd(ip, ix, H0, K, alpha)
+    loss, dZ = oracle.softmax_xent(Z, lab)
+    dH0 = oracle.appnp_bwd(ip, ix, dZ, K, alpha)
+    dHh, dW2, db2 = oracle.linear_bwd(Hh, p["W2"], dH0)
+    dZ1 = oracle.act_bwd("relu", Z1, dHh)
+    _, dW1, db1 = oracle.linear_bwd(X, p["W1"], dZ1, need_dX=False)
+    return loss, {"W1": dW1, "b1": db1, "W2": dW2, "b2": db2}
+
+
+def rgcn2(ip, ix, et, X, lab, p):
+    Z1 = oracle.rgcn_fwd(ip, ix, et, X, p["W1"]) + p["b1"]
+    H1 = oracle.act_fwd("relu", Z1)
+    Z2 = oracle.rgcn_fwd(ip, ix, et, H1, p["W2"]) + p["b2"]
+    loss, dZ2 = oracle.softmax_xent(Z2, lab)
+    dH1, dW2 = oracle.rgcn_bwd(ip, ix, et, H1, p["W2"], dZ2)
+    db2 = dZ2.sum(0)
+    dZ1 = oracle.act_bwd("relu", Z1, dH1)
+    _, dW1 = oracle.rgcn_bwd(ip, ix, et, X, p["W1"], dZ1, need_dX=False)
+    return loss, {"W1": dW1, "b1": dZ1.sum(0), "W2": dW2, "b2": db2}

@@ -65,13 +65,17 @@ def test_rgcn_bwd(env, Fin, Fout):
     dW = torch.empty((R, Fin, Fout), device="cuda")
     ws_b = L.seastar_rgcn_bwd_workspace(g.handle, Fin, Fout)
     ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    Z = rnd(14, (N, Fin)).astype(np.float64)           # fused activation backward on dX
+    Yact = oracle.act_fwd("relu", Z).astype(np.float32)
     L.seastar_rgcn_bwd(g.handle, dev(env, padded(X, ldx)), Fin, ldx, dev(env, padded(dA, ldd)), Fout, ldd,
-                       dev(env, W), None, dX, dW, ws, ws_b)
+                       dev(env, W), None, dev(env, padded(Yact, ldx)), "relu", dX, dW, ws, ws_b)
     rdX, rdW = oracle.rgcn_bwd(env["ip"], env["ix"], env["et"], X, W, dA)
-    assert rel_err(dX.cpu().numpy()[:, :Fin], rdX) <= TOL
+    assert rel_err(dX.cpu().numpy()[:, :Fin], oracle.act_bwd("relu", Z, rdX)) <= TOL
     assert rel_err(dW.cpu().numpy(), rdW) <= TOL
     # deterministic run to run (no atomics anywhere in the R-GCN backward)
     dW2 = torch.empty_like(dW)
+    dX2 = torch.empty_like(dX)
     L.seastar_rgcn_bwd(g.handle, dev(env, padded(X, ldx)), Fin, ldx, dev(env, padded(dA, ldd)), Fout, ldd,
-                       dev(env, W), None, None, dW2, ws, ws_b)
+                       dev(env, W), None, None, "none", dX2, dW2, ws, ws_b)
     assert torch.equal(dW, dW2)
+    assert rel_err(dX2.cpu().numpy()[:, :Fin], rdX) <= TOL
