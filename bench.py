@@ -245,26 +245,25 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
     from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
     from paper_conf_eurosys_wumcjlzcy21_b200.graph import Graph
+    from paper_conf_eurosys_wumcjlzcy21_b200 import partition
     from paper_conf_eurosys_wumcjlzcy21_b200.models import GAT2, GCN2, Comm
     L.seastar_device_check()
 
     t_setup = time.perf_counter()
     ip, ix, X, lab, gcn_p, gat_p = make_inputs()
     N = CFG.N
-    n_per = (N + world - 1) // world
-    rb, re = min(N, rank * n_per), min(N, (rank + 1) * n_per)
+    rb, re = partition.row_range(N, world, rank)
+    rows_all = partition.gathered_rows(N, world)
     g = Graph(ip, ix, row_begin=rb, row_end=re, device=dev)
     X_loc = torch.from_numpy(X[rb:re]).to(dev)
     lab_loc = torch.from_numpy(lab[rb:re]).to(dev)
     comm = Comm(world, rank)
     models = {}
     if args.model in ("both", "gcn"):
-        models["gcn"] = GCN2(g, X_loc, lab_loc, gcn_p, comm=comm, n_pad_rows=n_per * world)
+        models["gcn"] = GCN2(g, X_loc, lab_loc, gcn_p, comm=comm, n_pad_rows=rows_all)
     if args.model in ("both", "gat"):
         models["gat"] = GAT2(g, X_loc, lab_loc, gat_p, CFG.heads, CFG.extra["gat_hidden"], comm=comm,
-                             n_pad_rows=n_per * world)
-    if world > 1 and re - rb < n_per:
-        raise SystemExit("uneven partition: pad N to a multiple of the world size")
+                             n_pad_rows=rows_all)
     torch.cuda.synchronize()
     setup_s = time.perf_counter() - t_setup
 

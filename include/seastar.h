@@ -290,13 +290,15 @@ size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out);
 /* training-step glue kept on the GPU (DGL default loop)                         */
 /* ------------------------------------------------------------------------------------------ */
 /*
- * Mean softmax cross-entropy over M rows: loss (dev scalar) = mean_r (lse(Z_r) - Z_r[label_r]);
- * dZ = (softmax(Z) - onehot) / M.  Z [M,C] ld ldz, labels (dev) [M] int64, dZ may alias nothing.
+ * Softmax cross-entropy over this rank's M rows, normalised by the global row count n_total (>= M;
+ * = M on one GPU) so that per-rank gradients all-reduce to the full-batch gradient:
+ *   loss (dev scalar) = sum_r (lse(Z_r) - Z_r[label_r]) / n_total ;  dZ = (softmax(Z) - onehot) / n_total.
+ * Z [M,C] ld ldz, labels (dev) [M] int64, dZ [M,C] ld lddz or NULL.
  * workspace: seastar_softmax_xent_workspace() bytes.
  */
-seastar_status seastar_softmax_xent(const float* Z, int64_t M, int32_t C, int64_t ldz, const int64_t* labels,
-                                    float* loss, float* dZ, int64_t lddz, void* workspace, size_t ws_bytes,
-                                    seastar_stream stream);
+seastar_status seastar_softmax_xent(const float* Z, int64_t M, int64_t n_total, int32_t C, int64_t ldz,
+                                    const int64_t* labels, float* loss, float* dZ, int64_t lddz, void* workspace,
+                                    size_t ws_bytes, seastar_stream stream);
 size_t seastar_softmax_xent_workspace(int64_t M);
 /* out[j] = sum_r X[r,j] for j < F (deterministic two-stage), workspace: seastar_colsum_workspace() */
 seastar_status seastar_colsum(const float* X, int64_t M, int64_t F, int64_t ld, float* out, void* workspace,

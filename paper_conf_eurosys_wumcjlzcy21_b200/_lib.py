@@ -76,7 +76,7 @@ _SIGS = {
     "seastar_rgcn_fwd": ([_P, _P, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
     "seastar_rgcn_bwd": ([_P, _P, _I64, _I64, _P, _I64, _I64, _P, _P, _P, _I32, _P, _P, _P, _SZ, _P], _ST),
     "seastar_rgcn_bwd_workspace": ([_P, _I64, _I64], _SZ),
-    "seastar_softmax_xent": ([_P, _I64, _I32, _I64, _P, _P, _P, _I64, _P, _SZ, _P], _ST),
+    "seastar_softmax_xent": ([_P, _I64, _I64, _I32, _I64, _P, _P, _P, _I64, _P, _SZ, _P], _ST),
     "seastar_softmax_xent_workspace": ([_I64], _SZ),
     "seastar_colsum": ([_P, _I64, _I64, _I64, _P, _P, _SZ, _P], _ST),
     "seastar_colsum_workspace": ([_I64, _I64], _SZ),
@@ -296,8 +296,8 @@ def seastar_softmax_xent_workspace(M) -> int:
     return int(load().seastar_softmax_xent_workspace(M))
 
 
-def seastar_softmax_xent(Z, M, C, ldz, labels, loss, dZ, lddz, workspace, ws_bytes, stream=None) -> None:
-    _call("seastar_softmax_xent", _dptr(Z, "Z"), M, C, ldz, _dptr(labels, "labels"), _dptr(loss, "loss"),
+def seastar_softmax_xent(Z, M, n_total, C, ldz, labels, loss, dZ, lddz, workspace, ws_bytes, stream=None) -> None:
+    _call("seastar_softmax_xent", _dptr(Z, "Z"), M, n_total, C, ldz, _dptr(labels, "labels"), _dptr(loss, "loss"),
           _dptr(dZ, "dZ"), lddz, _dptr(workspace, "workspace"), ws_bytes, _stream(stream))
 
 

@@ -61,9 +61,9 @@ seastar_status colsum_impl(const float* X, int64_t M, int64_t F, int64_t ld, flo
 }
 
 // warp per row: loss_r = lse(z_r) - z_r[label]; dZ = (softmax - onehot) / M; per-block loss partials
-__global__ void __launch_bounds__(256) k_softmax_xent(const float* __restrict__ Z, int64_t M, int C, int64_t ldz,
-                                                      const int64_t* __restrict__ labels, float* __restrict__ dZ,
-                                                      int64_t lddz, float* __restrict__ part) {
+__global__ void __launch_bounds__(256) k_softmax_xent(const float* __restrict__ Z, int64_t M, int64_t n_total, int C,
+                                                      int64_t ldz, const int64_t* __restrict__ labels,
+                                                      float* __restrict__ dZ, int64_t lddz, float* __restrict__ part) {
     __shared__ float wl[8];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t r = blockIdx.x * 8 + w;
@@ -78,7 +78,7 @@ __global__ void __launch_bounds__(256) k_softmax_xent(const float* __restrict__ 
         for (int o = 16; o; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
         const float lse = m + logf(sum);
         const int64_t lab = labels[r];
-        const float inv = 1.f / (float)M;
+        const float inv = 1.f / (float)n_total;
         if (dZ)
             for (int c = lane; c < C; c += 32)
                 dZ[r * lddz + c] = (expf(__ldg(z + c) - lse) - (c == lab ? 1.f : 0.f)) * inv;
@@ -93,7 +93,7 @@ __global__ void __launch_bounds__(256) k_softmax_xent(const float* __restrict__ 
     }
 }
 
-__global__ void k_loss_final(const float* __restrict__ part, int64_t n, int64_t M, float* __restrict__ loss) {
+__global__ void k_loss_final(const float* __restrict__ part, int64_t n, int64_t n_total, float* __restrict__ loss) {
     __shared__ double red[256];
     double x = 0.0;
     for (int64_t i = threadIdx.x; i < n; i += 256) x += (double)part[i];
@@ -103,7 +103,7 @@ __global__ void k_loss_final(const float* __restrict__ part, int64_t n, int64_t 
         if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
         __syncthreads();
     }
-    if (threadIdx.x == 0) *loss = (float)(red[0] / (double)M);
+    if (threadIdx.x == 0) *loss = (float)(red[0] / (double)n_total);
 }
 
 __global__ void k_axpby(int64_t n, float a, const float* __restrict__ x, float b, float* __restrict__ y) {
@@ -146,18 +146,19 @@ seastar_status seastar_colsum(const float* X, int64_t M, int64_t F, int64_t ld, 
 
 size_t seastar_softmax_xent_workspace(int64_t M) { return (size_t)((M + 7) / 8 + 1) * sizeof(float) + 256; }
 
-seastar_status seastar_softmax_xent(const float* Z, int64_t M, int32_t C, int64_t ldz, const int64_t* labels,
-                                    float* loss, float* dZ, int64_t lddz, void* workspace, size_t ws_bytes,
-                                    seastar_stream stream) {
+seastar_status seastar_softmax_xent(const float* Z, int64_t M, int64_t n_total, int32_t C, int64_t ldz,
+                                    const int64_t* labels, float* loss, float* dZ, int64_t lddz, void* workspace,
+                                    size_t ws_bytes, seastar_stream stream) {
     SS_ARG(Z && labels && loss && workspace, "softmax_xent: NULL argument");
     SS_ARG(M >= 1 && C >= 1 && ldz >= C && (!dZ || lddz >= C), "softmax_xent: bad sizes");
+    SS_ARG(n_total >= M, "softmax_xent: n_total (%lld) < M (%lld)", (long long)n_total, (long long)M);
     SS_ARG(ws_bytes >= seastar_softmax_xent_workspace(M), "softmax_xent: workspace too small");
     SS_TRY(check_device());
     cudaStream_t s = to_stream(stream);
     const int64_t nblk = (M + 7) / 8;
     float* part = static_cast<float*>(workspace);
-    k_softmax_xent<<<(unsigned)nblk, 256, 0, s>>>(Z, M, C, ldz, labels, dZ, lddz, part);
-    k_loss_final<<<1, 256, 0, s>>>(part, nblk, M, loss);
+    k_softmax_xent<<<(unsigned)nblk, 256, 0, s>>>(Z, M, n_total, C, ldz, labels, dZ, lddz, part);
+    k_loss_final<<<1, 256, 0, s>>>(part, nblk, n_total, loss);
     return check_launch("k_softmax_xent");
 }
 

@@ -26,6 +26,15 @@ def _ld(F: int) -> int:
     return (F + 3) // 4 * 4
 
 
+def _local_rows(m) -> int:
+    """Rows of the per-rank buffers: the owned rows on one GPU; ceil(N/P) when partitioned, so every
+    rank contributes an equal chunk to the all-gathers (rows past n_loc are never written)."""
+    if m.comm.world == 1:
+        return m.n
+    assert m.rows_all % m.comm.world == 0 and m.rows_all // m.comm.world >= m.n
+    return m.rows_all // m.comm.world
+
+
 class Comm:
     """Row-partition plumbing.  P = 1: every gather is the identity (no copies)."""
 
@@ -117,7 +126,7 @@ class GCN2:
         self.P = _Params({"W1": params["W1"].shape, "b1": (self.H,), "W2": params["W2"].shape, "b2": (self.C,)},
                          params, dev)
         self.src_n, self.dst_n = g.degree_norms("both")
-        H, C, n = self.H, self.C, self.n
+        H, C, n = self.H, self.C, _local_rows(self)
         e = lambda r, c: torch.zeros((r, c), device=dev)
         self.T1 = e(n, H)          # src_norm * (X W1), local rows
         self.H1 = e(n, H)          # relu(dst_norm * sum T1 + b1)
@@ -156,8 +165,8 @@ class GCN2:
         L.seastar_gcn_fwd(g.handle, H1s_all, H, H, self.dst_n, None, "none", 0.0, None, self.P2)
         L.seastar_linear_fwd(self.P2, n, H, H, p.p("W2"), C, p.p("b2"), None, "none", self.logits, self.ldc)
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
-        L.seastar_softmax_xent(self.logits, n, C, self.ldc, self.lab, self.loss, self.dlogits, self.ldc, ws,
-                               ws.numel())
+        L.seastar_softmax_xent(self.logits, n, self.g.N, C, self.ldc, self.lab, self.loss, self.dlogits, self.ldc,
+                               ws, ws.numel())
         return self.loss
 
     def backward(self):
@@ -204,7 +213,7 @@ class GAT2:
         shapes = {"W1": (self.Fin, self.W1w), "al1": (heads, hidden), "ar1": (heads, hidden), "b1": (self.W1w,),
                   "W2": (self.W1w, self.C), "al2": (1, self.C), "ar2": (1, self.C), "b2": (self.C,)}
         self.P = _Params(shapes, params, dev)
-        n, W1w, C = self.n, self.W1w, self.C
+        n, W1w, C = _local_rows(self), self.W1w, self.C
         self.ld1, self.ld2 = _ld(W1w), _ld(C)
         e = lambda r, c: torch.zeros((r, c), device=dev)
         self.T1, self.A1, self.Y1 = e(n, self.ld1), e(n, self.ld1), e(n, self.ld1)
@@ -255,7 +264,8 @@ class GAT2:
         L.seastar_gat_fwd(g.handle, T2_all, el2_all, self.er2, 1, C, self.ld2, self.slope, p.p("b2"), "none", self.A2,
                           self.Y2, self.lse2)
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
-        L.seastar_softmax_xent(self.Y2, n, C, self.ld2, self.lab, self.loss, self.dY2, self.ld2, ws, ws.numel())
+        L.seastar_softmax_xent(self.Y2, n, self.g.N, C, self.ld2, self.lab, self.loss, self.dY2, self.ld2, ws,
+                               ws.numel())
         return self.loss
 
     def _layer_bwd(self, T, T_loc_ld, el, er, A, Y, lse, dY, act, H, F, D, D_all_buf, dT, del_, der, gathered,
@@ -316,7 +326,7 @@ class APPNPNet:
         self.P = _Params({"W1": params["W1"].shape, "b1": (self.Hd,), "W2": params["W2"].shape, "b2": (self.C,)},
                          params, dev)
         _, self.nrm = g.degree_norms("in")
-        n, Hd, C = self.n, self.Hd, self.C
+        n, Hd, C = _local_rows(self), self.Hd, self.C
         self.ldc = _ld(C)
         e = lambda r, c: torch.zeros((r, c), device=dev)
         self.Hh = e(n, Hd)
@@ -346,7 +356,7 @@ class APPNPNet:
                               self.nrm, self.Zs[k + 1])
         out = self.Z[self.K] if self.K > 0 else self.H0
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
-        L.seastar_softmax_xent(out, n, C, ld, self.lab, self.loss, self.G, ld, ws, ws.numel())
+        L.seastar_softmax_xent(out, n, self.g.N, C, ld, self.lab, self.loss, self.G, ld, ws, ws.numel())
         return self.loss
 
     def backward(self):
@@ -401,7 +411,11 @@ class RGCN2:
         assert X_loc.stride(0) % 4 == 0, "R-GCN input rows need a leading dimension that is a multiple of 4"
         self.P = _Params({"W1": params["W1"].shape, "b1": (self.Hd,), "W2": params["W2"].shape, "b2": (self.C,)},
                          params, dev)
-        n = self.n
+        n = _local_rows(self)
+        if X_loc.shape[0] < n:      # the input rows are all-gathered too: pad this rank's chunk
+            Xp = torch.zeros((n, X_loc.stride(0)), device=dev)
+            Xp[:X_loc.shape[0], :X_loc.shape[1]] = X_loc
+            self.X = Xp[:, :X_loc.shape[1]]
         self.ldh, self.ldc = _ld(self.Hd), _ld(self.C)
         e = lambda r, c: torch.zeros((r, c), device=dev)
         self.H1, self.dZ1 = e(n, self.ldh), e(n, self.ldh)
@@ -424,8 +438,8 @@ class RGCN2:
         L.seastar_rgcn_fwd(g.handle, self._H1_all, self.Hd, self.ldh, p.p("W2"), self.C, None, p.p("b2"), "none",
                            self.logits, self.ldc)
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
-        L.seastar_softmax_xent(self.logits, n, self.C, self.ldc, self.lab, self.loss, self.dlog, self.ldc, ws,
-                               ws.numel())
+        L.seastar_softmax_xent(self.logits, n, self.g.N, self.C, self.ldc, self.lab, self.loss, self.dlog, self.ldc,
+                               ws, ws.numel())
         return self.loss
 
     def backward(self):

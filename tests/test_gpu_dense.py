@@ -73,10 +73,14 @@ def test_softmax_xent(env, M, C):
     ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
     loss = torch.empty((1,), device="cuda")
     dZ = torch.empty((M, C), device="cuda")
-    L.seastar_softmax_xent(dev(env, Z), M, C, C, dev(env, lab), loss, dZ, C, ws, ws_b)
+    L.seastar_softmax_xent(dev(env, Z), M, M, C, C, dev(env, lab), loss, dZ, C, ws, ws_b)
     rl, rd = oracle.softmax_xent(Z, lab)
     assert abs(loss.item() - rl) <= TOL * abs(rl)
     assert rel_err(dZ.cpu().numpy(), rd) <= TOL
+    # a rank holding M of n_total rows scales by the global count
+    L.seastar_softmax_xent(dev(env, Z), M, 3 * M, C, C, dev(env, lab), loss, dZ, C, ws, ws_b)
+    assert abs(loss.item() - rl / 3) <= TOL * abs(rl)
+    assert rel_err(dZ.cpu().numpy(), rd / 3) <= TOL
 
 
 def test_colsum_axpby_adam(env):
