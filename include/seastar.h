@@ -207,22 +207,30 @@ seastar_status seastar_gat_attn_proj(const float* T, int64_t M, int32_t H, int32
  *   s_e = el_all[src(e),h] + er_loc[v,h];  z_e = LeakyReLU_slope(s_e);
  *   A[v,h,:] = sum_e softmax_e(z) T_all[src(e),h,:]  (0 for an empty row);
  *   lse[v,h] = log sum_e exp(z_e) (-inf for an empty row);  Y[v] = act(A[v] + bias).
- * T_all [N,H*F] ld ldt ; el_all [N,H] ; er_loc/lse_loc [n_loc,H] ; A_loc, Y_loc [n_loc,H*F] ld ldt.
+ * Optional (B_loc and b_loc both non-NULL): from the same gathered rows also
+ *   B[v,h,:] = sum_e a_e LeakyReLU'(s_e) T_all[src(e),h,:]   and   b[v,h] = sum_e a_e LeakyReLU'(s_e),
+ * the forward-only factors of der_v = sum_e ds_e = <dA_v, B_v> - c_v b_v, so that the backward needs no
+ * destination-major edge pass (seastar_gat_bwd_prep then emits der directly).
+ * T_all [N,H*F] ld ldt ; el_all [N,H] ; er_loc/lse_loc/b_loc [n_loc,H] ; A_loc, Y_loc, B_loc [n_loc,H*F] ld ldt.
  * Requires F % 4 == 0 or H == 1 for the 128-bit path (otherwise 32-bit loads are used).
  */
 seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float* el_all, const float* er_loc,
                                int32_t H, int32_t F, int64_t ldt, float slope, const float* bias, seastar_act act,
-                               float* A_loc, float* Y_loc, float* lse_loc, seastar_stream stream);
+                               float* A_loc, float* Y_loc, float* lse_loc, float* B_loc, float* b_loc,
+                               seastar_stream stream);
 /* leading dimension (floats) of the packed per-destination backward record D: round_up(H*F, 4) + 4*H */
 int64_t seastar_gat_record_ld(int32_t H, int32_t F);
 /*
  * Backward row pass over owned rows: dA = dY * act'(Y);  c[v,h] = <dA[v,h,:], A[v,h,:]>;
  * D_loc[v] = [ dA (H*F, padded to a multiple of 4) | per head (er, lse, c, 0) ]
  * (ld = seastar_gat_record_ld(H,F); every field is 16-byte aligned when D_loc is).
+ * If B_loc, b_loc (saved by seastar_gat_fwd) and der_loc [n_loc,H] are given, also
+ *   der_loc[v,h] = <dA[v,h,:], B[v,h,:]> - c[v,h] b[v,h]    (replaces seastar_gat_der).
  */
 seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const float* Y_loc, seastar_act act,
                                     const float* A_loc, const float* er_loc, const float* lse_loc, int32_t H,
-                                    int32_t F, int64_t ldt, float* D_loc, seastar_stream stream);
+                                    int32_t F, int64_t ldt, float* D_loc, const float* B_loc, const float* b_loc,
+                                    float* der_loc, seastar_stream stream);
 /*
  * Fused source-major backward over the reverse CSR, for every owned u and out-edge e = (u -> v):
  *   a_e = exp(LeakyReLU(el[u,h] + er[v,h]) - lse[v,h]);  g_e = <dA[v,h,:], T[u,h,:]>;

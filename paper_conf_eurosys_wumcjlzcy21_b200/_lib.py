@@ -66,9 +66,9 @@ _SIGS = {
     "seastar_gcn_fwd": ([_P, _P, _I64, _I64, _P, _P, _I32, _F, _P, _P, _P, _P, _P], _ST),
     "seastar_gcn_bwd": ([_P, _P, _I64, _I64, _P, _F, _P, _I32, _P, _P, _P, _P], _ST),
     "seastar_gat_attn_proj": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P], _ST),
-    "seastar_gat_fwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _I32, _P, _P, _P, _P], _ST),
+    "seastar_gat_fwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _I32, _P, _P, _P, _P, _P, _P], _ST),
     "seastar_gat_record_ld": ([_I32, _I32], _I64),
-    "seastar_gat_bwd_prep": ([_P, _P, _P, _I32, _P, _P, _P, _I32, _I32, _I64, _P, _P], _ST),
+    "seastar_gat_bwd_prep": ([_P, _P, _P, _I32, _P, _P, _P, _I32, _I32, _I64, _P, _P, _P, _P, _P], _ST),
     "seastar_gat_bwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P, _P], _ST),
     "seastar_gat_der": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P], _ST),
     "seastar_gat_attn_proj_bwd": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P, _P, _P, _P, _SZ, _P], _ST),
@@ -237,20 +237,22 @@ def seastar_gat_attn_proj(T, M, H, F, ldt, a_l, a_r, el, er, stream=None) -> Non
           _dptr(el, "el"), _dptr(er, "er"), _stream(stream))
 
 
-def seastar_gat_fwd(g, T_all, el_all, er_loc, H, F, ldt, slope, bias, act, A_loc, Y_loc, lse_loc,
-                    stream=None) -> None:
+def seastar_gat_fwd(g, T_all, el_all, er_loc, H, F, ldt, slope, bias, act, A_loc, Y_loc, lse_loc, B_loc=None,
+                    b_loc=None, stream=None) -> None:
     _call("seastar_gat_fwd", g, _dptr(T_all, "T"), _dptr(el_all, "el"), _dptr(er_loc, "er"), H, F, ldt,
           float(slope), _dptr(bias, "bias"), _act(act), _dptr(A_loc, "A"), _dptr(Y_loc, "Y"), _dptr(lse_loc, "lse"),
-          _stream(stream))
+          _dptr(B_loc, "B"), _dptr(b_loc, "b"), _stream(stream))
 
 
 def seastar_gat_record_ld(H, F) -> int:
     return int(load().seastar_gat_record_ld(H, F))
 
 
-def seastar_gat_bwd_prep(g, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, H, F, ldt, D_loc, stream=None) -> None:
+def seastar_gat_bwd_prep(g, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, H, F, ldt, D_loc, B_loc=None, b_loc=None,
+                         der_loc=None, stream=None) -> None:
     _call("seastar_gat_bwd_prep", g, _dptr(dY_loc, "dY"), _dptr(Y_loc, "Y"), _act(act), _dptr(A_loc, "A"),
-          _dptr(er_loc, "er"), _dptr(lse_loc, "lse"), H, F, ldt, _dptr(D_loc, "D"), _stream(stream))
+          _dptr(er_loc, "er"), _dptr(lse_loc, "lse"), H, F, ldt, _dptr(D_loc, "D"), _dptr(B_loc, "B"),
+          _dptr(b_loc, "b"), _dptr(der_loc, "der"), _stream(stream))
 
 
 def seastar_gat_bwd(g, T_loc, el_loc, D_all, H, F, ldt, slope, dT_loc, del_loc, stream=None) -> None:

@@ -150,6 +150,51 @@ __device__ __forceinline__ float act_grad_from_y(int act, float y) {
 
 inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
+// ----------------------------------------------------------------------------------------------
+// L2 residency of the gathered table.  Every edge of a graph kernel gathers a row of one table
+// (T, dP, the GAT record D, X ...) that is 15-90 MB and therefore *could* live in the 126 MB L2, while
+// the edge-index stream (4-8 B per edge, 0.5-1 GB) and the outputs stream through once.  Graph kernels
+// are launched with an access-policy window over the gathered table (hits persist, misses stream) and
+// read their index streams with evict-first loads (__ldcs).
+// ----------------------------------------------------------------------------------------------
+struct L2Window {
+    const void* base = nullptr;
+    size_t bytes = 0;
+};
+extern thread_local L2Window t_l2win;
+
+struct ScopedL2Window {
+    L2Window saved;
+    ScopedL2Window(const void* base, size_t bytes) : saved(t_l2win) { t_l2win = {base, bytes}; }
+    ~ScopedL2Window() { t_l2win = saved; }
+};
+
+size_t l2_persist_bytes();   // device set-aside for persisting lines (configured on first use), 0 if none
+
+template <typename... KArgs, typename... Args>
+inline void launch_k(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    cfg.attrs = attr;
+    cfg.numAttrs = 0;
+    const size_t persist = t_l2win.base && t_l2win.bytes ? l2_persist_bytes() : 0;
+    if (persist) {
+        const size_t win = t_l2win.bytes < ((size_t)128 << 20) ? t_l2win.bytes : ((size_t)128 << 20);
+        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[0].val.accessPolicyWindow.base_ptr = const_cast<void*>(t_l2win.base);
+        attr[0].val.accessPolicyWindow.num_bytes = win;
+        attr[0].val.accessPolicyWindow.hitRatio = persist >= win ? 1.0f : (float)persist / (float)win;
+        attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.numAttrs = 1;
+    }
+    cudaLaunchKernelEx(&cfg, kernel, args...);
+}
+
 inline int num_sms() {
     static int sms = 0;
     if (!sms) {

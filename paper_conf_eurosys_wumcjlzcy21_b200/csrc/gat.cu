@@ -35,6 +35,7 @@ struct GatFwdArgs {
     int H, F; int64_t ld; float slope;
     const float* bias; int act;
     float* A; float* Y; float* lse;
+    float* B; float* bsum;   // optional: der factors (see k_gat_fwd_hpl)
 };
 
 // lane geometry of the chunked kernels: chunk `chunk` covers floats [chunk*VEC, chunk*VEC+VEC)
@@ -70,13 +71,14 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
     const int64_t col = (int64_t)chunk * VEC;
     const float erv = (valid && active) ? __ldg(a.er + v * a.H + h) : 0.f;
 
-    float m = -INFINITY, ssum = 0.f, acc[VEC];
+    const bool SB = a.B != nullptr;     // fallback path: runtime flag
+    float m = -INFINITY, ssum = 0.f, acc[VEC], pacc[VEC], psum = 0.f;
 #pragma unroll
-    for (int i = 0; i < VEC; ++i) acc[i] = 0.f;
+    for (int i = 0; i < VEC; ++i) acc[i] = pacc[i] = 0.f;
 
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+        const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -99,14 +101,20 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
             for (int jj = 0; jj < UB; ++jj) mb = fmaxf(mb, z[jj]);
             const float corr = (m == -INFINITY) ? 0.f : expf(m - mb);
             ssum *= corr;
+            psum *= corr;
 #pragma unroll
-            for (int i = 0; i < VEC; ++i) acc[i] *= corr;
+            for (int i = 0; i < VEC; ++i) { acc[i] *= corr; pacc[i] *= corr; }
 #pragma unroll
             for (int jj = 0; jj < UB; ++jj) {
                 const float p = (z[jj] == -INFINITY) ? 0.f : expf(z[jj] - mb);
                 ssum += p;
+                const float pp = (SB && z[jj] > 0.f) ? p : 0.f;
+                psum += pp;
 #pragma unroll
-                for (int i = 0; i < VEC; ++i) acc[i] = fmaf(p, val[jj][i], acc[i]);
+                for (int i = 0; i < VEC; ++i) {
+                    acc[i] = fmaf(p, val[jj][i], acc[i]);
+                    pacc[i] = fmaf(pp, val[jj][i], pacc[i]);
+                }
             }
             m = mb;
         }
@@ -123,8 +131,12 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
         const float ca = (m == -INFINITY) ? 0.f : expf(m - mn);
         const float cb = (mo == -INFINITY) ? 0.f : expf(mo - mn);
         ssum = ssum * ca + so * cb;
+        psum = psum * ca + __shfl_xor_sync(gmask, psum, o, RL) * cb;
 #pragma unroll
-        for (int i = 0; i < VEC; ++i) acc[i] = acc[i] * ca + ao[i] * cb;
+        for (int i = 0; i < VEC; ++i) {
+            acc[i] = acc[i] * ca + ao[i] * cb;
+            pacc[i] = pacc[i] * ca + __shfl_xor_sync(gmask, pacc[i], o, RL) * cb;
+        }
         m = mn;
     }
     if (!valid || slot != 0 || !active) return;
@@ -145,12 +157,21 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
     } else {
         for (int i = 0; i < VEC && col + i < W; ++i) { pa[i] = outA[i]; py[i] = outY[i]; }
     }
-    if ((a.H == 1 && chunk == 0) || (a.H > 1 && col % a.F == 0))
+    if (SB) {
+        float* pb = a.B + v * a.ld + col;
+        for (int i = 0; i < VEC && col + i < W; ++i) pb[i] = a.slope * outA[i] + (1.f - a.slope) * pacc[i] * inv;
+    }
+    if ((a.H == 1 && chunk == 0) || (a.H > 1 && col % a.F == 0)) {
         a.lse[v * a.H + h] = ssum > 0.f ? m + logf(ssum) : -INFINITY;
+        if (SB) a.bsum[v * a.H + h] = ssum > 0.f ? a.slope + (1.f - a.slope) * psum * inv : 0.f;
+    }
 }
 
 // head-per-lane forward: warp per destination row; lane = (slot, head), S = 32/H edge slots.
-template <int F4>
+// SB: also accumulate the positive-logit part P_v = sum_{e: s_e > 0} a_e T_u (same gathered rows), from
+// which the epilogue writes B_v = sum_e a_e LReLU'(s_e) T_u and b_v = sum_e a_e LReLU'(s_e) -- the two
+// forward-only factors of der_v = <dA_v, B_v> - c_v b_v (so the backward needs no dst-major pass).
+template <int F4, bool SB>
 __global__ void __launch_bounds__(256) k_gat_fwd_hpl(const GatFwdArgs a) {
     constexpr int F = 4 * F4;
     constexpr int UB = F4 <= 2 ? 4 : (F4 <= 4 ? 2 : 1);
@@ -164,12 +185,14 @@ __global__ void __launch_bounds__(256) k_gat_fwd_hpl(const GatFwdArgs a) {
     const int64_t v = (int64_t)__ldg(a.perm + row) - a.vbase;
     const float erv = __ldg(a.er + v * H + h);
     const int64_t hoff = (int64_t)h * F;
-    float m = -INFINITY, ssum = 0.f, acc[F];
+    float m = -INFINITY, ssum = 0.f, acc[F], pacc[SB ? F : 1], psum = 0.f;
 #pragma unroll
     for (int i = 0; i < F; ++i) acc[i] = 0.f;
+#pragma unroll
+    for (int i = 0; i < (SB ? F : 1); ++i) pacc[i] = 0.f;
     for (int base = beg; base < end; base += 32) {
         const int n = min(32, end - base);
-        const int my = (lane < n) ? __ldg(a.nbr + base + lane) : 0;
+        const int my = (lane < n) ? __ldcs(a.nbr + base + lane) : 0;
         for (int i0 = 0; i0 < H; i0 += UB) {             // this slot's edges: k = slot + S * i
             if (i0 * S >= n) break;
             float z[UB], x[UB][F];
@@ -194,18 +217,31 @@ __global__ void __launch_bounds__(256) k_gat_fwd_hpl(const GatFwdArgs a) {
             float mb = m;
 #pragma unroll
             for (int jj = 0; jj < UB; ++jj) mb = fmaxf(mb, z[jj]);
-            const float corr = (m == -INFINITY) ? 0.f : expf(m - mb);
-            ssum *= corr;
+            if (mb > m) {                                 // rescale only when the running max moves
+                const float corr = (m == -INFINITY) ? 0.f : expf(m - mb);
+                ssum *= corr;
 #pragma unroll
-            for (int i = 0; i < F; ++i) acc[i] *= corr;
+                for (int i = 0; i < F; ++i) acc[i] *= corr;
+                if (SB) {
+                    psum *= corr;
+#pragma unroll
+                    for (int i = 0; i < (SB ? F : 1); ++i) pacc[i] *= corr;
+                }
+                m = mb;
+            }
 #pragma unroll
             for (int jj = 0; jj < UB; ++jj) {
-                const float p = (z[jj] == -INFINITY) ? 0.f : expf(z[jj] - mb);
+                const float p = (z[jj] == -INFINITY) ? 0.f : expf(z[jj] - m);
                 ssum += p;
 #pragma unroll
                 for (int i = 0; i < F; ++i) acc[i] = fmaf(p, x[jj][i], acc[i]);
+                if (SB) {
+                    const float pp = z[jj] > 0.f ? p : 0.f;
+                    psum += pp;
+#pragma unroll
+                    for (int i = 0; i < (SB ? F : 1); ++i) pacc[i] = fmaf(pp, x[jj][i], pacc[i]);
+                }
             }
-            m = mb;
         }
     }
     for (int o = H; o < 32; o <<= 1) {
@@ -217,6 +253,11 @@ __global__ void __launch_bounds__(256) k_gat_fwd_hpl(const GatFwdArgs a) {
         ssum = ssum * ca + so * cb;
 #pragma unroll
         for (int i = 0; i < F; ++i) acc[i] = acc[i] * ca + __shfl_xor_sync(0xffffffffu, acc[i], o) * cb;
+        if (SB) {
+            psum = psum * ca + __shfl_xor_sync(0xffffffffu, psum, o) * cb;
+#pragma unroll
+            for (int i = 0; i < (SB ? F : 1); ++i) pacc[i] = pacc[i] * ca + __shfl_xor_sync(0xffffffffu, pacc[i], o) * cb;
+        }
         m = mn;
     }
     if (slot != 0) return;
@@ -233,8 +274,15 @@ __global__ void __launch_bounds__(256) k_gat_fwd_hpl(const GatFwdArgs a) {
         }
         *reinterpret_cast<float4*>(pa + 4 * q) = make_float4(o4[0], o4[1], o4[2], o4[3]);
         *reinterpret_cast<float4*>(py + 4 * q) = make_float4(y4[0], y4[1], y4[2], y4[3]);
+        if (SB) {
+            float b4[4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) b4[i] = a.slope * o4[i] + (1.f - a.slope) * pacc[(4 * q + i) % (SB ? F : 1)] * inv;
+            *reinterpret_cast<float4*>(a.B + v * a.ld + hoff + 4 * q) = make_float4(b4[0], b4[1], b4[2], b4[3]);
+        }
     }
     a.lse[v * H + h] = ssum > 0.f ? m + logf(ssum) : -INFINITY;
+    if (SB) a.bsum[v * H + h] = ssum > 0.f ? a.slope + (1.f - a.slope) * psum * inv : 0.f;
 }
 
 // ============================================================================================
@@ -292,7 +340,7 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
 
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int myv = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+        const int myv = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -391,7 +439,7 @@ __global__ void __launch_bounds__(256) k_gat_der(const GatBwdArgs a) {
     float dr = 0.f;
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+        const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -464,7 +512,7 @@ __global__ void __launch_bounds__(256) k_gat_bwd_hpl(const GatBwdArgs a) {
     float dl = 0.f;
     for (int base = beg; base < end; base += 32) {
         const int n = min(32, end - base);
-        const int my = (lane < n) ? __ldg(a.nbr + base + lane) : 0;
+        const int my = (lane < n) ? __ldcs(a.nbr + base + lane) : 0;
         for (int i0 = 0; i0 < H; i0 += UB) {
             if (i0 * S >= n) break;
             float d[UB][F], ax[UB][3];
@@ -541,7 +589,7 @@ __global__ void __launch_bounds__(256) k_gat_der_hpl(const GatBwdArgs a) {
     float dr = 0.f;
     for (int base = beg; base < end; base += 32) {
         const int n = min(32, end - base);
-        const int my = (lane < n) ? __ldg(a.nbr + base + lane) : 0;
+        const int my = (lane < n) ? __ldcs(a.nbr + base + lane) : 0;
         for (int i0 = 0; i0 < H; i0 += UB) {
             if (i0 * S >= n) break;
             float t[UB][F], elu[UB];
@@ -603,9 +651,10 @@ __device__ __forceinline__ void load_chunks(const float* p, int col0, int W, flo
     }
 }
 
-template <int VPL, int L, int RL>
+template <int VPL, int L, int RL, bool SB>
 __global__ void __launch_bounds__(256) k_gat_fwd_h1(const GatFwdArgs a) {
     constexpr int NV = 4 * VPL, S = RL / L, UB = VPL <= 2 ? 4 : 2;
+    constexpr int NP = SB ? NV : 1;
     const int lane = threadIdx.x & 31;
     const int gl = lane % RL, slot = gl / L, c = gl % L;
     const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
@@ -617,12 +666,14 @@ __global__ void __launch_bounds__(256) k_gat_fwd_h1(const GatFwdArgs a) {
     const int64_t v = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;
     const int W = a.F, col0 = c * NV;
     const float erv = valid ? __ldg(a.er + v) : 0.f;
-    float m = -INFINITY, ssum = 0.f, acc[NV];
+    float m = -INFINITY, ssum = 0.f, acc[NV], pacc[NP], psum = 0.f;
 #pragma unroll
     for (int i = 0; i < NV; ++i) acc[i] = 0.f;
+#pragma unroll
+    for (int i = 0; i < NP; ++i) pacc[i] = 0.f;
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+        const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -643,18 +694,31 @@ __global__ void __launch_bounds__(256) k_gat_fwd_h1(const GatFwdArgs a) {
             float mb = m;
 #pragma unroll
             for (int jj = 0; jj < UB; ++jj) mb = fmaxf(mb, z[jj]);
-            const float corr = (m == -INFINITY) ? 0.f : expf(m - mb);
-            ssum *= corr;
+            if (mb > m) {
+                const float corr = (m == -INFINITY) ? 0.f : expf(m - mb);
+                ssum *= corr;
 #pragma unroll
-            for (int i = 0; i < NV; ++i) acc[i] *= corr;
+                for (int i = 0; i < NV; ++i) acc[i] *= corr;
+                if (SB) {
+                    psum *= corr;
+#pragma unroll
+                    for (int i = 0; i < NP; ++i) pacc[i] *= corr;
+                }
+                m = mb;
+            }
 #pragma unroll
             for (int jj = 0; jj < UB; ++jj) {
-                const float p = (z[jj] == -INFINITY) ? 0.f : expf(z[jj] - mb);
+                const float p = (z[jj] == -INFINITY) ? 0.f : expf(z[jj] - m);
                 ssum += p;
 #pragma unroll
                 for (int i = 0; i < NV; ++i) acc[i] = fmaf(p, x[jj][i], acc[i]);
+                if (SB) {
+                    const float pp = z[jj] > 0.f ? p : 0.f;
+                    psum += pp;
+#pragma unroll
+                    for (int i = 0; i < NP; ++i) pacc[i] = fmaf(pp, x[jj][i % NV], pacc[i]);
+                }
             }
-            m = mb;
         }
     }
 #pragma unroll
@@ -667,30 +731,45 @@ __global__ void __launch_bounds__(256) k_gat_fwd_h1(const GatFwdArgs a) {
         ssum = ssum * ca + so * cb;
 #pragma unroll
         for (int i = 0; i < NV; ++i) acc[i] = acc[i] * ca + __shfl_xor_sync(gmask, acc[i], o, RL) * cb;
+        if (SB) {
+            psum = psum * ca + __shfl_xor_sync(gmask, psum, o, RL) * cb;
+#pragma unroll
+            for (int i = 0; i < NP; ++i) pacc[i] = pacc[i] * ca + __shfl_xor_sync(gmask, pacc[i], o, RL) * cb;
+        }
         m = mn;
     }
     if (!valid || slot != 0) return;
     const float inv = ssum > 0.f ? 1.f / ssum : 0.f;
     float* pa = a.A + v * a.ld;
     float* py = a.Y + v * a.ld;
+    float* pb = SB ? a.B + v * a.ld : nullptr;
 #pragma unroll
     for (int q = 0; q < VPL; ++q) {
         const int col = col0 + 4 * q;
         if (col >= W) continue;
-        float o4[4], y4[4];
+        float o4[4], y4[4], b4[4];
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
             o4[i] = acc[4 * q + i] * inv;
             y4[i] = act_apply(a.act, o4[i] + ((a.bias && col + i < W) ? __ldg(a.bias + col + i) : 0.f));
+            b4[i] = SB ? a.slope * o4[i] + (1.f - a.slope) * pacc[(4 * q + i) % NP] * inv : 0.f;
         }
         if (col + 4 <= W) {
             *reinterpret_cast<float4*>(pa + col) = make_float4(o4[0], o4[1], o4[2], o4[3]);
             *reinterpret_cast<float4*>(py + col) = make_float4(y4[0], y4[1], y4[2], y4[3]);
+            if (SB) *reinterpret_cast<float4*>(pb + col) = make_float4(b4[0], b4[1], b4[2], b4[3]);
         } else {
-            for (int i = 0; i < 4 && col + i < W; ++i) { pa[col + i] = o4[i]; py[col + i] = y4[i]; }
+            for (int i = 0; i < 4 && col + i < W; ++i) {
+                pa[col + i] = o4[i];
+                py[col + i] = y4[i];
+                if (SB) pb[col + i] = b4[i];
+            }
         }
     }
-    if (c == 0) a.lse[v] = ssum > 0.f ? m + logf(ssum) : -INFINITY;
+    if (c == 0) {
+        a.lse[v] = ssum > 0.f ? m + logf(ssum) : -INFINITY;
+        if (SB) a.bsum[v] = ssum > 0.f ? a.slope + (1.f - a.slope) * psum * inv : 0.f;
+    }
 }
 
 // DER = false: source-major dT/del over REV; DER = true: destination-major der over FWD
@@ -729,7 +808,7 @@ __global__ void __launch_bounds__(256) k_gat_bwd_h1(const GatBwdArgs a) {
     for (int i = 0; i < NV; ++i) acc[i] = 0.f;
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+        const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -830,20 +909,24 @@ __global__ void k_gat_attn_proj(const float* __restrict__ T, int64_t M, int H, i
 __global__ void k_gat_bwd_prep(int64_t M, int H, int F, int64_t ldt, const float* __restrict__ dY,
                                const float* __restrict__ Y, int act, const float* __restrict__ A,
                                const float* __restrict__ er, const float* __restrict__ lse, float* __restrict__ D,
-                               int64_t ldd) {
+                               int64_t ldd, const float* __restrict__ B, const float* __restrict__ bsum,
+                               float* __restrict__ der) {
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i >= M * H) return;
     const int64_t v = i / H;
     const int h = (int)(i % H);
     const int64_t o = v * ldt + (int64_t)h * F;
     float* rec = D + v * ldd;
-    float cdot = 0.f;
+    float cdot = 0.f, bdot = 0.f;
     for (int f = 0; f < F; ++f) {
         float d = __ldg(dY + o + f);
         if (act != SEASTAR_ACT_NONE) d *= act_grad_from_y(act, __ldg(Y + o + f));
         rec[(int64_t)h * F + f] = d;
         cdot = fmaf(d, __ldg(A + o + f), cdot);
+        if (B) bdot = fmaf(d, __ldg(B + o + f), bdot);
     }
+    // der_v = sum_e a_e LReLU'(s_e) (g_e - c_v) = <dA_v, B_v> - c_v b_v   (B, b from the forward)
+    if (B) der[i] = bdot - cdot * __ldg(bsum + i);
     if (h == H - 1)   // zero the padding between dA and the aux block so vector loads read zeros
         for (int64_t f = (int64_t)H * F; f < rec_aux_offset(H * F); ++f) rec[f] = 0.f;
     float* aux = rec + rec_aux_offset(H * F) + 4 * h;
@@ -921,24 +1004,36 @@ static int hpl_f4(int H, int F, int64_t ldt, bool aligned) {
 
 #define SS_HPL_SWITCH(KERNEL, f4, grid, s, args)                      \
     switch (f4) {                                                     \
-        case 1: KERNEL<1><<<grid, 256, 0, s>>>(args); break;          \
-        case 2: KERNEL<2><<<grid, 256, 0, s>>>(args); break;          \
-        case 3: KERNEL<3><<<grid, 256, 0, s>>>(args); break;          \
-        case 4: KERNEL<4><<<grid, 256, 0, s>>>(args); break;          \
-        case 5: KERNEL<5><<<grid, 256, 0, s>>>(args); break;          \
-        case 6: KERNEL<6><<<grid, 256, 0, s>>>(args); break;          \
-        case 7: KERNEL<7><<<grid, 256, 0, s>>>(args); break;          \
-        default: KERNEL<8><<<grid, 256, 0, s>>>(args); break;         \
+        case 1: launch_k(KERNEL<1>, dim3(grid), dim3(256), 0, s, args); break;          \
+        case 2: launch_k(KERNEL<2>, dim3(grid), dim3(256), 0, s, args); break;          \
+        case 3: launch_k(KERNEL<3>, dim3(grid), dim3(256), 0, s, args); break;          \
+        case 4: launch_k(KERNEL<4>, dim3(grid), dim3(256), 0, s, args); break;          \
+        case 5: launch_k(KERNEL<5>, dim3(grid), dim3(256), 0, s, args); break;          \
+        case 6: launch_k(KERNEL<6>, dim3(grid), dim3(256), 0, s, args); break;          \
+        case 7: launch_k(KERNEL<7>, dim3(grid), dim3(256), 0, s, args); break;          \
+        default: launch_k(KERNEL<8>, dim3(grid), dim3(256), 0, s, args); break;         \
+    }
+
+#define SS_HPL_SWITCH_SB(KERNEL, SB, f4, grid, s, args)                          \
+    switch (f4) {                                                                 \
+        case 1: launch_k(KERNEL<1, SB>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 2: launch_k(KERNEL<2, SB>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 3: launch_k(KERNEL<3, SB>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 4: launch_k(KERNEL<4, SB>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 5: launch_k(KERNEL<5, SB>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 6: launch_k(KERNEL<6, SB>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 7: launch_k(KERNEL<7, SB>, dim3(grid), dim3(256), 0, s, args); break; \
+        default: launch_k(KERNEL<8, SB>, dim3(grid), dim3(256), 0, s, args); break; \
     }
 
 #define SS_CHUNK_SWITCH(KERNEL, VEC, L, RL, grid, s, args)            \
     switch (L) {                                                      \
-        case 1: KERNEL<VEC, 1, (RL < 4 ? 4 : RL)><<<grid, 256, 0, s>>>(args); break; \
-        case 2: KERNEL<VEC, 2, (RL < 4 ? 4 : RL)><<<grid, 256, 0, s>>>(args); break; \
-        case 4: KERNEL<VEC, 4, RL><<<grid, 256, 0, s>>>(args); break; \
-        case 8: KERNEL<VEC, 8, RL><<<grid, 256, 0, s>>>(args); break; \
-        case 16: KERNEL<VEC, 16, RL><<<grid, 256, 0, s>>>(args); break; \
-        default: KERNEL<VEC, 32, 32><<<grid, 256, 0, s>>>(args); break; \
+        case 1: launch_k(KERNEL<VEC, 1, 32>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 2: launch_k(KERNEL<VEC, 2, 32>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 4: launch_k(KERNEL<VEC, 4, RL>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 8: launch_k(KERNEL<VEC, 8, RL>, dim3(grid), dim3(256), 0, s, args); break; \
+        case 16: launch_k(KERNEL<VEC, 16, RL>, dim3(grid), dim3(256), 0, s, args); break; \
+        default: launch_k(KERNEL<VEC, 32, 32>, dim3(grid), dim3(256), 0, s, args); break; \
     }
 
 // chunked launches over the two degree classes: warp rows (RL = 32) and sub-warp rows (RL = L)
@@ -969,8 +1064,14 @@ static bool h1_geometry(int H, int F, int64_t ldt, bool aligned, int& vpl, int& 
 struct FwdH1 {
     template <int VPL, int L>
     static void run(const GatFwdArgs& a, int64_t split, int64_t n, cudaStream_t s) {
-        two_buckets(a, split, n, 4, [&](GatFwdArgs x, unsigned grid) { k_gat_fwd_h1<VPL, L, 32><<<grid, 256, 0, s>>>(x); },
-                    [&](GatFwdArgs x, unsigned grid) { k_gat_fwd_h1<VPL, L, 4><<<grid, 256, 0, s>>>(x); });
+        if (a.B)
+            two_buckets(a, split, n, 4,
+                        [&](GatFwdArgs x, unsigned grid) { launch_k(k_gat_fwd_h1<VPL, L, 32, true>, dim3(grid), dim3(256), 0, s, x); },
+                        [&](GatFwdArgs x, unsigned grid) { launch_k(k_gat_fwd_h1<VPL, L, 4, true>, dim3(grid), dim3(256), 0, s, x); });
+        else
+            two_buckets(a, split, n, 4,
+                        [&](GatFwdArgs x, unsigned grid) { launch_k(k_gat_fwd_h1<VPL, L, 32, false>, dim3(grid), dim3(256), 0, s, x); },
+                        [&](GatFwdArgs x, unsigned grid) { launch_k(k_gat_fwd_h1<VPL, L, 4, false>, dim3(grid), dim3(256), 0, s, x); });
     }
 };
 template <bool DER>
@@ -978,8 +1079,8 @@ struct BwdH1 {
     template <int VPL, int L>
     static void run(const GatBwdArgs& a, int64_t split, int64_t n, cudaStream_t s) {
         two_buckets(a, split, n, 4,
-                    [&](GatBwdArgs x, unsigned grid) { k_gat_bwd_h1<VPL, L, 32, DER><<<grid, 256, 0, s>>>(x); },
-                    [&](GatBwdArgs x, unsigned grid) { k_gat_bwd_h1<VPL, L, 4, DER><<<grid, 256, 0, s>>>(x); });
+                    [&](GatBwdArgs x, unsigned grid) { launch_k(k_gat_bwd_h1<VPL, L, 32, DER>, dim3(grid), dim3(256), 0, s, x); },
+                    [&](GatBwdArgs x, unsigned grid) { launch_k(k_gat_bwd_h1<VPL, L, 4, DER>, dim3(grid), dim3(256), 0, s, x); });
     }
 };
 template <class K, int VPL, class Args>
@@ -1015,21 +1116,21 @@ using namespace seastar;
         auto ls = [&](decltype(ARGS) x, unsigned grid) {                                                         \
             if (VEC4) {                                                                                          \
                 switch (L) {                                                                                     \
-                    case 1: KERNEL<4, 1, 4><<<grid, 256, 0, S>>>(x); break;                                      \
-                    case 2: KERNEL<4, 2, 4><<<grid, 256, 0, S>>>(x); break;                                      \
-                    case 4: KERNEL<4, 4, 4><<<grid, 256, 0, S>>>(x); break;                                      \
-                    case 8: KERNEL<4, 8, 8><<<grid, 256, 0, S>>>(x); break;                                      \
-                    case 16: KERNEL<4, 16, 16><<<grid, 256, 0, S>>>(x); break;                                   \
-                    default: KERNEL<4, 32, 32><<<grid, 256, 0, S>>>(x); break;                                   \
+                    case 1: launch_k(KERNEL<4, 1, 4>, dim3(grid), dim3(256), 0, S, x); break;                                      \
+                    case 2: launch_k(KERNEL<4, 2, 4>, dim3(grid), dim3(256), 0, S, x); break;                                      \
+                    case 4: launch_k(KERNEL<4, 4, 4>, dim3(grid), dim3(256), 0, S, x); break;                                      \
+                    case 8: launch_k(KERNEL<4, 8, 8>, dim3(grid), dim3(256), 0, S, x); break;                                      \
+                    case 16: launch_k(KERNEL<4, 16, 16>, dim3(grid), dim3(256), 0, S, x); break;                                   \
+                    default: launch_k(KERNEL<4, 32, 32>, dim3(grid), dim3(256), 0, S, x); break;                                   \
                 }                                                                                                \
             } else {                                                                                             \
                 switch (L) {                                                                                     \
-                    case 1: KERNEL<1, 1, 4><<<grid, 256, 0, S>>>(x); break;                                      \
-                    case 2: KERNEL<1, 2, 4><<<grid, 256, 0, S>>>(x); break;                                      \
-                    case 4: KERNEL<1, 4, 4><<<grid, 256, 0, S>>>(x); break;                                      \
-                    case 8: KERNEL<1, 8, 8><<<grid, 256, 0, S>>>(x); break;                                      \
-                    case 16: KERNEL<1, 16, 16><<<grid, 256, 0, S>>>(x); break;                                   \
-                    default: KERNEL<1, 32, 32><<<grid, 256, 0, S>>>(x); break;                                   \
+                    case 1: launch_k(KERNEL<1, 1, 4>, dim3(grid), dim3(256), 0, S, x); break;                                      \
+                    case 2: launch_k(KERNEL<1, 2, 4>, dim3(grid), dim3(256), 0, S, x); break;                                      \
+                    case 4: launch_k(KERNEL<1, 4, 4>, dim3(grid), dim3(256), 0, S, x); break;                                      \
+                    case 8: launch_k(KERNEL<1, 8, 8>, dim3(grid), dim3(256), 0, S, x); break;                                      \
+                    case 16: launch_k(KERNEL<1, 16, 16>, dim3(grid), dim3(256), 0, S, x); break;                                   \
+                    default: launch_k(KERNEL<1, 32, 32>, dim3(grid), dim3(256), 0, S, x); break;                                   \
                 }                                                                                                \
             }                                                                                                    \
         };                                                                                                       \
@@ -1053,8 +1154,11 @@ seastar_status seastar_gat_attn_proj(const float* T, int64_t M, int32_t H, int32
 
 seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float* el_all, const float* er_loc,
                                int32_t H, int32_t F, int64_t ldt, float slope, const float* bias, seastar_act act,
-                               float* A_loc, float* Y_loc, float* lse_loc, seastar_stream stream) {
+                               float* A_loc, float* Y_loc, float* lse_loc, float* B_loc, float* b_loc,
+                               seastar_stream stream) {
     SS_ARG(g && T_all && el_all && er_loc && A_loc && Y_loc && lse_loc, "gat_fwd: NULL argument");
+    SS_ARG((B_loc == nullptr) == (b_loc == nullptr), "gat_fwd: pass both B_loc and b_loc or neither");
+    SS_ARG(!B_loc || (aligned16(B_loc) == aligned16(A_loc)), "gat_fwd: B_loc must be aligned like A_loc");
     SS_ARG(H >= 1 && F >= 1 && ldt >= (int64_t)H * F, "gat_fwd: bad sizes H=%d F=%d ldt=%lld", H, F, (long long)ldt);
     SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "gat_fwd: bad activation");
     SS_TRY(check_device());
@@ -1064,12 +1168,13 @@ seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float*
     a.vbase = g->row_begin;
     a.T = T_all; a.el = el_all; a.er = er_loc;
     a.H = H; a.F = F; a.ld = ldt; a.slope = slope; a.bias = bias; a.act = act;
-    a.A = A_loc; a.Y = Y_loc; a.lse = lse_loc;
+    a.A = A_loc; a.Y = Y_loc; a.lse = lse_loc; a.B = B_loc; a.bsum = b_loc;
     const int f4 = hpl_f4(H, F, ldt, aligned16(T_all) && aligned16(A_loc) && aligned16(Y_loc));
     if (f4) {
         a.row_begin = 0; a.row_end = g->fwd.n_rows;
         const unsigned grid = (unsigned)((g->fwd.n_rows + 7) / 8);
-        if (grid) SS_HPL_SWITCH(k_gat_fwd_hpl, f4, grid, s, a);
+        if (grid && a.B) SS_HPL_SWITCH_SB(k_gat_fwd_hpl, true, f4, grid, s, a);
+        if (grid && !a.B) SS_HPL_SWITCH_SB(k_gat_fwd_hpl, false, f4, grid, s, a);
         return check_launch("k_gat_fwd_hpl");
     }
     int vpl = 0, Lh = 0;
@@ -1089,8 +1194,11 @@ seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float*
 
 seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const float* Y_loc, seastar_act act,
                                     const float* A_loc, const float* er_loc, const float* lse_loc, int32_t H,
-                                    int32_t F, int64_t ldt, float* D_loc, seastar_stream stream) {
+                                    int32_t F, int64_t ldt, float* D_loc, const float* B_loc, const float* b_loc,
+                                    float* der_loc, seastar_stream stream) {
     SS_ARG(g && dY_loc && A_loc && er_loc && lse_loc && D_loc, "gat_bwd_prep: NULL argument");
+    SS_ARG((B_loc == nullptr) == (b_loc == nullptr) && (B_loc == nullptr) == (der_loc == nullptr),
+           "gat_bwd_prep: pass B_loc, b_loc and der_loc together or none of them");
     SS_ARG(act == SEASTAR_ACT_NONE || Y_loc, "gat_bwd_prep: Y_loc is required for act != NONE");
     SS_ARG(H >= 1 && F >= 1 && ldt >= (int64_t)H * F, "gat_bwd_prep: bad sizes");
     SS_TRY(check_device());
@@ -1098,7 +1206,8 @@ seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const 
     if (M == 0) return SEASTAR_OK;
     const int64_t n = M * H;
     k_gat_bwd_prep<<<(unsigned)((n + 255) / 256), 256, 0, to_stream(stream)>>>(
-        M, H, F, ldt, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, D_loc, seastar_gat_record_ld(H, F));
+        M, H, F, ldt, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, D_loc, seastar_gat_record_ld(H, F), B_loc, b_loc,
+        der_loc);
     return check_launch("k_gat_bwd_prep");
 }
 
@@ -1115,6 +1224,7 @@ seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float*
     a.T = T_loc; a.el = el_loc; a.D = D_all;
     a.H = H; a.F = F; a.ldt = ldt; a.ldd = seastar_gat_record_ld(H, F); a.slope = slope;
     a.dT = dT_loc; a.del = del_loc;
+    ScopedL2Window win(D_all, (size_t)g->N * a.ldd * sizeof(float));
     const int f4 = hpl_f4(H, F, ldt, aligned16(T_loc) && aligned16(D_all) && aligned16(dT_loc));
     if (f4) {
         a.row_begin = 0; a.row_end = g->rev.n_rows;

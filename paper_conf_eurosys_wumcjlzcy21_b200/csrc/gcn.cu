@@ -64,7 +64,7 @@ __global__ void __launch_bounds__(256) k_aggregate(const AggArgs a) {
 
         for (int base = beg; base < end; base += RL) {
             const int n = min(RL, end - base);
-            const int my = (gl < n) ? __ldg(a.nbr + base + gl) : 0;
+            const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
 #pragma unroll
             for (int j0 = 0; j0 < L; j0 += UB) {
                 if (j0 * S >= n) break;
@@ -151,12 +151,12 @@ static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s) {
     constexpr int threads = 256;
     if (warp_rows) {
         const int64_t blocks = (rows + (threads / 32) - 1) / (threads / 32);
-        k_aggregate<VEC, L, 32><<<(unsigned)blocks, threads, 0, s>>>(a);
+        launch_k(k_aggregate<VEC, L, 32>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
     } else {
         constexpr int RL = L < 4 ? 4 : L;   // at least 4 lanes per row group keeps index loads useful
         const int64_t per_block = threads / RL;
         const int64_t blocks = (rows + per_block - 1) / per_block;
-        k_aggregate<VEC, L, RL><<<(unsigned)blocks, threads, 0, s>>>(a);
+        launch_k(k_aggregate<VEC, L, RL>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
     }
 }
 

@@ -7,6 +7,7 @@
 // (stable by construction, ranks from prefix scans), so the result is bit-exact and unique.
 #include <cub/cub.cuh>
 #include <stdarg.h>
+#include <stdlib.h>
 
 #include <mutex>
 #include <vector>
@@ -35,6 +36,28 @@ seastar_status check_launch(const char* where) {
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_status(e, where);
     return SEASTAR_OK;
+}
+
+thread_local L2Window t_l2win;
+
+size_t l2_persist_bytes() {
+    static std::mutex mu;
+    static long long per_dev[64];
+    static bool init[64] = {false};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 0;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!init[dev]) {
+        init[dev] = true;
+        per_dev[dev] = 0;
+        int maxp = 0;
+        if (getenv("SEASTAR_NO_L2_PERSIST") == nullptr &&
+            cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev) == cudaSuccess && maxp > 0 &&
+            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp) == cudaSuccess)
+            per_dev[dev] = maxp;
+        cudaGetLastError();
+    }
+    return (size_t)per_dev[dev];
 }
 
 seastar_status check_device() {

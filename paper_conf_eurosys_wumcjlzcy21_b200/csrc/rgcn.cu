@@ -102,8 +102,8 @@ __global__ void __launch_bounds__(512) k_rgcn_rows(const RgcnRowArgs a) {
             int my_u = 0, my_t = 0;
             float my_w = 0.f;
             if (gl < n) {
-                my_u = __ldg(a.nbr + base + gl);
-                my_t = __ldg(a.typ + base + gl);
+                my_u = __ldcs(a.nbr + base + gl);
+                my_t = __ldcs(a.typ + base + gl);
                 my_w = a.norm_user ? __ldg(a.norm_user + __ldg(a.eid + base + gl)) : __ldg(a.norm + base + gl);
             }
 #pragma unroll
@@ -258,7 +258,7 @@ static seastar_status launch_rows(const RgcnRowArgs& a, size_t smem, cudaStream_
     int64_t blocks = (int64_t)per_sm * num_sms();
     const int64_t need = (groups + (512 / RL) - 1) / (512 / RL);
     if (blocks > need) blocks = need;
-    k_rgcn_rows<L, RL><<<(unsigned)blocks, 512, smem, s>>>(a);
+    launch_k(k_rgcn_rows<L, RL>, dim3((unsigned)blocks), dim3(512), smem, s, a);
     return check_launch("k_rgcn_rows");
 }
 
@@ -309,6 +309,7 @@ seastar_status seastar_rgcn_fwd(seastar_graph g, const float* X_all, int64_t F_i
     a.vbase = g->row_begin;
     a.table = X_all; a.ldt = ldx; a.W = W; a.R = g->R; a.Fg = (int)F_in; a.Fo = (int)F_out; a.transpose = 0;
     a.out = Y_loc; a.ldo = ldy; a.bias = bias; a.act = act;
+    ScopedL2Window win(X_all, (size_t)g->N * ldx * sizeof(float));
     return launch_rows_L(g->fwd, a, to_stream(stream));
 }
 
@@ -341,6 +342,7 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
         a.vbase = g->row_begin;
         a.table = dA_all; a.ldt = ldd; a.W = W; a.R = g->R; a.Fg = (int)F_out; a.Fo = (int)F_in; a.transpose = 1;
         a.out = dX_loc; a.ldo = ldx; a.bias = nullptr; a.act = act; a.Yact = Yact_loc;
+        ScopedL2Window win(dA_all, (size_t)g->N * ldd * sizeof(float));
         SS_TRY(launch_rows_L(g->rev, a, s));
     }
     if (dW) {
@@ -352,13 +354,14 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
             d.n_tasks = g->tm.n_tasks;
             d.X = X_all; d.ldx = ldx; d.dA = dA_all; d.ldd = ldd; d.Fin = (int)F_in; d.Fout = (int)F_out;
             d.part = static_cast<float*>(workspace);
+            ScopedL2Window win(X_all, (size_t)g->N * ldx * sizeof(float));
             int64_t blocks = (g->tm.n_tasks + 7) / 8;
             const int64_t cap = 16 * (int64_t)num_sms();
             if (blocks > cap) blocks = cap;
             const int Cg = (int)((F_in + 3) / 4);
             const int L = pow2_ceil(Cg);
             const int npl = pow2_ceil((FF + 31) / 32);
-#define RGCN_DW(LL, NN) k_rgcn_dw<LL, NN><<<(unsigned)blocks, 256, 0, s>>>(d)
+#define RGCN_DW(LL, NN) launch_k(k_rgcn_dw<LL, NN>, dim3((unsigned)blocks), dim3(256), 0, s, d)
 #define RGCN_DW_L(LL)                                                   \
     switch (npl) {                                                      \
         case 1: RGCN_DW(LL, 1); break;                                  \

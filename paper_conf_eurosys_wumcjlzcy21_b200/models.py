@@ -197,11 +197,17 @@ class GCN2:
 
 class GAT2:
     """2-layer GAT (Fig. 2 / Fig. 3): F_in -> heads x hidden (ELU, concat) -> 1 x C, softmax-xent.
-    LeakyReLU slope 0.2, attention vectors a_l (source) / a_r (destination) per head."""
+    LeakyReLU slope 0.2, attention vectors a_l (source) / a_r (destination) per head.
+
+    save_der_factors=True (default): the forward also writes B_v, b_v so the backward row pass emits der
+    directly (one edge pass per layer backward instead of two); False uses the dst-major
+    seastar_gat_der pass instead (less memory)."""
 
     def __init__(self, g: Graph, X_loc: torch.Tensor, labels_loc: torch.Tensor, params: dict, heads: int,
-                 hidden: int, lr=0.005, slope=0.2, comm: Comm | None = None, n_pad_rows: int | None = None):
+                 hidden: int, lr=0.005, slope=0.2, comm: Comm | None = None, n_pad_rows: int | None = None,
+                 save_der_factors: bool = True):
         self.g, self.X, self.lab, self.lr, self.slope = g, X_loc, labels_loc, lr, slope
+        self.save_B = save_der_factors
         self.comm = comm or Comm()
         dev = X_loc.device
         self.n, self.N = g.n_loc, g.N
@@ -227,6 +233,8 @@ class GAT2:
         self.del1, self.del2 = e(n, heads), e(n, 1)
         self.der1, self.der2 = e(n, heads), e(n, 1)
         self.dY1 = e(n, self.ld1)
+        self.B1, self.bs1 = (e(n, self.ld1), e(n, heads)) if self.save_B else (None, None)
+        self.B2, self.bs2 = (e(n, self.ld2), e(n, 1)) if self.save_B else (None, None)
         self.loss = torch.zeros(1, device=dev)
         self.ws = _Ws(dev)
         P = self.comm.world
@@ -254,24 +262,26 @@ class GAT2:
         self._gathered1 = (T1_all, el1_all)
         self._t("gat_fwd1")
         L.seastar_gat_fwd(g.handle, T1_all, el1_all, self.er1, H, F, self.ld1, self.slope, p.p("b1"), "elu", self.A1,
-                          self.Y1, self.lse1)
+                          self.Y1, self.lse1, self.B1, self.bs1)
         self._t("gat_fwd1_end")
         L.seastar_linear_fwd(self.Y1, n, W, self.ld1, p.p("W2"), C, None, None, "none", self.T2, self.ld2)
         L.seastar_gat_attn_proj(self.T2, n, 1, C, self.ld2, p.p("al2"), p.p("ar2"), self.el2, self.er2)
         T2_all = self.comm.all_gather(self.T2_all, self.T2)
         el2_all = self.comm.all_gather(self.el2_all, self.el2)
         self._gathered2 = (T2_all, el2_all)
+        self._t("gat_fwd2")
         L.seastar_gat_fwd(g.handle, T2_all, el2_all, self.er2, 1, C, self.ld2, self.slope, p.p("b2"), "none", self.A2,
-                          self.Y2, self.lse2)
+                          self.Y2, self.lse2, self.B2, self.bs2)
+        self._t("gat_fwd2_end")
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
         L.seastar_softmax_xent(self.Y2, n, self.g.N, C, self.ld2, self.lab, self.loss, self.dY2, self.ld2, ws,
                                ws.numel())
         return self.loss
 
     def _layer_bwd(self, T, T_loc_ld, el, er, A, Y, lse, dY, act, H, F, D, D_all_buf, dT, del_, der, gathered,
-                   al, ar, dal, dar, db, tag):
+                   al, ar, dal, dar, db, tag, B, bs):
         g, n = self.g, self.n
-        L.seastar_gat_bwd_prep(g.handle, dY, Y, act, A, er, lse, H, F, T_loc_ld, D)
+        L.seastar_gat_bwd_prep(g.handle, dY, Y, act, A, er, lse, H, F, T_loc_ld, D, B, bs, der if B is not None else None)
         ldd = L.seastar_gat_record_ld(H, F)
         ws = self.ws.need(max(L.seastar_colsum_workspace(n, H * F), L.seastar_gat_attn_proj_bwd_workspace(n, H, F)))
         L.seastar_colsum(D, n, H * F, ldd, db, ws, ws.numel())       # db = sum_v dA[v] (dA = first H*F columns)
@@ -279,9 +289,10 @@ class GAT2:
         self._t(f"gat_bwd{tag}")
         L.seastar_gat_bwd(g.handle, T, el, D_all, H, F, T_loc_ld, self.slope, dT, del_)
         self._t(f"gat_bwd{tag}_end")
-        self._t(f"gat_der{tag}")
-        L.seastar_gat_der(g.handle, gathered[0], gathered[1], D, H, F, T_loc_ld, self.slope, der)
-        self._t(f"gat_der{tag}_end")
+        if B is None:
+            self._t(f"gat_der{tag}")
+            L.seastar_gat_der(g.handle, gathered[0], gathered[1], D, H, F, T_loc_ld, self.slope, der)
+            self._t(f"gat_der{tag}_end")
         L.seastar_gat_attn_proj_bwd(T, n, H, F, T_loc_ld, al, ar, del_, der, dT, dal, dar, ws, ws.numel())
 
     def backward(self):
@@ -289,14 +300,14 @@ class GAT2:
         H, F, W, C = self.H1, self.F1, self.W1w, self.C
         self._layer_bwd(self.T2, self.ld2, self.el2, self.er2, self.A2, self.Y2, self.lse2, self.dY2, "none", 1, C,
                         self.D2, self.D2_all, self.dT2, self.del2, self.der2, self._gathered2, p.p("al2"),
-                        p.p("ar2"), p.g("al2"), p.g("ar2"), p.g("b2"), "2")
+                        p.p("ar2"), p.g("al2"), p.g("ar2"), p.g("b2"), "2", self.B2, self.bs2)
         ws = self.ws.need(max(L.seastar_linear_bwd_weight_workspace(n, W, C),
                               L.seastar_linear_bwd_weight_workspace(n, self.Fin, W)))
         L.seastar_linear_bwd_weight(self.Y1, n, W, self.ld1, self.dT2, C, self.ld2, p.g("W2"), None, ws, ws.numel())
         L.seastar_linear_bwd_data(self.dT2, n, C, self.ld2, p.p("W2"), W, None, None, "none", self.dY1, self.ld1)
         self._layer_bwd(self.T1, self.ld1, self.el1, self.er1, self.A1, self.Y1, self.lse1, self.dY1, "elu", H, F,
                         self.D1, self.D1_all, self.dT1, self.del1, self.der1, self._gathered1, p.p("al1"),
-                        p.p("ar1"), p.g("al1"), p.g("ar1"), p.g("b1"), "1")
+                        p.p("ar1"), p.g("al1"), p.g("ar1"), p.g("b1"), "1", self.B1, self.bs1)
         ws = self.ws.need(L.seastar_linear_bwd_weight_workspace(n, self.Fin, W))
         L.seastar_linear_bwd_weight(self.X, n, self.Fin, self.X.stride(0), self.dT1, W, self.ld1, p.g("W1"), None, ws,
                                     ws.numel())

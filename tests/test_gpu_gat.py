@@ -26,13 +26,17 @@ def dev(env, a):
     return env["torch"].from_numpy(np.ascontiguousarray(a)).cuda()
 
 
-def run_fwd(env, g, N, H, F, ld, T, el, er, b, act, slope=0.2):
+def run_fwd(env, g, N, H, F, ld, T, el, er, b, act, slope=0.2, save_B=False):
     torch, L = env["torch"], env["L"]
     A = torch.full((N, ld), float("nan"), device="cuda")
     Y = torch.full((N, ld), float("nan"), device="cuda")
     lse = torch.empty((N, H), device="cuda")
+    B = torch.full((N, ld), float("nan"), device="cuda") if save_B else None
+    bs = torch.empty((N, H), device="cuda") if save_B else None
     L.seastar_gat_fwd(g.handle, dev(env, padded(T, ld)), dev(env, el), dev(env, er), H, F, ld, slope,
-                      None if b is None else dev(env, b), act, A, Y, lse)
+                      None if b is None else dev(env, b), act, A, Y, lse, B, bs)
+    if save_B:
+        return A, Y, lse, B, bs
     return A, Y, lse
 
 
@@ -94,7 +98,12 @@ def test_gat_bwd_chain(env, H, F):
     dY = rnd(15, (N, W))
     ldd = L.seastar_gat_record_ld(H, F)
     D = torch.empty((N, ldd), device="cuda")
-    L.seastar_gat_bwd_prep(g.handle, dev(env, padded(dY, ld)), Y, act, A, dev(env, er32), lse, H, F, ld, D)
+    # forward-saved der factors (B, b) -> the row pass emits der; must agree with the dst-major pass
+    A_b, Y_b, lse_b, Bf, bsf = run_fwd(env, g, N, H, F, ld, T, el32, er32, b, act, save_B=True)
+    assert torch.equal(A_b[:, :W], A[:, :W]) and torch.equal(lse_b, lse)   # saving B does not perturb the forward
+    dr_b = torch.empty((N, H), device="cuda")
+    L.seastar_gat_bwd_prep(g.handle, dev(env, padded(dY, ld)), Y, act, A, dev(env, er32), lse, H, F, ld, D, Bf, bsf,
+                           dr_b)
     dT = torch.full((N, ld), float("nan"), device="cuda")
     dl = torch.empty((N, H), device="cuda")
     Td = dev(env, padded(T, ld))
@@ -108,6 +117,7 @@ def test_gat_bwd_chain(env, H, F):
     assert rel_err(dT.cpu().numpy()[:, :W], dTr.reshape(N, W)) <= TOL
     assert rel_err(dl.cpu().numpy(), dlr) <= TOL
     assert rel_err(dr.cpu().numpy(), drr) <= TOL
+    assert rel_err(dr_b.cpu().numpy(), drr) <= TOL
     # projection backward: dT += del a_l + der a_r ; da_l, da_r
     ws_b = L.seastar_gat_attn_proj_bwd_workspace(N, H, F)
     ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")

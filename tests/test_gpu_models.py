@@ -46,7 +46,8 @@ def test_gcn2(env):
     assert not np.array_equal(m.P.p("W1").cpu().numpy(), p["W1"])
 
 
-def test_gat2(env):
+@pytest.mark.parametrize("save_B", [True, False])
+def test_gat2(env, save_B):
     ip, ix = synth.powerlaw_sym(1500, 12000, 0.6, 32)
     N, Fin, heads, hid, C = 1500, 200, 8, 8, 41
     X, lab = synth.uniform(11, (N, Fin)), synth.labels(12, N, C)
@@ -54,7 +55,7 @@ def test_gat2(env):
          "ar1": synth.uniform(15, (heads, hid), -0.5, 0.5), "b1": synth.uniform(16, (heads * hid,), -0.1, 0.1),
          "W2": synth.glorot(17, heads * hid, C), "al2": synth.uniform(18, (1, C), -0.5, 0.5),
          "ar2": synth.uniform(19, (1, C), -0.5, 0.5), "b2": synth.uniform(20, (C,), -0.1, 0.1)}
-    m = env["models"].GAT2(env["Graph"](ip, ix), dev(env, X), dev(env, lab), p, heads, hid)
+    m = env["models"].GAT2(env["Graph"](ip, ix), dev(env, X), dev(env, lab), p, heads, hid, save_der_factors=save_B)
     check(m, *model_ref.gat2(ip, ix, X, lab, {k: v.astype(np.float64) for k, v in p.items()}, heads, hid))
 
 
