@@ -146,11 +146,15 @@ seastar_status seastar_graph_degree_norms(seastar_graph g, int32_t mode, float* 
 /*
  * Y[r,:] = row_scale[r] * act(X[r,:] W + bias)      for r < M
  *   X (dev) [M,K] ld ldx ; W (dev) [K,Nout] row-major (ld Nout) ; bias [Nout] or NULL ;
- *   row_scale [M] or NULL ; Y (dev) [M,Nout] ld ldy.  fp32 in, fp32 accumulate, fp32 out.
+ *   row_scale [M] or NULL ; Y (dev) [M,Nout] ld ldy.  fp32 in / out, fp32-accurate.
+ * With a workspace of seastar_linear_fwd_workspace(K, Nout) bytes, ldx % 4 == 0, a 16-byte aligned X,
+ * M >= 128, K >= 32 and Nout <= 128 it runs on the tcgen05 tensor cores (TMA-fed, TMEM accumulators,
+ * 3xTF32 hi/lo split: W is split once per call into the workspace); otherwise a SIMT fp32 kernel.
  */
 seastar_status seastar_linear_fwd(const float* X, int64_t M, int64_t K, int64_t ldx, const float* W,
                                   int64_t Nout, const float* bias, const float* row_scale, seastar_act act,
-                                  float* Y, int64_t ldy, seastar_stream stream);
+                                  float* Y, int64_t ldy, void* workspace, size_t ws_bytes, seastar_stream stream);
+size_t seastar_linear_fwd_workspace(int64_t K, int64_t Nout);
 /*
  * dX[r,:] = row_scale[r] * (dY[r,:] W^T) * act'(Yact[r,:])
  *   dY [M,Nout] ld ldy ; W [K,Nout] row-major ; row_scale [M] or NULL ; Yact [M,K] ld ldx or NULL (the

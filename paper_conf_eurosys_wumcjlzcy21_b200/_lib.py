@@ -59,7 +59,8 @@ _SIGS = {
     "seastar_graph_info": ([_P, ctypes.POINTER(seastar_graph_info_t)], _ST),
     "seastar_graph_export": ([_P, _I32, _P, _P, _P, _P, _P, _P, _P, _P], _ST),
     "seastar_graph_degree_norms": ([_P, _I32, _P, _P, _P], _ST),
-    "seastar_linear_fwd": ([_P, _I64, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
+    "seastar_linear_fwd": ([_P, _I64, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P, _SZ, _P], _ST),
+    "seastar_linear_fwd_workspace": ([_I64, _I64], _SZ),
     "seastar_linear_bwd_data": ([_P, _I64, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
     "seastar_linear_bwd_weight": ([_P, _I64, _I64, _I64, _P, _I64, _I64, _P, _P, _P, _SZ, _P], _ST),
     "seastar_linear_bwd_weight_workspace": ([_I64, _I64, _I64], _SZ),
@@ -197,9 +198,15 @@ def seastar_graph_degree_norms(g, mode, src_norm_loc=None, dst_norm_loc=None, st
 
 
 # ----------------------------------------------------------------------------------- dense
-def seastar_linear_fwd(X, M, K, ldx, W, Nout, bias, row_scale, act, Y, ldy, stream=None) -> None:
+def seastar_linear_fwd_workspace(K, Nout) -> int:
+    return int(load().seastar_linear_fwd_workspace(K, Nout))
+
+
+def seastar_linear_fwd(X, M, K, ldx, W, Nout, bias, row_scale, act, Y, ldy, workspace=None, ws_bytes=0,
+                       stream=None) -> None:
     _call("seastar_linear_fwd", _dptr(X, "X"), M, K, ldx, _dptr(W, "W"), Nout, _dptr(bias, "bias"),
-          _dptr(row_scale, "row_scale"), _act(act), _dptr(Y, "Y"), ldy, _stream(stream))
+          _dptr(row_scale, "row_scale"), _act(act), _dptr(Y, "Y"), ldy, _dptr(workspace, "workspace"), ws_bytes,
+          _stream(stream))
 
 
 def seastar_linear_bwd_data(dY, M, Nout, ldy, W, K, row_scale, Yact, act, dX, ldx, stream=None) -> None:

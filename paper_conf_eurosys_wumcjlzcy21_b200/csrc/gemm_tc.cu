@@ -1,0 +1,345 @@
+// gemm_tc.cu -- a4: the dense per-layer transform Y = row_scale * act(X W + bias) on the 5th-generation
+// tensor cores (tcgen05, kind::tf32) with an fp32-accurate 3xTF32 split.
+//
+// Shape: X [M, K] row-major fp32 (M = vertices, up to millions; K = feature width), W [K, N] (N <= 256).
+// One CTA computes a 128 x NP tile (NP = N rounded up to 16) over the whole K range:
+//   warp 0      : TMA producer -- cp.async.bulk.tensor loads 128 x 32 fp32 X tiles (SWIZZLE_128B) into a
+//                 STAGES-deep ring, completion signalled on an mbarrier (expect_tx);
+//   warps 2..5  : split -- per stage, X_hi = rna_tf32(X) in place and X_lo = X - X_hi, and the W chunk
+//                 (read from L2, written K-major with the same 128B swizzle) as W_hi / W_lo;
+//                 then the epilogue (tcgen05.ld of the TMEM accumulator, bias / activation / row scale);
+//   warp 1      : TMEM allocation and the MMA issuer -- one elected thread issues, per 8-wide K step,
+//                 hi*hi + hi*lo + lo*hi into the fp32 accumulator in TMEM and commits each stage back to
+//                 the producer (tcgen05.commit -> mbarrier).
+// Because X_hi and W_hi are exactly representable in tf32 the products are independent of how the MMA
+// unit rounds its inputs; the dropped lo*lo term is < 2^-22 relative.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <mutex>
+
+#include "common.cuh"
+
+namespace seastar {
+
+struct TcArgs {
+    int64_t M, K, N;
+    const float* Wsplit;            // [nk][W_hi tile | W_lo tile], each NP x 32 K-major, 128B-swizzled
+    float* Y; int64_t ldy;
+    const float* bias; const float* row_scale; int act;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    const uint32_t a = smem_u32(bar);
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}" ::"r"(a), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* tm, int x, int y, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+        ::"r"(smem_u32(dst)), "l"(reinterpret_cast<uint64_t>(tm)), "r"(x), "r"(y), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void bulk_copy(void* dst, const float* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(reinterpret_cast<uint64_t>(src)), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ float rna_tf32(float x) {
+    uint32_t r;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+    return __uint_as_float(r);
+}
+// K-major operand, 128B swizzle, 8-row groups 1024 B apart (sm100 descriptor version 1)
+__device__ __forceinline__ uint64_t smem_desc_k128(const void* p) {
+    const uint32_t a = smem_u32(p);
+    uint64_t d = (uint64_t)((a >> 4) & 0x3FFF);
+    d |= (uint64_t)1 << 16;                 // leading byte offset (unused for swizzled K-major)
+    d |= (uint64_t)(1024 >> 4) << 32;       // stride byte offset
+    d |= (uint64_t)1 << 46;                 // version
+    d |= (uint64_t)2 << 61;                 // SWIZZLE_128B
+    return d;
+}
+__device__ __forceinline__ void mma_tf32(uint32_t tmem, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}" ::"r"(tmem), "l"(da), "l"(db), "r"(idesc),
+        "r"(acc));
+}
+__device__ __forceinline__ void mma_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+                 : "memory");
+}
+
+template <int NP>
+struct TcCfg {
+    static constexpr int BM = 128, BK = 32;
+    static constexpr int STAGES = NP <= 64 ? 4 : (NP <= 128 ? 3 : 2);
+    static constexpr uint32_t A_BYTES = BM * BK * 4;          // 16 KB
+    static constexpr uint32_t B_BYTES = NP * BK * 4;          // NP rows of 128 B
+    static constexpr uint32_t STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
+    // G independent accumulators, K-chunk kc -> accumulator kc % G: each accumulates ~nk/G chunks, which
+    // bounds the error of the tensor core's accumulation; the epilogue sums them in fp32 registers
+    static constexpr int G = NP <= 64 ? 8 : (NP <= 128 ? 4 : 2);
+    static constexpr uint32_t TMEM_COLS = (G * NP) <= 32 ? 32 : ((G * NP) <= 64 ? 64 : ((G * NP) <= 128 ? 128 :
+                                          ((G * NP) <= 256 ? 256 : 512)));
+    static constexpr size_t SMEM = (size_t)STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+};
+
+template <int NP>
+__global__ void __launch_bounds__(192, 1) k_gemm_tc(const __grid_constant__ CUtensorMap tmX, const TcArgs a) {
+    using C = TcCfg<NP>;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + (size_t)C::STAGES * C::STAGE_BYTES);
+    uint64_t* full = bars;                       // TMA landed
+    uint64_t* split = bars + C::STAGES;          // hi/lo written (128 arrivals)
+    uint64_t* empty = bars + 2 * C::STAGES;      // MMAs done reading
+    uint64_t* accum = bars + 3 * C::STAGES;      // accumulator complete
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * C::STAGES + 1);
+    auto A_hi = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES; };
+    auto A_lo = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + C::A_BYTES; };
+    auto B_hi = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + 2 * C::A_BYTES; };
+    auto B_lo = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + 2 * C::A_BYTES + C::B_BYTES; };
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t m0 = (int64_t)blockIdx.x * C::BM;
+    const int nk = (int)((a.K + C::BK - 1) / C::BK);
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < C::STAGES; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&split[s], 128);
+            mbar_init(&empty[s], 1);
+        }
+        mbar_init(accum, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(C::TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0) {
+        // ---------------- TMA producer ----------------
+        if (lane == 0) {
+            for (int kc = 0; kc < nk; ++kc) {
+                const int s = kc % C::STAGES;
+                if (kc >= C::STAGES) mbar_wait(&empty[s], ((kc / C::STAGES) - 1) & 1);
+                mbar_expect_tx(&full[s], C::A_BYTES + 2 * C::B_BYTES);
+                tma_load_2d(A_hi(s), &tmX, kc * C::BK, (int)m0, &full[s]);
+                // the pre-split, pre-swizzled W_hi | W_lo tiles of this K chunk: one contiguous bulk copy
+                bulk_copy(B_hi(s), a.Wsplit + (size_t)kc * 2 * C::B_BYTES / sizeof(float), 2 * C::B_BYTES, &full[s]);
+            }
+        }
+    } else if (warp == 1) {
+        // ---------------- MMA issuer ----------------
+        // instruction descriptor: D f32, A/B tf32, both K-major, N = NP, M = 128
+        const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NP >> 3) << 17) | ((128u >> 4) << 24);
+        for (int kc = 0; kc < nk; ++kc) {
+            const int s = kc % C::STAGES;
+            mbar_wait(&split[s], (kc / C::STAGES) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            if (lane == 0) {
+                const uint64_t ah = smem_desc_k128(A_hi(s)), al = smem_desc_k128(A_lo(s));
+                const uint64_t bh = smem_desc_k128(B_hi(s)), bl = smem_desc_k128(B_lo(s));
+#pragma unroll
+                const uint32_t d = tmem + (uint32_t)((kc % C::G) * NP);
+#pragma unroll
+                for (int ks = 0; ks < C::BK / 8; ++ks) {
+                    const uint64_t adv = (uint64_t)((ks * 8 * 4) >> 4);   // 32 B per 8-wide K step
+                    mma_tf32(d, al + adv, bh + adv, idesc, (kc >= C::G || ks > 0) ? 1u : 0u);
+                    mma_tf32(d, ah + adv, bl + adv, idesc, 1u);
+                    mma_tf32(d, ah + adv, bh + adv, idesc, 1u);
+                }
+                mma_commit(&empty[s]);
+                if (kc == nk - 1) mma_commit(accum);
+            }
+            __syncwarp();
+        }
+    } else {
+        // ---------------- split (then epilogue) ----------------
+        const int t = threadIdx.x - 64;                     // 0..127
+        for (int kc = 0; kc < nk; ++kc) {
+            const int s = kc % C::STAGES;
+            const int k0 = kc * C::BK;
+            // full[s] also proves the MMAs of this stage's previous use are done (the producer armed it
+            // only after empty[s]), so the stage's W buffers may be rewritten now
+            mbar_wait(&full[s], (kc / C::STAGES) & 1);
+            (void)k0;
+            // elementwise over the 16 KB tile, consecutive lanes on consecutive 16 B chunks (conflict-free;
+            // the swizzle only permutes chunks, so hi and lo land at the same offsets as their source)
+            float4* ph = reinterpret_cast<float4*>(A_hi(s));
+            float4* pl = reinterpret_cast<float4*>(A_lo(s));
+            float4 xv[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) xv[q] = ph[q * 128 + t];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const float4 x = xv[q];
+                const float4 h = make_float4(rna_tf32(x.x), rna_tf32(x.y), rna_tf32(x.z), rna_tf32(x.w));
+                ph[q * 128 + t] = h;
+                pl[q * 128 + t] = make_float4(x.x - h.x, x.y - h.y, x.z - h.z, x.w - h.w);
+            }
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive(&split[s]);
+        }
+        // ---------------- epilogue ----------------
+        mbar_wait(accum, 0);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const int q4 = warp & 3;                         // TMEM lane quarter accessible to this warp
+        const int r = q4 * 32 + lane;
+        const int64_t gm = m0 + r;
+        const float rs = (gm < a.M && a.row_scale) ? __ldg(a.row_scale + gm) : 1.f;
+        const int nacc = nk < C::G ? nk : C::G;
+#pragma unroll 1
+        for (int c0 = 0; c0 < NP; c0 += 16) {
+            float accv[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) accv[j] = 0.f;
+            for (int g = 0; g < nacc; ++g) {          // fixed order: deterministic
+                uint32_t v[16];
+                asm volatile(
+                    "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
+                    "[%16];"
+                    : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                      "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+                      "=r"(v[15])
+                    : "r"(tmem + ((uint32_t)(q4 * 32) << 16) + (uint32_t)(g * NP + c0)));
+                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+                for (int j = 0; j < 16; ++j) accv[j] += __uint_as_float(v[j]);
+            }
+            if (gm < a.M) {
+                float* y = a.Y + gm * a.ldy;
+#pragma unroll
+                for (int j = 0; j < 16; ++j) {
+                    const int64_t n = c0 + j;
+                    if (n < a.N) {
+                        const float z = accv[j] + (a.bias ? __ldg(a.bias + n) : 0.f);
+                        y[n] = rs * act_apply(a.act, z);
+                    }
+                }
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 1) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C::TMEM_COLS));
+    }
+}
+
+// W [K, N] -> per 32-wide K chunk: W_hi = rna_tf32(W) and W_lo = W - W_hi as NP x 32 K-major tiles in the
+// 128B-swizzled layout the UMMA descriptor expects (element (n, k) at n*128 + ((k/4 ^ n%8)*16 | (k%4)*4))
+__global__ void k_split_w(const float* __restrict__ W, int64_t K, int64_t N, int NP, float* __restrict__ out) {
+    const int64_t nk = (K + 31) / 32;
+    const int64_t total = nk * NP * 32;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t kc = i / (NP * 32);
+        const int r = (int)(i % (NP * 32));
+        const int n = r / 32, k = r % 32;
+        const int64_t gk = kc * 32 + k;
+        const float w = (n < N && gk < K) ? W[gk * N + n] : 0.f;
+        const float wh = rna_tf32(w);
+        const uint32_t off = (uint32_t)(n * 128 + ((((k >> 2) ^ (n & 7)) << 4) | ((k & 3) << 2))) / 4;
+        float* tile = out + kc * 2 * NP * 32;
+        tile[off] = wh;
+        tile[NP * 32 + off] = w - wh;
+    }
+}
+
+size_t linear_fwd_tc_workspace(int64_t K, int64_t N) {
+    const int64_t np = (N + 15) / 16 * 16;
+    return (size_t)((K + 31) / 32) * 2 * np * 32 * sizeof(float) + 256;
+}
+
+// ------------------------------------------------------------------------------------------------
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+        cudaGetLastError();
+    });
+    return fn;
+}
+
+template <int NP>
+static seastar_status launch_tc_np(const CUtensorMap& tm, const TcArgs& a, cudaStream_t s) {
+    using C = TcCfg<NP>;
+    static bool attr = false;
+    if (!attr) {
+        SS_CUDA(cudaFuncSetAttribute(k_gemm_tc<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
+        attr = true;
+    }
+    const unsigned grid = (unsigned)((a.M + C::BM - 1) / C::BM);
+    k_gemm_tc<NP><<<grid, 192, C::SMEM, s>>>(tm, a);
+    return check_launch("k_gemm_tc");
+}
+
+// returns SEASTAR_ERR_UNSUPPORTED (without launching) when the tensor-core path does not apply
+seastar_status linear_fwd_tc(const float* X, int64_t M, int64_t K, int64_t ldx, const float* W, int64_t N,
+                             const float* bias, const float* row_scale, int act, float* Y, int64_t ldy,
+                             void* ws, size_t ws_bytes, cudaStream_t s) {
+    if (getenv("SEASTAR_NO_TCGEN05") || M < 128 || K < 32 || N > 128 || (ldx % 4) != 0 || !aligned16(X) ||
+        M >= (1LL << 31) || K >= (1LL << 31) || !ws || !aligned16(ws) || ws_bytes < linear_fwd_tc_workspace(K, N))
+        return SEASTAR_ERR_UNSUPPORTED;
+    auto enc = encode_fn();
+    if (!enc) return SEASTAR_ERR_UNSUPPORTED;
+    CUtensorMap tm;
+    cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)M};
+    cuuint64_t strides[1] = {(cuuint64_t)ldx * sizeof(float)};
+    cuuint32_t box[2] = {32, 128};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(X), dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return SEASTAR_ERR_UNSUPPORTED;
+    const int np = (int)((N + 15) / 16 * 16);
+    float* wsplit = static_cast<float*>(ws);
+    {
+        const int64_t total = (K + 31) / 32 * np * 32;
+        k_split_w<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(W, K, N, np, wsplit);
+        SS_TRY(check_launch("k_split_w"));
+    }
+    TcArgs a{M, K, N, wsplit, Y, ldy, bias, row_scale, act};
+    switch (np) {
+        case 16: return launch_tc_np<16>(tm, a, s);
+        case 32: return launch_tc_np<32>(tm, a, s);
+        case 48: return launch_tc_np<48>(tm, a, s);
+        case 64: return launch_tc_np<64>(tm, a, s);
+        case 80: return launch_tc_np<80>(tm, a, s);
+        case 96: return launch_tc_np<96>(tm, a, s);
+        case 128: return launch_tc_np<128>(tm, a, s);
+        default: return SEASTAR_ERR_UNSUPPORTED;
+    }
+}
+
+}  // namespace seastar

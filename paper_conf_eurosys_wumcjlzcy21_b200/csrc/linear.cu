@@ -213,6 +213,10 @@ static void tn_geometry(int64_t M, int64_t K, int64_t& ktiles, int64_t& nsplit, 
 
 seastar_status colsum_impl(const float* X, int64_t M, int64_t F, int64_t ld, float* out, void* ws, size_t ws_bytes,
                            cudaStream_t s);
+seastar_status linear_fwd_tc(const float* X, int64_t M, int64_t K, int64_t ldx, const float* W, int64_t N,
+                             const float* bias, const float* row_scale, int act, float* Y, int64_t ldy,
+                             void* ws, size_t ws_bytes, cudaStream_t s);
+size_t linear_fwd_tc_workspace(int64_t K, int64_t N);
 size_t colsum_ws(int64_t M, int64_t F);
 
 }  // namespace seastar
@@ -221,13 +225,19 @@ using namespace seastar;
 
 extern "C" {
 
+size_t seastar_linear_fwd_workspace(int64_t K, int64_t Nout) { return linear_fwd_tc_workspace(K, Nout); }
+
 seastar_status seastar_linear_fwd(const float* X, int64_t M, int64_t K, int64_t ldx, const float* W, int64_t Nout,
                                   const float* bias, const float* row_scale, seastar_act act, float* Y, int64_t ldy,
-                                  seastar_stream stream) {
+                                  void* workspace, size_t ws_bytes, seastar_stream stream) {
     SS_ARG(X && W && Y, "linear_fwd: NULL argument");
     SS_ARG(M >= 0 && K >= 1 && Nout >= 1 && ldx >= K && ldy >= Nout, "linear_fwd: bad sizes");
     SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "linear_fwd: bad activation");
     SS_TRY(check_device());
+    // tcgen05 3xTF32 path (TMA needs ldx % 4 == 0 and a 16-byte aligned X); SIMT fp32 otherwise
+    const seastar_status st =
+        linear_fwd_tc(X, M, K, ldx, W, Nout, bias, row_scale, act, Y, ldy, workspace, ws_bytes, to_stream(stream));
+    if (st != SEASTAR_ERR_UNSUPPORTED) return st;
     GemmArgs g{X, ldx, W, Nout, 1, Y, ldy, M, K, Nout, bias, row_scale, act, nullptr, 0};
     return launch_gemm(g, to_stream(stream));
 }

@@ -91,6 +91,12 @@ class _Params:
         L.seastar_adam(self.flat, self.grad, self.m, self.v, self.n, lr, b1, b2, eps, self.step)
 
 
+def _linear(ws, X, M, K, ldx, W, N, bias, row_scale, act, Y, ldy):
+    """seastar_linear_fwd with its workspace (tensor-core path: W is split into tf32 hi/lo tiles there)."""
+    buf = ws.need(L.seastar_linear_fwd_workspace(K, N))
+    L.seastar_linear_fwd(X, M, K, ldx, W, N, bias, row_scale, act, Y, ldy, buf, buf.numel())
+
+
 class _Ws:
     """Grow-only byte workspace shared by the deterministic reductions."""
 
@@ -154,7 +160,7 @@ class GCN2:
 
     def forward(self):
         g, p, H, C, n = self.g, self.P, self.H, self.C, self.n
-        L.seastar_linear_fwd(self.X, n, self.Fin, self.X.stride(0), p.p("W1"), H, None, self.src_n, "none",
+        _linear(self.ws, self.X, n, self.Fin, self.X.stride(0), p.p("W1"), H, None, self.src_n, "none",
                              self.T1, H)
         T1_all = self.comm.all_gather(self.T1_all, self.T1)
         self._t("gcn_fwd1")
@@ -163,7 +169,7 @@ class GCN2:
         self._t("gcn_fwd1_end")
         H1s_all = self.comm.all_gather(self.H1s_all, self.H1s)
         L.seastar_gcn_fwd(g.handle, H1s_all, H, H, self.dst_n, None, "none", 0.0, None, self.P2)
-        L.seastar_linear_fwd(self.P2, n, H, H, p.p("W2"), C, p.p("b2"), None, "none", self.logits, self.ldc)
+        _linear(self.ws, self.P2, n, H, H, p.p("W2"), C, p.p("b2"), None, "none", self.logits, self.ldc)
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
         L.seastar_softmax_xent(self.logits, n, self.g.N, C, self.ldc, self.lab, self.loss, self.dlogits, self.ldc,
                                ws, ws.numel())
@@ -254,7 +260,7 @@ class GAT2:
     def forward(self):
         g, p, n = self.g, self.P, self.n
         H, F, W, C = self.H1, self.F1, self.W1w, self.C
-        L.seastar_linear_fwd(self.X, n, self.Fin, self.X.stride(0), p.p("W1"), W, None, None, "none", self.T1,
+        _linear(self.ws, self.X, n, self.Fin, self.X.stride(0), p.p("W1"), W, None, None, "none", self.T1,
                              self.ld1)
         L.seastar_gat_attn_proj(self.T1, n, H, F, self.ld1, p.p("al1"), p.p("ar1"), self.el1, self.er1)
         T1_all = self.comm.all_gather(self.T1_all, self.T1)
@@ -264,7 +270,7 @@ class GAT2:
         L.seastar_gat_fwd(g.handle, T1_all, el1_all, self.er1, H, F, self.ld1, self.slope, p.p("b1"), "elu", self.A1,
                           self.Y1, self.lse1, self.B1, self.bs1)
         self._t("gat_fwd1_end")
-        L.seastar_linear_fwd(self.Y1, n, W, self.ld1, p.p("W2"), C, None, None, "none", self.T2, self.ld2)
+        _linear(self.ws, self.Y1, n, W, self.ld1, p.p("W2"), C, None, None, "none", self.T2, self.ld2)
         L.seastar_gat_attn_proj(self.T2, n, 1, C, self.ld2, p.p("al2"), p.p("ar2"), self.el2, self.er2)
         T2_all = self.comm.all_gather(self.T2_all, self.T2)
         el2_all = self.comm.all_gather(self.el2_all, self.el2)
@@ -357,10 +363,10 @@ class APPNPNet:
 
     def forward(self):
         g, p, n, Hd, C, ld = self.g, self.P, self.n, self.Hd, self.C, self.ldc
-        L.seastar_linear_fwd(self.X, n, self.Fin, self.X.stride(0), p.p("W1"), Hd, p.p("b1"), None, "relu", self.Hh,
+        _linear(self.ws, self.X, n, self.Fin, self.X.stride(0), p.p("W1"), Hd, p.p("b1"), None, "relu", self.Hh,
                              Hd)
-        L.seastar_linear_fwd(self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), None, "none", self.H0, ld)
-        L.seastar_linear_fwd(self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), self.nrm, "none", self.Zs[0], ld)
+        _linear(self.ws, self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), None, "none", self.H0, ld)
+        _linear(self.ws, self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), self.nrm, "none", self.Zs[0], ld)
         for k in range(self.K):
             Zs_all = self.comm.all_gather(self.Zs_all, self.Zs[k])
             L.seastar_gcn_fwd(g.handle, Zs_all, C, ld, self.nrm, None, "none", self.alpha, self.H0, self.Z[k + 1],
@@ -374,7 +380,7 @@ class APPNPNet:
         g, p, n, Hd, C, ld, a = self.g, self.P, self.n, self.Hd, self.C, self.ldc, self.alpha
         # G = dL/dZ^K ; for k = K-1..0: dH0 += a G ; G <- (1-a) n sum_out n G
         self.dH0.zero_()
-        L.seastar_linear_fwd(self.G, n, C, ld, self._eye(C), C, None, self.nrm, "none", self.Gs[0], ld) \
+        _linear(self.ws, self.G, n, C, ld, self._eye(C), C, None, self.nrm, "none", self.Gs[0], ld) \
             if self.K > 0 else None
         cur = 0
         G = self.G

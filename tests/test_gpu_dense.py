@@ -42,6 +42,33 @@ def test_linear_fwd(env, M, K, N):
     assert np.isnan(Y.cpu().numpy()[:, N:]).all()
 
 
+TC_SHAPES = [(128, 32, 16), (1000, 602, 16), (5003, 602, 64), (777, 64, 41), (3001, 1433, 70), (300, 8710, 8),
+             (2048, 100, 128), (129, 33, 1)]
+
+
+@pytest.mark.parametrize("M,K,N", TC_SHAPES)
+def test_linear_fwd_tcgen05(env, M, K, N):
+    """ldx % 4 == 0 and 16-B aligned X -> the tcgen05 3xTF32 kernel (TMA + TMEM); must meet the fp32 tolerance."""
+    torch, L = env["torch"], env["L"]
+    X, W, b = rnd(41, (M, K)), rnd(42, (K, N)), rnd(43, (N,))
+    rs = rnd(44, (M,), 0.5, 2.0)
+    ldx = (K + 3) // 4 * 4 + 4
+    ldy = (N + 3) // 4 * 4
+    Y = torch.full((M, ldy), float("nan"), device="cuda")
+    ws_b = L.seastar_linear_fwd_workspace(K, N)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    L.seastar_linear_fwd(dev(env, padded(X, ldx)), M, K, ldx, dev(env, W), N, dev(env, b), dev(env, rs), "relu",
+                         Y, ldy, ws, ws_b)
+    ref = oracle.act_fwd("relu", oracle.linear_fwd(X, W, b)) * rs.astype(np.float64)[:, None]
+    assert rel_err(Y.cpu().numpy()[:, :N], ref) <= TOL
+    if ldy > N:
+        assert np.isnan(Y.cpu().numpy()[:, N:]).all()
+    # large-magnitude inputs: the hi/lo split keeps fp32 accuracy (1xTF32 would miss by ~1e-3)
+    X2 = (X.astype(np.float64) * 1e3 + 0.123456789).astype(np.float32)
+    L.seastar_linear_fwd(dev(env, padded(X2, ldx)), M, K, ldx, dev(env, W), N, None, None, "none", Y, ldy, ws, ws_b)
+    assert rel_err(Y.cpu().numpy()[:, :N], oracle.linear_fwd(X2, W)) <= TOL
+
+
 @pytest.mark.parametrize("M,K,N", SHAPES)
 def test_linear_bwd(env, M, K, N):
     torch, L = env["torch"], env["L"]
