@@ -76,9 +76,11 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
 #pragma unroll
     for (int i = 0; i < VEC; ++i) acc[i] = pacc[i] = 0.f;
 
+    int nxt = (gl < end - beg) ? __ldcs(a.nbr + beg + gl) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
+        const int my = nxt;
+        nxt = (gl < end - base - RL) ? __ldcs(a.nbr + base + RL + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -190,9 +192,11 @@ __global__ void __launch_bounds__(256) k_gat_fwd_hpl(const GatFwdArgs a) {
     for (int i = 0; i < F; ++i) acc[i] = 0.f;
 #pragma unroll
     for (int i = 0; i < (SB ? F : 1); ++i) pacc[i] = 0.f;
+    int nxt = (lane < end - beg) ? __ldcs(a.nbr + beg + lane) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += 32) {
         const int n = min(32, end - base);
-        const int my = (lane < n) ? __ldcs(a.nbr + base + lane) : 0;
+        const int my = nxt;
+        nxt = (lane < end - base - 32) ? __ldcs(a.nbr + base + 32 + lane) : 0;
         for (int i0 = 0; i0 < H; i0 += UB) {             // this slot's edges: k = slot + S * i
             if (i0 * S >= n) break;
             float z[UB], x[UB][F];
@@ -338,9 +342,11 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
 #pragma unroll
     for (int i = 0; i < VEC; ++i) acc[i] = 0.f;
 
+    int nxt = (gl < end - beg) ? __ldcs(a.nbr + beg + gl) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int myv = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
+        const int myv = nxt;
+        nxt = (gl < end - base - RL) ? __ldcs(a.nbr + base + RL + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -437,9 +443,11 @@ __global__ void __launch_bounds__(256) k_gat_der(const GatBwdArgs a) {
     for (int i = 0; i < VEC; ++i)
         if (!(valid && active) || col + i >= W) d[i] = 0.f;
     float dr = 0.f;
+    int nxt = (gl < end - beg) ? __ldcs(a.nbr + beg + gl) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
+        const int my = nxt;
+        nxt = (gl < end - base - RL) ? __ldcs(a.nbr + base + RL + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -510,9 +518,11 @@ __global__ void __launch_bounds__(256) k_gat_bwd_hpl(const GatBwdArgs a) {
     for (int i = 0; i < F; ++i) acc[i] = 0.f;
     const float elu = __ldg(a.el + u * H + h);
     float dl = 0.f;
+    int nxt = (lane < end - beg) ? __ldcs(a.nbr + beg + lane) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += 32) {
         const int n = min(32, end - base);
-        const int my = (lane < n) ? __ldcs(a.nbr + base + lane) : 0;
+        const int my = nxt;
+        nxt = (lane < end - base - 32) ? __ldcs(a.nbr + base + 32 + lane) : 0;
         for (int i0 = 0; i0 < H; i0 += UB) {
             if (i0 * S >= n) break;
             float d[UB][F], ax[UB][3];
@@ -587,9 +597,11 @@ __global__ void __launch_bounds__(256) k_gat_der_hpl(const GatBwdArgs a) {
     const float4 x4 = ldg4(rec + rec_aux_offset(H * F) + 4 * h);
     const float erv = x4.x, lsev = x4.y, cvv = x4.z;
     float dr = 0.f;
+    int nxt = (lane < end - beg) ? __ldcs(a.nbr + beg + lane) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += 32) {
         const int n = min(32, end - base);
-        const int my = (lane < n) ? __ldcs(a.nbr + base + lane) : 0;
+        const int my = nxt;
+        nxt = (lane < end - base - 32) ? __ldcs(a.nbr + base + 32 + lane) : 0;
         for (int i0 = 0; i0 < H; i0 += UB) {
             if (i0 * S >= n) break;
             float t[UB][F], elu[UB];
@@ -671,9 +683,11 @@ __global__ void __launch_bounds__(256) k_gat_fwd_h1(const GatFwdArgs a) {
     for (int i = 0; i < NV; ++i) acc[i] = 0.f;
 #pragma unroll
     for (int i = 0; i < NP; ++i) pacc[i] = 0.f;
+    int nxt = (gl < end - beg) ? __ldcs(a.nbr + beg + gl) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
+        const int my = nxt;
+        nxt = (gl < end - base - RL) ? __ldcs(a.nbr + base + RL + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
@@ -806,9 +820,11 @@ __global__ void __launch_bounds__(256) k_gat_bwd_h1(const GatBwdArgs a) {
     float acc[NV], dsum = 0.f;
 #pragma unroll
     for (int i = 0; i < NV; ++i) acc[i] = 0.f;
+    int nxt = (gl < end - beg) ? __ldcs(a.nbr + beg + gl) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
-        const int my = (gl < n) ? __ldcs(a.nbr + base + gl) : 0;
+        const int my = nxt;
+        nxt = (gl < end - base - RL) ? __ldcs(a.nbr + base + RL + gl) : 0;
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;

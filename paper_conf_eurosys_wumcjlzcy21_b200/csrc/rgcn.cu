@@ -97,15 +97,23 @@ __global__ void __launch_bounds__(512) k_rgcn_rows(const RgcnRowArgs a) {
                 }
             }
         };
+        // edge-record prefetch: the next chunk's (u, type, norm) loads are in flight during this chunk
+        int nx_u = 0, nx_t = 0;
+        float nx_w = 0.f;
+        auto fetch = [&](int b) {
+            nx_u = 0; nx_t = 0; nx_w = 0.f;
+            if (gl < end - b) {
+                nx_u = __ldcs(a.nbr + b + gl);
+                nx_t = __ldcs(a.typ + b + gl);
+                nx_w = a.norm_user ? __ldg(a.norm_user + __ldg(a.eid + b + gl)) : __ldg(a.norm + b + gl);
+            }
+        };
+        fetch(beg);
         for (int base = beg; base < end; base += RL) {
             const int n = min(RL, end - base);
-            int my_u = 0, my_t = 0;
-            float my_w = 0.f;
-            if (gl < n) {
-                my_u = __ldcs(a.nbr + base + gl);
-                my_t = __ldcs(a.typ + base + gl);
-                my_w = a.norm_user ? __ldg(a.norm_user + __ldg(a.eid + base + gl)) : __ldg(a.norm + base + gl);
-            }
+            const int my_u = nx_u, my_t = nx_t;
+            const float my_w = nx_w;
+            fetch(base + RL);
 #pragma unroll
             for (int j0 = 0; j0 < L; j0 += UB) {
                 if (j0 * S >= n) break;
