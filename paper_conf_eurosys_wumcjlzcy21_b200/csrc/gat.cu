@@ -24,6 +24,13 @@
 
 #include "common.cuh"
 
+#ifndef GAT_MB_FWD
+#define GAT_MB_FWD 3   // min resident 256-thread blocks per SM (<= 85 regs): measured best on Reddit
+#endif
+#ifndef GAT_MB_BWD
+#define GAT_MB_BWD 3
+#endif
+
 namespace seastar {
 
 __device__ __forceinline__ float lrelu(float x, float slope) { return x > 0.f ? x : slope * x; }
@@ -174,7 +181,7 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
 // which the epilogue writes B_v = sum_e a_e LReLU'(s_e) T_u and b_v = sum_e a_e LReLU'(s_e) -- the two
 // forward-only factors of der_v = <dA_v, B_v> - c_v b_v (so the backward needs no dst-major pass).
 template <int F4, bool SB>
-__global__ void __launch_bounds__(256) k_gat_fwd_hpl(const GatFwdArgs a) {
+__global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_hpl(const GatFwdArgs a) {
     constexpr int F = 4 * F4;
     constexpr int UB = F4 <= 2 ? 4 : (F4 <= 4 ? 2 : 1);
     const int H = a.H;
@@ -496,7 +503,7 @@ __global__ void __launch_bounds__(256) k_gat_der(const GatBwdArgs a) {
 
 // head-per-lane source-major backward (REV CSR)
 template <int F4>
-__global__ void __launch_bounds__(256) k_gat_bwd_hpl(const GatBwdArgs a) {
+__global__ void __launch_bounds__(256, GAT_MB_BWD) k_gat_bwd_hpl(const GatBwdArgs a) {
     constexpr int F = 4 * F4;
     constexpr int UB = F4 <= 2 ? 4 : (F4 <= 4 ? 2 : 1);
     const int H = a.H, S = 32 / H;
@@ -664,7 +671,7 @@ __device__ __forceinline__ void load_chunks(const float* p, int col0, int W, flo
 }
 
 template <int VPL, int L, int RL, bool SB>
-__global__ void __launch_bounds__(256) k_gat_fwd_h1(const GatFwdArgs a) {
+__global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs a) {
     constexpr int NV = 4 * VPL, S = RL / L, UB = VPL <= 2 ? 4 : 2;
     constexpr int NP = SB ? NV : 1;
     const int lane = threadIdx.x & 31;
@@ -788,7 +795,7 @@ __global__ void __launch_bounds__(256) k_gat_fwd_h1(const GatFwdArgs a) {
 
 // DER = false: source-major dT/del over REV; DER = true: destination-major der over FWD
 template <int VPL, int L, int RL, bool DER>
-__global__ void __launch_bounds__(256) k_gat_bwd_h1(const GatBwdArgs a) {
+__global__ void __launch_bounds__(256, GAT_MB_BWD) k_gat_bwd_h1(const GatBwdArgs a) {
     constexpr int NV = 4 * VPL, S = RL / L, UB = VPL <= 2 ? 4 : 2;
     const int lane = threadIdx.x & 31;
     const int gl = lane % RL, slot = gl / L, c = gl % L;
