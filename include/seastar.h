@@ -226,7 +226,8 @@ seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float*
 int64_t seastar_gat_record_ld(int32_t H, int32_t F);
 /*
  * Backward row pass over owned rows: dA = dY * act'(Y);  c[v,h] = <dA[v,h,:], A[v,h,:]>;
- * D_loc[v] = [ dA (H*F, padded to a multiple of 4) | per head (er, lse, c, 0) ]
+ * D_loc[v] = [ dA (H*F, zero-padded to a multiple of 4) | per head (er, lse, c, nl2) ],
+ * nl2 = -lse * log2(e) (the backward kernels form a_e = 2^(LeakyReLU(s_e) log2(e) + nl2))
  * (ld = seastar_gat_record_ld(H,F); every field is 16-byte aligned when D_loc is).
  * If B_loc, b_loc (saved by seastar_gat_fwd) and der_loc [n_loc,H] are given, also
  *   der_loc[v,h] = <dA[v,h,:], B[v,h,:]> - c[v,h] b[v,h]    (replaces seastar_gat_der).
