@@ -86,23 +86,29 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
                  : "memory");
 }
 
+#ifndef TC_TWO_CTAS
+#define TC_TWO_CTAS 1
+#endif
 template <int NP>
 struct TcCfg {
     static constexpr int BM = 128, BK = 32;
-    static constexpr int STAGES = NP <= 64 ? 4 : (NP <= 128 ? 3 : 2);
+    // NP <= 64: two co-resident CTAs per SM (2 stages each), so one CTA's prologue / epilogue overlaps
+    // the other's TMA stream; wider tiles: one CTA with a deeper ring
+    static constexpr int CTAS = (TC_TWO_CTAS && NP <= 64) ? 2 : 1;
+    static constexpr int STAGES = CTAS == 2 ? 2 : (NP <= 64 ? 4 : (NP <= 128 ? 3 : 2));
     static constexpr uint32_t A_BYTES = BM * BK * 4;          // 16 KB
     static constexpr uint32_t B_BYTES = NP * BK * 4;          // NP rows of 128 B
     static constexpr uint32_t STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
     // G independent accumulators, K-chunk kc -> accumulator kc % G: each accumulates ~nk/G chunks, which
     // bounds the error of the tensor core's accumulation; the epilogue sums them in fp32 registers
-    static constexpr int G = NP <= 64 ? 8 : (NP <= 128 ? 4 : 2);
+    static constexpr int G = (NP <= 32 || (NP <= 64 && CTAS == 1)) ? 8 : (NP <= 128 ? 4 : 2);
     static constexpr uint32_t TMEM_COLS = (G * NP) <= 32 ? 32 : ((G * NP) <= 64 ? 64 : ((G * NP) <= 128 ? 128 :
                                           ((G * NP) <= 256 ? 256 : 512)));
     static constexpr size_t SMEM = (size_t)STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 };
 
 template <int NP>
-__global__ void __launch_bounds__(192, 1) k_gemm_tc(const __grid_constant__ CUtensorMap tmX, const TcArgs a) {
+__global__ void __launch_bounds__(192, TcCfg<NP>::CTAS) k_gemm_tc(const __grid_constant__ CUtensorMap tmX, const TcArgs a) {
     using C = TcCfg<NP>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -340,6 +346,272 @@ seastar_status linear_fwd_tc(const float* X, int64_t M, int64_t K, int64_t ldx, 
         case 128: return launch_tc_np<128>(tm, a, s);
         default: return SEASTAR_ERR_UNSUPPORTED;
     }
+}
+
+
+// ================================================================================================
+// dW = X^T dY on tcgen05 (3xTF32), both operands MN-major straight from TMA -- no transpose pass.
+//   D[k, n] (128 x NP32 per CTA) = sum_m X[m, k] dY[m, n] over the CTA's row split.
+// A = X^T (M' = k, K' = m): a TMA box of 32 k-columns x 32 m-rows (SWIZZLE_128B_ATOM_32B) lands as
+// the canonical MN-major tf32 layout (128 B rows, 32 B chunks swizzled within 4-row groups); the 4
+// column blocks of the 128-wide k tile sit LBO = 4 KB apart.  B = dY^T likewise (NP32 / 32 column blocks; columns >= N
+// are zero-filled by TMA).  Each 8-row K step advances both descriptors by 1024 B.
+// Row splits are multiples of 32 rows, so every 32-row chunk belongs to exactly one split; the
+// per-split partials [nsplit][K][N] are summed in split order afterwards (deterministic).
+// ================================================================================================
+struct TcTnArgs {
+    int64_t M, K, N;
+    int64_t rows_per_split;
+    float* part;                     // [nsplit][K][N]
+};
+
+template <int NP32>
+struct TcTnCfg {
+    static constexpr int BM = 128, BR = 32;                   // k tile, rows per stage
+    static constexpr int CTAS = 2, STAGES = 2;
+    static constexpr uint32_t A_BYTES = BM * BR * 4;           // 16 KB
+    static constexpr uint32_t B_BYTES = NP32 * BR * 4;         // 4 KB per 32 columns
+    static constexpr uint32_t STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
+    static constexpr int G = NP32 <= 32 ? 8 : 4;               // interleaved accumulators (<= 256 cols)
+    static constexpr uint32_t TMEM_COLS = G * NP32 <= 128 ? 128 : 256;
+    static constexpr size_t SMEM = (size_t)STAGES * STAGE_BYTES + 1024 + 256;
+};
+
+// MN-major tf32 operand: the only UMMA layout for it is SWIZZLE_128B_BASE32B (layout type 1): 128 B
+// rows along MN (32 elements) whose 32 B chunks are XOR-permuted by (row & 3) -- what TMA writes with
+// CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B.  LBO = bytes between 32-element MN blocks, SBO = bytes between
+// 4-row K groups (512 for densely stacked rows).
+__device__ __forceinline__ uint64_t smem_desc_mn32b(const void* p, uint32_t lbo) {
+    const uint32_t a = smem_u32(p);
+    uint64_t d = (uint64_t)((a >> 4) & 0x3FFF);
+    d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
+    d |= (uint64_t)(512 >> 4) << 32;
+    d |= (uint64_t)1 << 46;
+    d |= (uint64_t)1 << 61;
+    return d;
+}
+
+template <int NP32>
+__global__ void __launch_bounds__(192, TcTnCfg<NP32>::CTAS)
+    k_gemm_tc_tn(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmY, const TcTnArgs a) {
+    using C = TcTnCfg<NP32>;
+    constexpr int NB = NP32 / 32;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + (size_t)C::STAGES * C::STAGE_BYTES);
+    uint64_t* full = bars;
+    uint64_t* split = bars + C::STAGES;
+    uint64_t* empty = bars + 2 * C::STAGES;
+    uint64_t* accum = bars + 3 * C::STAGES;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * C::STAGES + 1);
+    auto A_hi = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES; };
+    auto A_lo = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + C::A_BYTES; };
+    auto B_hi = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + 2 * C::A_BYTES; };
+    auto B_lo = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + 2 * C::A_BYTES + C::B_BYTES; };
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int k0 = blockIdx.x * C::BM;
+    const int64_t r0 = (int64_t)blockIdx.y * a.rows_per_split;
+    const int64_t r1 = min(a.M, r0 + a.rows_per_split);
+    const int nch = (int)((r1 - r0 + C::BR - 1) / C::BR);
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < C::STAGES; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&split[s], 128);
+            mbar_init(&empty[s], 1);
+        }
+        mbar_init(accum, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(C::TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0 && nch > 0) {
+            for (int c = 0; c < nch; ++c) {
+                const int s = c % C::STAGES;
+                if (c >= C::STAGES) mbar_wait(&empty[s], ((c / C::STAGES) - 1) & 1);
+                mbar_expect_tx(&full[s], C::A_BYTES + C::B_BYTES);
+                const int m = (int)(r0 + (int64_t)c * C::BR);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) tma_load_2d(A_hi(s) + j * 4096, &tmX, k0 + 32 * j, m, &full[s]);
+#pragma unroll
+                for (int j = 0; j < NB; ++j) tma_load_2d(B_hi(s) + j * 4096, &tmY, 32 * j, m, &full[s]);
+            }
+        }
+    } else if (warp == 1) {
+        // D f32, A/B tf32, both MN-major (bits 15, 16), N = NP32, M = 128
+        const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 15) | (1u << 16) |
+                               ((uint32_t)(NP32 >> 3) << 17) | ((128u >> 4) << 24);
+        for (int c = 0; c < nch; ++c) {
+            const int s = c % C::STAGES;
+            mbar_wait(&split[s], (c / C::STAGES) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            if (lane == 0) {
+                const uint32_t d = tmem + (uint32_t)((c % C::G) * NP32);
+#pragma unroll
+                for (int ks = 0; ks < C::BR / 8; ++ks) {
+                    const uint64_t ah = smem_desc_mn32b(A_hi(s) + ks * 1024, 4096);
+                    const uint64_t al = smem_desc_mn32b(A_lo(s) + ks * 1024, 4096);
+                    const uint64_t bh = smem_desc_mn32b(B_hi(s) + ks * 1024, 4096);
+                    const uint64_t bl = smem_desc_mn32b(B_lo(s) + ks * 1024, 4096);
+                    mma_tf32(d, al, bh, idesc, (c >= C::G || ks > 0) ? 1u : 0u);
+                    mma_tf32(d, ah, bl, idesc, 1u);
+                    mma_tf32(d, ah, bh, idesc, 1u);
+                }
+                mma_commit(&empty[s]);
+                if (c == nch - 1) mma_commit(accum);
+            }
+            __syncwarp();
+        }
+    } else {
+        const int t = threadIdx.x - 64;
+        for (int c = 0; c < nch; ++c) {
+            const int s = c % C::STAGES;
+            mbar_wait(&full[s], (c / C::STAGES) & 1);
+            // elementwise hi / lo split in place (layout preserving, conflict-free 16 B chunks)
+            float4* ph = reinterpret_cast<float4*>(A_hi(s));
+            float4* pl = reinterpret_cast<float4*>(A_lo(s));
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const float4 x = ph[q * 128 + t];
+                const float4 h = make_float4(rna_tf32(x.x), rna_tf32(x.y), rna_tf32(x.z), rna_tf32(x.w));
+                ph[q * 128 + t] = h;
+                pl[q * 128 + t] = make_float4(x.x - h.x, x.y - h.y, x.z - h.z, x.w - h.w);
+            }
+            float4* qh = reinterpret_cast<float4*>(B_hi(s));
+            float4* ql = reinterpret_cast<float4*>(B_lo(s));
+#pragma unroll
+            for (int q = 0; q < NB * 2; ++q) {
+                const float4 x = qh[q * 128 + t];
+                const float4 h = make_float4(rna_tf32(x.x), rna_tf32(x.y), rna_tf32(x.z), rna_tf32(x.w));
+                qh[q * 128 + t] = h;
+                ql[q * 128 + t] = make_float4(x.x - h.x, x.y - h.y, x.z - h.z, x.w - h.w);
+            }
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive(&split[s]);
+        }
+        // epilogue: partial[split][k0 + r][n] = sum_g acc_g[r][n]
+        const int q4 = warp & 3;
+        const int r = q4 * 32 + lane;
+        const int64_t gk = k0 + r;
+        float* prow = a.part + ((int64_t)blockIdx.y * a.K + gk) * a.N;
+        if (nch > 0) {
+            mbar_wait(accum, 0);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        }
+        const int nacc = nch < C::G ? nch : C::G;
+#pragma unroll 1
+        for (int c0 = 0; c0 < NP32; c0 += 16) {
+            float accv[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) accv[j] = 0.f;
+            for (int g = 0; g < nacc; ++g) {
+                uint32_t v[16];
+                asm volatile(
+                    "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
+                    "[%16];"
+                    : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                      "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+                      "=r"(v[15])
+                    : "r"(tmem + ((uint32_t)(q4 * 32) << 16) + (uint32_t)(g * NP32 + c0)));
+                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+                for (int j = 0; j < 16; ++j) accv[j] += __uint_as_float(v[j]);
+            }
+            if (gk < a.K) {
+#pragma unroll
+                for (int j = 0; j < 16; ++j)
+                    if (c0 + j < a.N) prow[c0 + j] = accv[j];
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 1) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C::TMEM_COLS));
+    }
+}
+
+// row splits (multiples of 32 rows) so that ktiles x nsplit fills ~4 waves of 2 CTAs per SM
+static void tc_tn_geometry(int64_t M, int64_t K, int64_t& ktiles, int64_t& nsplit, int64_t& rows_per_split) {
+    ktiles = (K + 127) / 128;
+    int64_t want = (8 * num_sms() + ktiles - 1) / ktiles;
+    int64_t max_split = (M + 255) / 256;
+    nsplit = want < max_split ? want : max_split;
+    if (nsplit < 1) nsplit = 1;
+    rows_per_split = (M + nsplit - 1) / nsplit;
+    rows_per_split = (rows_per_split + 31) / 32 * 32;
+    nsplit = (M + rows_per_split - 1) / rows_per_split;
+    if (nsplit < 1) nsplit = 1;
+}
+
+size_t linear_bwd_weight_tc_part_bytes(int64_t M, int64_t K, int64_t N) {
+    int64_t kt, ns, rps;
+    tc_tn_geometry(M > 0 ? M : 1, K, kt, ns, rps);
+    return (size_t)ns * K * N * sizeof(float);
+}
+
+template <int NP32>
+static seastar_status launch_tc_tn(const CUtensorMap& tx, const CUtensorMap& ty, const TcTnArgs& a, dim3 grid,
+                                   cudaStream_t s) {
+    using C = TcTnCfg<NP32>;
+    static bool attr = false;
+    if (!attr) {
+        SS_CUDA(cudaFuncSetAttribute(k_gemm_tc_tn<NP32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
+        attr = true;
+    }
+    k_gemm_tc_tn<NP32><<<grid, 192, C::SMEM, s>>>(tx, ty, a);
+    return check_launch("k_gemm_tc_tn");
+}
+
+// writes the per-split partials into part (linear_bwd_weight_tc_part_bytes) and returns the split
+// count in *nsplit_out; SEASTAR_ERR_UNSUPPORTED (nothing launched) when the path does not apply
+seastar_status linear_bwd_weight_tc(const float* X, int64_t M, int64_t K, int64_t ldx, const float* dY, int64_t N,
+                                    int64_t ldy, float* part, int64_t* nsplit_out, cudaStream_t s) {
+    if (getenv("SEASTAR_NO_TCGEN05") || M < 256 || K < 32 || N > 64 || (ldx % 4) != 0 || (ldy % 4) != 0 ||
+        !aligned16(X) || !aligned16(dY) || M >= (1LL << 31) || K >= (1LL << 31))
+        return SEASTAR_ERR_UNSUPPORTED;
+    auto enc = encode_fn();
+    if (!enc) return SEASTAR_ERR_UNSUPPORTED;
+    CUtensorMap tx, ty;
+    {
+        cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)M};
+        cuuint64_t strides[1] = {(cuuint64_t)ldx * sizeof(float)};
+        cuuint32_t box[2] = {32, 32};
+        cuuint32_t estr[2] = {1, 1};
+        if (enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(X), dims, strides, box, estr,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            return SEASTAR_ERR_UNSUPPORTED;
+    }
+    {
+        cuuint64_t dims[2] = {(cuuint64_t)N, (cuuint64_t)M};
+        cuuint64_t strides[1] = {(cuuint64_t)ldy * sizeof(float)};
+        cuuint32_t box[2] = {32, 32};
+        cuuint32_t estr[2] = {1, 1};
+        if (enc(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(dY), dims, strides, box, estr,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            return SEASTAR_ERR_UNSUPPORTED;
+    }
+    int64_t kt, ns, rps;
+    tc_tn_geometry(M, K, kt, ns, rps);
+    TcTnArgs a{M, K, N, rps, part};
+    *nsplit_out = ns;
+    const dim3 grid((unsigned)kt, (unsigned)ns);
+    return N <= 32 ? launch_tc_tn<32>(tx, ty, a, grid, s) : launch_tc_tn<64>(tx, ty, a, grid, s);
 }
 
 }  // namespace seastar

@@ -218,6 +218,9 @@ seastar_status linear_fwd_tc(const float* X, int64_t M, int64_t K, int64_t ldx, 
                              void* ws, size_t ws_bytes, cudaStream_t s);
 size_t linear_fwd_tc_workspace(int64_t K, int64_t N);
 size_t colsum_ws(int64_t M, int64_t F);
+size_t linear_bwd_weight_tc_part_bytes(int64_t M, int64_t K, int64_t N);
+seastar_status linear_bwd_weight_tc(const float* X, int64_t M, int64_t K, int64_t ldx, const float* dY, int64_t N,
+                                    int64_t ldy, float* part, int64_t* nsplit_out, cudaStream_t s);
 
 }  // namespace seastar
 
@@ -258,7 +261,10 @@ seastar_status seastar_linear_bwd_data(const float* dY, int64_t M, int64_t Nout,
 size_t seastar_linear_bwd_weight_workspace(int64_t M, int64_t K, int64_t Nout) {
     int64_t kt, ns, rps;
     tn_geometry(M > 0 ? M : 1, K, kt, ns, rps);
-    return (size_t)ns * K * Nout * sizeof(float) + colsum_ws(M, Nout) + 512;
+    size_t part = (size_t)ns * K * Nout * sizeof(float);
+    const size_t tc = linear_bwd_weight_tc_part_bytes(M, K, Nout);
+    if (tc > part) part = tc;
+    return part + colsum_ws(M, Nout) + 512;
 }
 
 seastar_status seastar_linear_bwd_weight(const float* X, int64_t M, int64_t K, int64_t ldx, const float* dY,
@@ -271,18 +277,24 @@ seastar_status seastar_linear_bwd_weight(const float* X, int64_t M, int64_t K, i
     SS_TRY(check_device());
     cudaStream_t s = to_stream(stream);
     int64_t kt, ns, rps;
-    tn_geometry(M, K, kt, ns, rps);
     float* part = static_cast<float*>(workspace);
-    dim3 grid((unsigned)kt, (unsigned)ns);
-    if (Nout <= 16) k_gemm_tn<16><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
-    else if (Nout <= 32) k_gemm_tn<32><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
-    else k_gemm_tn<64><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
-    SS_TRY(check_launch("k_gemm_tn"));
+    // tcgen05 3xTF32 path (MN-major TMA operands); SIMT fp32 otherwise
+    const seastar_status st = linear_bwd_weight_tc(X, M, K, ldx, dY, Nout, ldy, part, &ns, s);
+    if (st == SEASTAR_ERR_UNSUPPORTED) {
+        tn_geometry(M, K, kt, ns, rps);
+        dim3 grid((unsigned)kt, (unsigned)ns);
+        if (Nout <= 16) k_gemm_tn<16><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
+        else if (Nout <= 32) k_gemm_tn<32><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
+        else k_gemm_tn<64><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
+        SS_TRY(check_launch("k_gemm_tn"));
+    } else if (st != SEASTAR_OK) {
+        return st;
+    }
     const int64_t n = K * Nout;
     k_sum_splits<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(part, ns, n, dW);
     SS_TRY(check_launch("k_sum_splits"));
     if (db) {
-        size_t off = ((size_t)ns * K * Nout * sizeof(float) + 255) & ~size_t(255);
+        size_t off = ((seastar_linear_bwd_weight_workspace(M, K, Nout) - colsum_ws(M, Nout) - 512) + 255) & ~size_t(255);
         SS_TRY(colsum_impl(dY, M, Nout, ldy, db, static_cast<char*>(workspace) + off, ws_bytes - off, s));
     }
     return SEASTAR_OK;

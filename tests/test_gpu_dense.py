@@ -133,3 +133,31 @@ def test_colsum_axpby_adam(env):
         L.seastar_adam(pd, dev(env, g), md, vd, n, 0.01, 0.9, 0.999, 1e-8, step)
         oracle.adam(pr, g, mr, vr, 0.01, t)
     assert rel_err(pd.cpu().numpy() - p, pr - p) <= 1e-4   # update magnitude ~lr; compare the deltas
+
+
+TC_TN_SHAPES = [(256, 32, 1), (1000, 602, 16), (5003, 602, 64), (3001, 64, 41), (300, 8710, 8), (4099, 100, 33),
+                (20000, 128, 32), (233, 602, 16)]
+
+
+@pytest.mark.parametrize("M,K,N", TC_TN_SHAPES)
+def test_linear_bwd_weight_tcgen05(env, M, K, N):
+    """ldx % 4 == ldy % 4 == 0 (16-B aligned rows) -> the tcgen05 MN-major 3xTF32 dW kernel (M >= 256)."""
+    torch, L = env["torch"], env["L"]
+    X, dY = rnd(51, (M, K)), rnd(52, (M, N))
+    ldx = (K + 3) // 4 * 4 + 4
+    ldy = (N + 3) // 4 * 4
+    ws_b = L.seastar_linear_bwd_weight_workspace(M, K, N)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    dW = torch.full((K, N), float("nan"), device="cuda")
+    db = torch.empty((N,), device="cuda")
+    L.seastar_linear_bwd_weight(dev(env, padded(X, ldx)), M, K, ldx, dev(env, padded(dY, ldy)), N, ldy, dW, db, ws,
+                                ws_b)
+    _, rdW, rdb = oracle.linear_bwd(X, np.zeros((K, N), np.float32), dY)
+    assert rel_err(dW.cpu().numpy(), rdW) <= TOL
+    assert rel_err(db.cpu().numpy(), rdb) <= TOL
+    # large-magnitude rows: the hi/lo split keeps fp32 accuracy
+    X2 = (X.astype(np.float64) * 1e3 + 0.123456789).astype(np.float32)
+    L.seastar_linear_bwd_weight(dev(env, padded(X2, ldx)), M, K, ldx, dev(env, padded(dY, ldy)), N, ldy, dW, db, ws,
+                                ws_b)
+    _, rdW2, _ = oracle.linear_bwd(X2, np.zeros((K, N), np.float32), dY)
+    assert rel_err(dW.cpu().numpy(), rdW2) <= TOL
