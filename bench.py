@@ -30,7 +30,6 @@ sys.path.insert(0, ROOT)
 
 import synth  # noqa: E402
 
-CFG = synth.CONFIGS["reddit"]
 
 
 def parse():
@@ -43,6 +42,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-edges", type=int, default=10_000_000)
+    ap.add_argument("--workload", default="reddit", choices=list(synth.CONFIGS),
+                    help="BASELINE config to train (default: configs[4], the Reddit-shaped GCN+GAT headline)")
     return ap.parse_args()
 
 
@@ -50,23 +51,8 @@ def parse():
 # inputs (seeded, synthetic, Reddit-shaped)
 # ------------------------------------------------------------------------------------------
 def make_inputs():
-    ip, ix = synth.make_graph(CFG)
-    X = synth.uniform(CFG.feat_seed, (CFG.N, CFG.F_in), -1.0, 1.0)
-    lab = synth.labels(CFG.label_seed, CFG.N, CFG.classes)
-    H, C = CFG.hidden, CFG.classes
-    gcn_p = {"W1": synth.glorot(CFG.weight_seed(1), CFG.F_in, H), "b1": np.zeros(H, np.float32),
-             "W2": synth.glorot(CFG.weight_seed(2), H, C), "b2": np.zeros(C, np.float32)}
-    heads, hid = CFG.heads, CFG.extra["gat_hidden"]
-    Wd = heads * hid
-    gat_p = {"W1": synth.glorot(CFG.weight_seed(11), CFG.F_in, Wd),
-             "al1": synth.glorot(CFG.weight_seed(12), hid, 1, (heads, hid)),
-             "ar1": synth.glorot(CFG.weight_seed(13), hid, 1, (heads, hid)),
-             "b1": np.zeros(Wd, np.float32),
-             "W2": synth.glorot(CFG.weight_seed(14), Wd, C),
-             "al2": synth.glorot(CFG.weight_seed(15), C, 1, (1, C)),
-             "ar2": synth.glorot(CFG.weight_seed(16), C, 1, (1, C)),
-             "b2": np.zeros(C, np.float32)}
-    return ip, ix, X, lab, gcn_p, gat_p
+    w = synth.workload("reddit")
+    return w["indptr"], w["indices"], w["X"], w["labels"], w["gcn"], w["gat"]
 
 
 # ------------------------------------------------------------------------------------------
@@ -88,6 +74,11 @@ def bytes_gat_bwd(E, n, H, F):
     W = H * F
     ldd = (W + 3) // 4 * 4 + 4 * H
     return E * (4 + 4 * ldd) + n * (8 + 4 * W + 4 * H + 4 * W + 4 * H)
+
+
+def bytes_rgcn_fwd(E, n, Fin, Fout):
+    # per edge 4B src + 4B type + 4B norm + the gathered input row; per row off+perm 8B, output row
+    return E * (12 + 4 * Fin) + n * (8 + 4 * Fout)
 
 
 def bytes_gat_der(E, n, H, F):
@@ -186,6 +177,28 @@ def oracle_sample(ip, ix, X, sample_edges, seed=0):
     return edges, dt, desc
 
 
+def oracle_step(w, names):
+    """One whole oracle training step (forward + backward, fp64 edge loops) of the config's model(s) on
+    the whole graph -- configs[0..3] are small enough to run in full."""
+    from oracle import model_ref
+    cfg = w["cfg"]
+    ip, ix, X, lab = w["indptr"], w["indices"], w["X"], w["labels"]
+    f64 = lambda p: {k: np.asarray(v, np.float64) for k, v in p.items()}
+    t0 = time.perf_counter()
+    for k in names:
+        if k == "gcn":
+            model_ref.gcn2(ip, ix, X, lab, f64(w["gcn"]))
+        elif k == "gat":
+            model_ref.gat2(ip, ix, X, lab, f64(w["gat"]), cfg.heads, cfg.extra.get("gat_hidden", cfg.hidden))
+        elif k == "appnp":
+            model_ref.appnp(ip, ix, X, lab, f64(w["appnp"]), cfg.K, cfg.alpha)
+        elif k == "rgcn":
+            model_ref.rgcn2(ip, ix, w["etypes"], X, lab, f64(w["rgcn"]))
+    dt = time.perf_counter() - t0
+    return cfg.E * len(names), dt, (f"one whole oracle training step (forward + backward, fp64) of {'+'.join(names)} "
+                                    f"on the full {cfg.name} graph ({cfg.E} edges); edges/s = E per model / wall time")
+
+
 def omp_threads():
     try:
         return int(os.environ.get("OMP_NUM_THREADS", "")) or os.cpu_count()
@@ -194,16 +207,24 @@ def omp_threads():
 
 
 def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle, as written, on the box's host cores (rank 0 only), on the same
+    workload, metric and unit as the GPU arm; each step is a bounded sample of that workload (Reddit:
+    the first vertex ids covering ~cpu_sample_edges/4 in-edges; configs[0..3]: one whole step)."""
     if rank != 0:
         return
-    ip, ix = synth.make_graph(CFG)
-    X = synth.uniform(CFG.feat_seed, (CFG.N, CFG.F_in), -1.0, 1.0)
-    sample = max(200_000, args.cpu_sample_edges // 4)
+    w = synth.workload(args.workload)
+    cfg = w["cfg"]
+    names = [k for k in ("gcn", "gat", "appnp", "rgcn") if k in w]
+
+    def one():
+        if args.workload == "reddit":
+            return oracle_sample(w["indptr"], w["indices"], w["X"], max(200_000, args.cpu_sample_edges // 4))
+        return oracle_step(w, names)
     for _ in range(args.warmup):
-        oracle_sample(ip, ix, X, sample)
+        one()
     tot_e, tot_t, desc = 0, 0.0, ""
     for _ in range(args.steps):
-        e, t, desc = oracle_sample(ip, ix, X, sample)
+        e, t, desc = one()
         tot_e += e
         tot_t += t
     v = tot_e / tot_t
@@ -211,13 +232,61 @@ def run_reference(args, rank, world):
             "value": v, "unit": "edges/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1000 * tot_t / args.steps, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": "reddit-shaped GCN+GAT (oracle sample)", "N": CFG.N, "E": CFG.E},
+            "config": {"workload": WORKLOAD_DESC[args.workload], "name": args.workload, "N": cfg.N, "E": cfg.E},
             "cpu_baseline": {"value": v, "unit": "edges/s", "cores": omp_threads(), "kind": "oracle", "sample": desc},
             "e2e": {"value": v, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 # ------------------------------------------------------------------------------------------
+# workloads: which models one step trains, and the per-kernel algorithmic bytes
+# ------------------------------------------------------------------------------------------
+WORKLOAD_DESC = {
+    "reddit": "reddit-shaped full-graph training: 2-layer GCN (602-16-41) + 2-layer GAT (602-8x8-1x41), one epoch "
+              "each per step",
+    "cora_gcn": "cora-shaped 2-layer GCN (1433-16-7), one training epoch per step",
+    "corafull_gat": "corafull-shaped 2-layer GAT (8710-8x8-1x70), one training epoch per step",
+    "physics_appnp": "coauthor-physics-shaped APPNP (MLP 8415-64-5, K=10, alpha=0.1), one training epoch per step",
+    "am_rgcn": "am-shaped 2-layer R-GCN (16-16-11, 133 relations, 1/c_{v,r}), one training epoch per step",
+}
+
+
+def build_models(name, w, g, X_loc, lab_loc, comm, rows_all, which):
+    from paper_conf_eurosys_wumcjlzcy21_b200.models import GAT2, GCN2, APPNPNet, RGCN2
+    cfg = w["cfg"]
+    models = {}
+    if "gcn" in w and which in ("both", "gcn"):
+        models["gcn"] = GCN2(g, X_loc, lab_loc, w["gcn"], comm=comm, n_pad_rows=rows_all)
+    if "gat" in w and which in ("both", "gat"):
+        models["gat"] = GAT2(g, X_loc, lab_loc, w["gat"], cfg.heads, cfg.extra.get("gat_hidden", cfg.hidden),
+                             comm=comm, n_pad_rows=rows_all)
+    if "appnp" in w:
+        models["appnp"] = APPNPNet(g, X_loc, lab_loc, w["appnp"], K=cfg.K, alpha=cfg.alpha, comm=comm,
+                                   n_pad_rows=rows_all)
+    if "rgcn" in w:
+        models["rgcn"] = RGCN2(g, X_loc, lab_loc, w["rgcn"], comm=comm, n_pad_rows=rows_all)
+    return models
+
+
+def kernel_bytes(cfg, g):
+    info = g.info
+    E_f, E_r, n = info["num_fwd_edges"], info["num_rev_edges"], g.n_loc
+    H, C = cfg.hidden, cfg.classes
+    if cfg.model == "appnp":
+        return {"appnp_fwd": bytes_gcn_agg(E_f, n, C, 2, 1), "appnp_bwd": bytes_gcn_agg(E_r, n, C, 2, 0)}
+    if cfg.model == "rgcn":
+        return {"rgcn_fwd1": bytes_rgcn_fwd(E_f, n, cfg.F_in, H)}
+    heads, hid = cfg.heads, cfg.extra.get("gat_hidden", cfg.hidden)
+    return {"gat_fwd1": bytes_gat_fwd(E_f, n, heads, hid), "gat_bwd1": bytes_gat_bwd(E_r, n, heads, hid),
+            "gat_fwd2": bytes_gat_fwd(E_f, n, 1, C), "gat_bwd2": bytes_gat_bwd(E_r, n, 1, C),
+            "gcn_fwd1": bytes_gcn_agg(E_f, n, H, 1, 0), "gcn_bwd2": bytes_gcn_agg(E_r, n, H, 1, 1),
+            "gat_der1": bytes_gat_der(E_f, n, heads, hid), "gat_der2": bytes_gat_der(E_f, n, 1, C)}
+
+
+# our kernels launched per training epoch (counted from the ncu launch list, profiles/r1/launches_*.csv)
+LAUNCHES_PER_EPOCH = {"gcn": 20, "gat": 31, "appnp": 47, "rgcn": 12}
+
+
 def main():
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -247,27 +316,27 @@ def main():
     from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
     from paper_conf_eurosys_wumcjlzcy21_b200.graph import Graph
     from paper_conf_eurosys_wumcjlzcy21_b200 import partition
-    from paper_conf_eurosys_wumcjlzcy21_b200.models import GAT2, GCN2, Comm
+    from paper_conf_eurosys_wumcjlzcy21_b200.models import Comm
     L.seastar_device_check()
 
     t_setup = time.perf_counter()
-    ip, ix, X, lab, gcn_p, gat_p = make_inputs()
-    N = CFG.N
+    w = synth.workload(args.workload)
+    cfg = w["cfg"]
+    ip, ix, X, lab = w["indptr"], w["indices"], w["X"], w["labels"]
+    N = cfg.N
     rb, re = partition.row_range(N, world, rank)
     rows_all = partition.gathered_rows(N, world)
-    g = Graph(ip, ix, row_begin=rb, row_end=re, device=dev)
+    if cfg.typed:
+        g = Graph(ip, ix, w["etypes"], num_etypes=cfg.R, rgcn_norm=True, row_begin=rb, row_end=re, device=dev)
+    else:
+        g = Graph(ip, ix, row_begin=rb, row_end=re, device=dev)
     # input rows padded to a 16-byte multiple so the dense transform can stream X with TMA
-    X_pad = torch.zeros((re - rb, (CFG.F_in + 3) // 4 * 4), device=dev)
-    X_loc = X_pad[:, :CFG.F_in]
+    X_pad = torch.zeros((re - rb, (cfg.F_in + 3) // 4 * 4), device=dev)
+    X_loc = X_pad[:, :cfg.F_in]
     X_loc.copy_(torch.from_numpy(X[rb:re]))
     lab_loc = torch.from_numpy(lab[rb:re]).to(dev)
     comm = Comm(world, rank)
-    models = {}
-    if args.model in ("both", "gcn"):
-        models["gcn"] = GCN2(g, X_loc, lab_loc, gcn_p, comm=comm, n_pad_rows=rows_all)
-    if args.model in ("both", "gat"):
-        models["gat"] = GAT2(g, X_loc, lab_loc, gat_p, CFG.heads, CFG.extra["gat_hidden"], comm=comm,
-                             n_pad_rows=rows_all)
+    models = build_models(args.workload, w, g, X_loc, lab_loc, comm, rows_all, args.model)
     torch.cuda.synchronize()
     setup_s = time.perf_counter() - t_setup
 
@@ -328,7 +397,7 @@ def main():
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         total_ms = t.item()
     ms_per_step = total_ms / args.steps
-    E = CFG.E
+    E = cfg.E
     edges_per_step = E * len(models)
     value = edges_per_step / (ms_per_step / 1e3)
 
@@ -341,31 +410,26 @@ def main():
         ts = [a.elapsed_time(b) for a, b in zip(evs, ends)]
         if ts:
             kernels[name] = statistics.mean(ts)
-    info = g.info
-    E_f, E_r, n = info["num_fwd_edges"], info["num_rev_edges"], g.n_loc
-    alg = {"gat_fwd1": bytes_gat_fwd(E_f, n, 8, 8), "gat_bwd1": bytes_gat_bwd(E_r, n, 8, 8),
-           "gat_fwd2": bytes_gat_fwd(E_f, n, 1, 41),
-           "gat_bwd2": bytes_gat_bwd(E_r, n, 1, 41), "gcn_fwd1": bytes_gcn_agg(E_f, n, 16, 1, 0),
-           "gcn_bwd2": bytes_gcn_agg(E_r, n, 16, 1, 1), "gat_der1": bytes_gat_der(E_f, n, 8, 8),
-           "gat_der2": bytes_gat_der(E_f, n, 1, 41)}
+    alg = kernel_bytes(cfg, g)
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
     except Exception:
         pass
     hbm = peaks.get("hbm_gbs", 6650.0)
-    dom = max(kernels, key=kernels.get) if kernels else None
+    known = {k: v for k, v in kernels.items() if k in alg}
+    dom = max(known, key=known.get) if known else None
     roofline = None
     if dom:
-        ach = alg.get(dom, 0) / (kernels[dom] / 1e3) / 1e9
+        ach = alg[dom] / (kernels[dom] / 1e3) / 1e9
         traffic = None
         try:
             tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-            traffic = tr.get(dom)
+            traffic = tr.get(f"{args.workload}:{dom}", tr.get(dom) if args.workload == "reddit" else None)
         except Exception:
             pass
         roofline = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": hbm, "unit": "GB/s",
-                    "frac": ach / hbm, "traffic": traffic, "algorithmic_bytes": alg.get(dom),
+                    "frac": ach / hbm, "traffic": traffic, "algorithmic_bytes": alg[dom],
                     "ms": kernels[dom], "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback"}
     kern_out = {k: {"ms": v, "GB/s": (alg[k] / (v / 1e3) / 1e9) if k in alg else None} for k, v in kernels.items()}
 
@@ -402,23 +466,23 @@ def main():
     # ---- CPU oracle baseline (rank 0, N = 1 only) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        e, t, desc = oracle_sample(ip, ix, X, args.cpu_sample_edges)
+        if args.workload == "reddit":
+            e, t, desc = oracle_sample(ip, ix, X, args.cpu_sample_edges)
+        else:
+            e, t, desc = oracle_step(w, list(models))
         cpu = {"value": e / t, "unit": "edges/s", "cores": omp_threads(), "kind": "oracle", "sample": desc,
                "seconds": t}
 
-    gpu_launches = None
     if rank == 0:
-        # kernels of ours per epoch, counted from the ncu launch list (profiles/r1/launches.txt)
-        per_epoch = {"gcn": 20, "gat": 31}
-        gpu_launches = args.steps * sum(per_epoch[k] for k in models)
+        gpu_launches = args.steps * sum(LAUNCHES_PER_EPOCH[k] for k in models)
         line = {
             "metric": "GAT/GCN train epoch ms and edges/s at 1/2/4/8 B200; achieved HBM GB/s",
             "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "f32", "data": "synthetic",
-            "config": {"workload": "reddit-shaped full-graph training: 2-layer GCN (602-16-41) + 2-layer GAT "
-                                   "(602-8x8-1x41), one epoch each per step",
-                       "N": CFG.N, "E": E, "F_in": CFG.F_in, "classes": CFG.classes,
+            "config": {"workload": WORKLOAD_DESC[args.workload] if args.model == "both" or args.workload != "reddit"
+                       else f"reddit-shaped full-graph training: {args.model} only",
+                       "name": args.workload, "N": cfg.N, "E": E, "F_in": cfg.F_in, "classes": cfg.classes,
                        "parallelism": f"row-partition x{world}", "l2": "flushed (256 MB write) between steps",
                        "epoch_ms": {k: statistics.mean(v) for k, v in model_ms.items()},
                        "edges_per_s": {k: E / (statistics.mean(v) / 1e3) for k, v in model_ms.items()},

@@ -164,8 +164,10 @@ seastar_status seastar_linear_bwd_data(const float* dY, int64_t M, int64_t Nout,
                                        int64_t K, const float* row_scale, const float* Yact, seastar_act act,
                                        float* dX, int64_t ldx, seastar_stream stream);
 /*
- * dW = X^T dY  ([K,Nout]) and, if db != NULL, db = sum_r dY[r,:].  Deterministic split-M
- * reduction through `workspace` (dev) of seastar_linear_bwd_weight_workspace() bytes.
+ * dW = X^T dY  ([K,Nout], any Nout >= 1, produced in column chunks of 64) and, if db != NULL,
+ * db = sum_r dY[r,:].  Deterministic split-M reduction through `workspace` (dev) of
+ * seastar_linear_bwd_weight_workspace() bytes; the split partials are summed in split order with an
+ * fp64 accumulator.
  */
 seastar_status seastar_linear_bwd_weight(const float* X, int64_t M, int64_t K, int64_t ldx, const float* dY,
                                          int64_t Nout, int64_t ldy, float* dW, float* db, void* workspace,

@@ -24,6 +24,9 @@ rgcn_norm/fwd/bwd          sum_r sum_{u in N_r(v)} 1/c_{v,r} h_u W_r           L
 softmax_xent, adam         DGL default training loop                             L481
 =========================  ===================================================  ==================
 
+``oracle/model_ref.py`` composes these functions into whole training steps of the four models (the
+reference the GPU models are compared with, and the CPU baseline ``bench.py`` times for configs[0..3]).
+
 Every pin of these functions (hand fixtures, closed forms, dense brute force, finite differences)
 is in ``tests/test_oracle_*.py``.
 """

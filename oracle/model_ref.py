@@ -5,10 +5,10 @@ readings of DESIGN.md §3; the GPU models in paper_conf_eurosys_wumcjlzcy21_b200
 them parameter by parameter."""
 import numpy as np
 
-import oracle
+import oracle  # noqa: F401  (package of the oracle functions composed here)
 
 
-def gcn2(ip, ix, X, lab, p):
+def gcn2(ip, ix, X, lab, p, acts=None):
     in_n, out_n = oracle.degree_norms(ip, ix)
     T = oracle.linear_fwd(X, p["W1"])
     Z1 = oracle.gcn_aggregate(ip, ix, T, out_n, in_n) + p["b1"]
@@ -22,6 +22,8 @@ def gcn2(ip, ix, X, lab, p):
     db1 = dZ1.sum(0)
     dT = oracle.gcn_aggregate_T(ip, ix, dZ1, out_n, in_n)
     _, dW1, _ = oracle.linear_bwd(X, p["W1"], dT, need_dX=False, need_db=False)
+    if acts is not None:
+        acts.update(H1=H1, logits=logits)
     return loss, {"W1": dW1, "b1": db1, "W2": dW2, "b2": db2}
 
 
@@ -45,7 +47,7 @@ def _gat_layer_bwd(ip, ix, Xin, W, al, ar, T, el, er, Z, act, dY, H, F, need_dX)
     return dX, dW, dal, dar, db
 
 
-def gat2(ip, ix, X, lab, p, heads, hidden):
+def gat2(ip, ix, X, lab, p, heads, hidden, acts=None):
     C = p["W2"].shape[1]
     T1, el1, er1, Z1, Y1 = _gat_layer_fwd(ip, ix, X, p["W1"], p["al1"], p["ar1"], p["b1"], "elu", heads, hidden)
     T2, el2, er2, Z2, Y2 = _gat_layer_fwd(ip, ix, Y1, p["W2"], p["al2"], p["ar2"], p["b2"], "none", 1, C)
@@ -54,10 +56,12 @@ def gat2(ip, ix, X, lab, p, heads, hidden):
                                                dY2, 1, C, True)
     _, dW1, dal1, dar1, db1 = _gat_layer_bwd(ip, ix, X, p["W1"], p["al1"], p["ar1"], T1, el1, er1, Z1, "elu", dY1,
                                              heads, hidden, False)
+    if acts is not None:
+        acts.update(Y1=Y1, Y2=Y2)
     return loss, {"W1": dW1, "al1": dal1, "ar1": dar1, "b1": db1, "W2": dW2, "al2": dal2, "ar2": dar2, "b2": db2}
 
 
-def appnp(ip, ix, X, lab, p, K, alpha):
+def appnp(ip, ix, X, lab, p, K, alpha, acts=None):
     Z1 = oracle.linear_fwd(X, p["W1"], p["b1"])
     Hh = oracle.act_fwd("relu", Z1)
     H0 = oracle.linear_fwd(Hh, p["W2"], p["b2"])
@@ -67,10 +71,12 @@ def appnp(ip, ix, X, lab, p, K, alpha):
     dHh, dW2, db2 = oracle.linear_bwd(Hh, p["W2"], dH0)
     dZ1 = oracle.act_bwd("relu", Z1, dHh)
     _, dW1, db1 = oracle.linear_bwd(X, p["W1"], dZ1, need_dX=False)
+    if acts is not None:
+        acts.update(Z=Z)
     return loss, {"W1": dW1, "b1": db1, "W2": dW2, "b2": db2}
 
 
-def rgcn2(ip, ix, et, X, lab, p):
+def rgcn2(ip, ix, et, X, lab, p, acts=None):
     Z1 = oracle.rgcn_fwd(ip, ix, et, X, p["W1"]) + p["b1"]
     H1 = oracle.act_fwd("relu", Z1)
     Z2 = oracle.rgcn_fwd(ip, ix, et, H1, p["W2"]) + p["b2"]
@@ -79,4 +85,6 @@ def rgcn2(ip, ix, et, X, lab, p):
     db2 = dZ2.sum(0)
     dZ1 = oracle.act_bwd("relu", Z1, dH1)
     _, dW1 = oracle.rgcn_bwd(ip, ix, et, X, p["W1"], dZ1, need_dX=False)
+    if acts is not None:
+        acts.update(H1=H1, logits=Z2)
     return loss, {"W1": dW1, "b1": dZ1.sum(0), "W2": dW2, "b2": db2}

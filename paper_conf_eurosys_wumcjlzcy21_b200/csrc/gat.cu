@@ -381,23 +381,25 @@ __global__ void k_gat_bwd_prep(int64_t M, int H, int F, int64_t ldt, const float
     const int h = (int)(i % H);
     const int64_t o = v * ldt + (int64_t)h * F;
     float* rec = D + v * ldd;
-    float cdot = 0.f, bdot = 0.f;
+    // c and der in fp64: der = <dA, B> - c b cancels down to the LeakyReLU-negative part of the softmax
+    // (|der| << |c|), so the two dot products are carried at double precision (F FMAs per (v,h))
+    double cdot = 0.0, bdot = 0.0;
     for (int f = 0; f < F; ++f) {
         float d = __ldg(dY + o + f);
         if (act != SEASTAR_ACT_NONE) d *= act_grad_from_y(act, __ldg(Y + o + f));
         rec[(int64_t)h * F + f] = d;
-        cdot = fmaf(d, __ldg(A + o + f), cdot);
-        if (B) bdot = fmaf(d, __ldg(B + o + f), bdot);
+        cdot = fma((double)d, (double)__ldg(A + o + f), cdot);
+        if (B) bdot = fma((double)d, (double)__ldg(B + o + f), bdot);
     }
     // der_v = sum_e a_e LReLU'(s_e) (g_e - c_v) = <dA_v, B_v> - c_v b_v   (B, b from the forward)
-    if (B) der[i] = bdot - cdot * __ldg(bsum + i);
+    if (B) der[i] = (float)(bdot - cdot * (double)__ldg(bsum + i));
     if (h == H - 1)   // zero the padding between dA and the aux block so vector loads read zeros
         for (int64_t f = (int64_t)H * F; f < rec_aux_offset(H * F); ++f) rec[f] = 0.f;
     float* aux = rec + rec_aux_offset(H * F) + 4 * h;
     aux[0] = __ldg(er + i);
     const float l = __ldg(lse + i);
     aux[1] = l;
-    aux[2] = cdot;
+    aux[2] = (float)cdot;
     aux[3] = -l * kLog2e;   // nl2: a_e = ex2(LReLU(s_e) log2 e + nl2)
 }
 

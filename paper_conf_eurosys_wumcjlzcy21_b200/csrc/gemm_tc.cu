@@ -86,6 +86,36 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
                  : "memory");
 }
 
+// Add TMEM slot (j & 1) -- the finished accumulation segment j -- into the fp32 register accumulators
+// of this thread's row (lane quarter q4), in column order, then hand the slot back to the MMA issuer.
+template <int NP>
+__device__ __forceinline__ void drain_segment(uint32_t tmem, int j, int q4, uint64_t* seg_done, uint64_t* slot_free,
+                                              float (&racc)[NP]) {
+    const int slot = j & 1;
+    mbar_wait(&seg_done[slot], (j >> 1) & 1);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll
+    for (int c0 = 0; c0 < NP; c0 += 16) {
+        uint32_t v[16];
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+            : "r"(tmem + ((uint32_t)(q4 * 32) << 16) + (uint32_t)(slot * NP + c0)));
+        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+        for (int q = 0; q < 16; ++q) racc[c0 + q] += __uint_as_float(v[q]);
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    mbar_arrive(&slot_free[slot]);
+}
+
+#ifndef TC_SEG
+#define TC_SEG 2
+#endif
+#ifndef TC_TN_SEG
+#define TC_TN_SEG 2
+#endif
 #ifndef TC_TWO_CTAS
 #define TC_TWO_CTAS 1
 #endif
@@ -99,11 +129,12 @@ struct TcCfg {
     static constexpr uint32_t A_BYTES = BM * BK * 4;          // 16 KB
     static constexpr uint32_t B_BYTES = NP * BK * 4;          // NP rows of 128 B
     static constexpr uint32_t STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
-    // G independent accumulators, K-chunk kc -> accumulator kc % G: each accumulates ~nk/G chunks, which
-    // bounds the error of the tensor core's accumulation; the epilogue sums them in fp32 registers
-    static constexpr int G = (NP <= 32 || (NP <= 64 && CTAS == 1)) ? 8 : (NP <= 128 ? 4 : 2);
-    static constexpr uint32_t TMEM_COLS = (G * NP) <= 32 ? 32 : ((G * NP) <= 64 ? 64 : ((G * NP) <= 128 ? 128 :
-                                          ((G * NP) <= 256 ? 256 : 512)));
+    // accumulation segments of SEG K chunks ping-pong between two TMEM slots; after each segment the
+    // epilogue warps add the slot into fp32 registers (IEEE round-to-nearest), so the tensor core's own
+    // accumulation never spans more than SEG * 12 MMAs (this keeps the K = 8,415 / 8,710
+    // transforms of the Physics / CoraFull configs within 1e-6)
+    static constexpr int SEG = TC_SEG;
+    static constexpr uint32_t TMEM_COLS = (2 * NP) <= 32 ? 32 : ((2 * NP) <= 64 ? 64 : ((2 * NP) <= 128 ? 128 : 256));
     static constexpr size_t SMEM = (size_t)STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 };
 
@@ -116,8 +147,9 @@ __global__ void __launch_bounds__(192, TcCfg<NP>::CTAS) k_gemm_tc(const __grid_c
     uint64_t* full = bars;                       // TMA landed
     uint64_t* split = bars + C::STAGES;          // hi/lo written (128 arrivals)
     uint64_t* empty = bars + 2 * C::STAGES;      // MMAs done reading
-    uint64_t* accum = bars + 3 * C::STAGES;      // accumulator complete
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * C::STAGES + 1);
+    uint64_t* seg_done = bars + 3 * C::STAGES;   // [2] segment accumulated in TMEM slot b
+    uint64_t* slot_free = seg_done + 2;          // [2] slot b drained into registers (128 arrivals)
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(seg_done + 4);
     auto A_hi = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES; };
     auto A_lo = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + C::A_BYTES; };
     auto B_hi = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + 2 * C::A_BYTES; };
@@ -133,7 +165,10 @@ __global__ void __launch_bounds__(192, TcCfg<NP>::CTAS) k_gemm_tc(const __grid_c
             mbar_init(&split[s], 128);
             mbar_init(&empty[s], 1);
         }
-        mbar_init(accum, 1);
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(&seg_done[b], 1);
+            mbar_init(&slot_free[b], 128);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
     }
@@ -165,28 +200,34 @@ __global__ void __launch_bounds__(192, TcCfg<NP>::CTAS) k_gemm_tc(const __grid_c
         const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NP >> 3) << 17) | ((128u >> 4) << 24);
         for (int kc = 0; kc < nk; ++kc) {
             const int s = kc % C::STAGES;
+            const int j = kc / C::SEG, slot = j & 1;
+            const bool first = (kc % C::SEG) == 0;
+            if (first && j >= 2) mbar_wait(&slot_free[slot], ((j >> 1) - 1) & 1);   // segment j-2 drained
             mbar_wait(&split[s], (kc / C::STAGES) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
             if (lane == 0) {
                 const uint64_t ah = smem_desc_k128(A_hi(s)), al = smem_desc_k128(A_lo(s));
                 const uint64_t bh = smem_desc_k128(B_hi(s)), bl = smem_desc_k128(B_lo(s));
-#pragma unroll
-                const uint32_t d = tmem + (uint32_t)((kc % C::G) * NP);
+                const uint32_t d = tmem + (uint32_t)(slot * NP);
 #pragma unroll
                 for (int ks = 0; ks < C::BK / 8; ++ks) {
                     const uint64_t adv = (uint64_t)((ks * 8 * 4) >> 4);   // 32 B per 8-wide K step
-                    mma_tf32(d, al + adv, bh + adv, idesc, (kc >= C::G || ks > 0) ? 1u : 0u);
+                    mma_tf32(d, al + adv, bh + adv, idesc, (!first || ks > 0) ? 1u : 0u);
                     mma_tf32(d, ah + adv, bl + adv, idesc, 1u);
                     mma_tf32(d, ah + adv, bh + adv, idesc, 1u);
                 }
                 mma_commit(&empty[s]);
-                if (kc == nk - 1) mma_commit(accum);
+                if ((kc % C::SEG) == C::SEG - 1 || kc == nk - 1) mma_commit(&seg_done[slot]);
             }
             __syncwarp();
         }
     } else {
-        // ---------------- split (then epilogue) ----------------
+        // ---------------- split, segment drains (then epilogue) ----------------
         const int t = threadIdx.x - 64;                     // 0..127
+        const int q4 = warp & 3;                            // TMEM lane quarter accessible to this warp
+        float racc[NP];
+#pragma unroll
+        for (int j = 0; j < NP; ++j) racc[j] = 0.f;
         for (int kc = 0; kc < nk; ++kc) {
             const int s = kc % C::STAGES;
             const int k0 = kc * C::BK;
@@ -210,42 +251,22 @@ __global__ void __launch_bounds__(192, TcCfg<NP>::CTAS) k_gemm_tc(const __grid_c
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             mbar_arrive(&split[s]);
+            // one segment behind the MMAs: drain segment j-1 once segment j is fully split
+            if (((kc % C::SEG) == C::SEG - 1 || kc == nk - 1) && kc / C::SEG >= 1)
+                drain_segment<NP>(tmem, kc / C::SEG - 1, q4, seg_done, slot_free, racc);
         }
-        // ---------------- epilogue ----------------
-        mbar_wait(accum, 0);
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const int q4 = warp & 3;                         // TMEM lane quarter accessible to this warp
+        if (nk > 0) drain_segment<NP>(tmem, (nk - 1) / C::SEG, q4, seg_done, slot_free, racc);
+        // ---------------- epilogue: bias, activation, row scale ----------------
         const int r = q4 * 32 + lane;
         const int64_t gm = m0 + r;
-        const float rs = (gm < a.M && a.row_scale) ? __ldg(a.row_scale + gm) : 1.f;
-        const int nacc = nk < C::G ? nk : C::G;
-#pragma unroll 1
-        for (int c0 = 0; c0 < NP; c0 += 16) {
-            float accv[16];
+        if (gm < a.M) {
+            const float rs = a.row_scale ? __ldg(a.row_scale + gm) : 1.f;
+            float* y = a.Y + gm * a.ldy;
 #pragma unroll
-            for (int j = 0; j < 16; ++j) accv[j] = 0.f;
-            for (int g = 0; g < nacc; ++g) {          // fixed order: deterministic
-                uint32_t v[16];
-                asm volatile(
-                    "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
-                    "[%16];"
-                    : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-                      "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
-                      "=r"(v[15])
-                    : "r"(tmem + ((uint32_t)(q4 * 32) << 16) + (uint32_t)(g * NP + c0)));
-                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-#pragma unroll
-                for (int j = 0; j < 16; ++j) accv[j] += __uint_as_float(v[j]);
-            }
-            if (gm < a.M) {
-                float* y = a.Y + gm * a.ldy;
-#pragma unroll
-                for (int j = 0; j < 16; ++j) {
-                    const int64_t n = c0 + j;
-                    if (n < a.N) {
-                        const float z = accv[j] + (a.bias ? __ldg(a.bias + n) : 0.f);
-                        y[n] = rs * act_apply(a.act, z);
-                    }
+            for (int j = 0; j < NP; ++j) {
+                if (j < a.N) {
+                    const float z = racc[j] + (a.bias ? __ldg(a.bias + j) : 0.f);
+                    y[j] = rs * act_apply(a.act, z);
                 }
             }
         }
@@ -372,8 +393,10 @@ struct TcTnCfg {
     static constexpr uint32_t A_BYTES = BM * BR * 4;           // 16 KB
     static constexpr uint32_t B_BYTES = NP32 * BR * 4;         // 4 KB per 32 columns
     static constexpr uint32_t STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
-    static constexpr int G = NP32 <= 32 ? 8 : 4;               // interleaved accumulators (<= 256 cols)
-    static constexpr uint32_t TMEM_COLS = G * NP32 <= 128 ? 128 : 256;
+    // segments of SEG 32-row chunks ping-pong between two TMEM slots and are drained into fp32
+    // registers (drain_segment, as in k_gemm_tc): no TMEM accumulation spans more than SEG * 12 MMAs
+    static constexpr int SEG = TC_TN_SEG;
+    static constexpr uint32_t TMEM_COLS = 2 * NP32 <= 64 ? 64 : 128;
     static constexpr size_t SMEM = (size_t)STAGES * STAGE_BYTES + 1024 + 256;
 };
 
@@ -402,8 +425,9 @@ __global__ void __launch_bounds__(192, TcTnCfg<NP32>::CTAS)
     uint64_t* full = bars;
     uint64_t* split = bars + C::STAGES;
     uint64_t* empty = bars + 2 * C::STAGES;
-    uint64_t* accum = bars + 3 * C::STAGES;
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * C::STAGES + 1);
+    uint64_t* seg_done = bars + 3 * C::STAGES;   // [2]
+    uint64_t* slot_free = seg_done + 2;          // [2] (128 arrivals)
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(seg_done + 4);
     auto A_hi = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES; };
     auto A_lo = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + C::A_BYTES; };
     auto B_hi = [&](int s) { return smem + (size_t)s * C::STAGE_BYTES + 2 * C::A_BYTES; };
@@ -421,7 +445,10 @@ __global__ void __launch_bounds__(192, TcTnCfg<NP32>::CTAS)
             mbar_init(&split[s], 128);
             mbar_init(&empty[s], 1);
         }
-        mbar_init(accum, 1);
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(&seg_done[b], 1);
+            mbar_init(&slot_free[b], 128);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
@@ -455,27 +482,34 @@ __global__ void __launch_bounds__(192, TcTnCfg<NP32>::CTAS)
                                ((uint32_t)(NP32 >> 3) << 17) | ((128u >> 4) << 24);
         for (int c = 0; c < nch; ++c) {
             const int s = c % C::STAGES;
+            const int j = c / C::SEG, slot = j & 1;
+            const bool first = (c % C::SEG) == 0;
+            if (first && j >= 2) mbar_wait(&slot_free[slot], ((j >> 1) - 1) & 1);   // segment j-2 drained
             mbar_wait(&split[s], (c / C::STAGES) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
             if (lane == 0) {
-                const uint32_t d = tmem + (uint32_t)((c % C::G) * NP32);
+                const uint32_t d = tmem + (uint32_t)(slot * NP32);
 #pragma unroll
                 for (int ks = 0; ks < C::BR / 8; ++ks) {
                     const uint64_t ah = smem_desc_mn32b(A_hi(s) + ks * 1024, 4096);
                     const uint64_t al = smem_desc_mn32b(A_lo(s) + ks * 1024, 4096);
                     const uint64_t bh = smem_desc_mn32b(B_hi(s) + ks * 1024, 4096);
                     const uint64_t bl = smem_desc_mn32b(B_lo(s) + ks * 1024, 4096);
-                    mma_tf32(d, al, bh, idesc, (c >= C::G || ks > 0) ? 1u : 0u);
+                    mma_tf32(d, al, bh, idesc, (!first || ks > 0) ? 1u : 0u);
                     mma_tf32(d, ah, bl, idesc, 1u);
                     mma_tf32(d, ah, bh, idesc, 1u);
                 }
                 mma_commit(&empty[s]);
-                if (c == nch - 1) mma_commit(accum);
+                if ((c % C::SEG) == C::SEG - 1 || c == nch - 1) mma_commit(&seg_done[slot]);
             }
             __syncwarp();
         }
     } else {
         const int t = threadIdx.x - 64;
+        const int q4 = warp & 3;
+        float racc[NP32];
+#pragma unroll
+        for (int j = 0; j < NP32; ++j) racc[j] = 0.f;
         for (int c = 0; c < nch; ++c) {
             const int s = c % C::STAGES;
             mbar_wait(&full[s], (c / C::STAGES) & 1);
@@ -500,40 +534,18 @@ __global__ void __launch_bounds__(192, TcTnCfg<NP32>::CTAS)
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             mbar_arrive(&split[s]);
+            if (((c % C::SEG) == C::SEG - 1 || c == nch - 1) && c / C::SEG >= 1)
+                drain_segment<NP32>(tmem, c / C::SEG - 1, q4, seg_done, slot_free, racc);
         }
-        // epilogue: partial[split][k0 + r][n] = sum_g acc_g[r][n]
-        const int q4 = warp & 3;
+        if (nch > 0) drain_segment<NP32>(tmem, (nch - 1) / C::SEG, q4, seg_done, slot_free, racc);
+        // epilogue: partial[split][k0 + r][n]
         const int r = q4 * 32 + lane;
         const int64_t gk = k0 + r;
-        float* prow = a.part + ((int64_t)blockIdx.y * a.K + gk) * a.N;
-        if (nch > 0) {
-            mbar_wait(accum, 0);
-            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        }
-        const int nacc = nch < C::G ? nch : C::G;
-#pragma unroll 1
-        for (int c0 = 0; c0 < NP32; c0 += 16) {
-            float accv[16];
+        if (gk < a.K) {
+            float* prow = a.part + ((int64_t)blockIdx.y * a.K + gk) * a.N;
 #pragma unroll
-            for (int j = 0; j < 16; ++j) accv[j] = 0.f;
-            for (int g = 0; g < nacc; ++g) {
-                uint32_t v[16];
-                asm volatile(
-                    "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
-                    "[%16];"
-                    : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-                      "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
-                      "=r"(v[15])
-                    : "r"(tmem + ((uint32_t)(q4 * 32) << 16) + (uint32_t)(g * NP32 + c0)));
-                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-#pragma unroll
-                for (int j = 0; j < 16; ++j) accv[j] += __uint_as_float(v[j]);
-            }
-            if (gk < a.K) {
-#pragma unroll
-                for (int j = 0; j < 16; ++j)
-                    if (c0 + j < a.N) prow[c0 + j] = accv[j];
-            }
+            for (int j = 0; j < NP32; ++j)
+                if (j < a.N) prow[j] = racc[j];
         }
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");

@@ -191,12 +191,15 @@ __global__ void __launch_bounds__(256) k_gemm_tn(const float* __restrict__ X, in
     }
 }
 
-__global__ void k_sum_splits(const float* __restrict__ part, int64_t nsplit, int64_t n, float* __restrict__ out) {
-    const int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (j >= n) return;
-    float x = 0.f;
-    for (int64_t b = 0; b < nsplit; ++b) x += part[b * n + j];
-    out[j] = x;
+// out[k * ldo + j] = sum_b part[b][k][j] (split order, fp64 accumulator) for one column chunk of width nc
+__global__ void k_sum_splits(const float* __restrict__ part, int64_t nsplit, int64_t K, int64_t nc,
+                             float* __restrict__ out, int64_t ldo) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t n = K * nc;
+    if (i >= n) return;
+    double x = 0.0;
+    for (int64_t b = 0; b < nsplit; ++b) x += (double)part[b * n + i];
+    out[(i / nc) * ldo + (i % nc)] = (float)x;
 }
 
 static void tn_geometry(int64_t M, int64_t K, int64_t& ktiles, int64_t& nsplit, int64_t& rows_per_split) {
@@ -258,11 +261,16 @@ seastar_status seastar_linear_bwd_data(const float* dY, int64_t M, int64_t Nout,
     return launch_gemm(g, to_stream(stream));
 }
 
+// dW is produced in column chunks of at most 64 outputs (the width one tcgen05 / SIMT tile covers);
+// each chunk's row-split partials go through the workspace and are summed in split order
+static const int64_t kBwdWChunk = 64;
+
 size_t seastar_linear_bwd_weight_workspace(int64_t M, int64_t K, int64_t Nout) {
+    const int64_t nc = Nout < kBwdWChunk ? Nout : kBwdWChunk;
     int64_t kt, ns, rps;
     tn_geometry(M > 0 ? M : 1, K, kt, ns, rps);
-    size_t part = (size_t)ns * K * Nout * sizeof(float);
-    const size_t tc = linear_bwd_weight_tc_part_bytes(M, K, Nout);
+    size_t part = (size_t)ns * K * nc * sizeof(float);
+    const size_t tc = linear_bwd_weight_tc_part_bytes(M, K, nc);
     if (tc > part) part = tc;
     return part + colsum_ws(M, Nout) + 512;
 }
@@ -271,28 +279,31 @@ seastar_status seastar_linear_bwd_weight(const float* X, int64_t M, int64_t K, i
                                          int64_t Nout, int64_t ldy, float* dW, float* db, void* workspace,
                                          size_t ws_bytes, seastar_stream stream) {
     SS_ARG(X && dY && dW && workspace, "linear_bwd_weight: NULL argument");
-    SS_ARG(M >= 1 && K >= 1 && Nout >= 1 && Nout <= 64 && ldx >= K && ldy >= Nout,
-           "linear_bwd_weight: bad sizes (need 1 <= Nout <= 64)");
+    SS_ARG(M >= 1 && K >= 1 && Nout >= 1 && ldx >= K && ldy >= Nout, "linear_bwd_weight: bad sizes");
     SS_ARG(ws_bytes >= seastar_linear_bwd_weight_workspace(M, K, Nout), "linear_bwd_weight: workspace too small");
     SS_TRY(check_device());
     cudaStream_t s = to_stream(stream);
-    int64_t kt, ns, rps;
     float* part = static_cast<float*>(workspace);
-    // tcgen05 3xTF32 path (MN-major TMA operands); SIMT fp32 otherwise
-    const seastar_status st = linear_bwd_weight_tc(X, M, K, ldx, dY, Nout, ldy, part, &ns, s);
-    if (st == SEASTAR_ERR_UNSUPPORTED) {
-        tn_geometry(M, K, kt, ns, rps);
-        dim3 grid((unsigned)kt, (unsigned)ns);
-        if (Nout <= 16) k_gemm_tn<16><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
-        else if (Nout <= 32) k_gemm_tn<32><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
-        else k_gemm_tn<64><<<grid, 256, 0, s>>>(X, ldx, dY, ldy, M, K, Nout, rps, part);
-        SS_TRY(check_launch("k_gemm_tn"));
-    } else if (st != SEASTAR_OK) {
-        return st;
+    for (int64_t c0 = 0; c0 < Nout; c0 += kBwdWChunk) {
+        const int64_t nc = Nout - c0 < kBwdWChunk ? Nout - c0 : kBwdWChunk;
+        const float* dYc = dY + c0;
+        int64_t kt, ns, rps;
+        // tcgen05 3xTF32 path (MN-major TMA operands); SIMT fp32 otherwise
+        const seastar_status st = linear_bwd_weight_tc(X, M, K, ldx, dYc, nc, ldy, part, &ns, s);
+        if (st == SEASTAR_ERR_UNSUPPORTED) {
+            tn_geometry(M, K, kt, ns, rps);
+            dim3 grid((unsigned)kt, (unsigned)ns);
+            if (nc <= 16) k_gemm_tn<16><<<grid, 256, 0, s>>>(X, ldx, dYc, ldy, M, K, nc, rps, part);
+            else if (nc <= 32) k_gemm_tn<32><<<grid, 256, 0, s>>>(X, ldx, dYc, ldy, M, K, nc, rps, part);
+            else k_gemm_tn<64><<<grid, 256, 0, s>>>(X, ldx, dYc, ldy, M, K, nc, rps, part);
+            SS_TRY(check_launch("k_gemm_tn"));
+        } else if (st != SEASTAR_OK) {
+            return st;
+        }
+        const int64_t n = K * nc;
+        k_sum_splits<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(part, ns, K, nc, dW + c0, Nout);
+        SS_TRY(check_launch("k_sum_splits"));
     }
-    const int64_t n = K * Nout;
-    k_sum_splits<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(part, ns, n, dW);
-    SS_TRY(check_launch("k_sum_splits"));
     if (db) {
         size_t off = ((seastar_linear_bwd_weight_workspace(M, K, Nout) - colsum_ws(M, Nout) - 512) + 255) & ~size_t(255);
         SS_TRY(colsum_impl(dY, M, Nout, ldy, db, static_cast<char*>(workspace) + off, ws_bytes - off, s));

@@ -360,6 +360,11 @@ class APPNPNet:
         P = self.comm.world
         self.Zs_all = e(self.rows_all, self.ldc) if P > 1 else None
         self.Gs_all = e(self.rows_all, self.ldc) if P > 1 else None
+        self.timer = None
+
+    def _t(self, name):
+        if self.timer is not None:
+            self.timer(name)
 
     def forward(self):
         g, p, n, Hd, C, ld = self.g, self.P, self.n, self.Hd, self.C, self.ldc
@@ -369,8 +374,10 @@ class APPNPNet:
         _linear(self.ws, self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), self.nrm, "none", self.Zs[0], ld)
         for k in range(self.K):
             Zs_all = self.comm.all_gather(self.Zs_all, self.Zs[k])
+            self._t("appnp_fwd") if k == 0 else None
             L.seastar_gcn_fwd(g.handle, Zs_all, C, ld, self.nrm, None, "none", self.alpha, self.H0, self.Z[k + 1],
                               self.nrm, self.Zs[k + 1])
+            self._t("appnp_fwd_end") if k == 0 else None
         out = self.Z[self.K] if self.K > 0 else self.H0
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
         L.seastar_softmax_xent(out, n, self.g.N, C, ld, self.lab, self.loss, self.G, ld, ws, ws.numel())
@@ -388,7 +395,9 @@ class APPNPNet:
             L.seastar_axpby(n * ld, a, G, 1.0, self.dH0)
             Gs_all = self.comm.all_gather(self.Gs_all, self.Gs[cur])
             nxt = self.Gtmp if G is self.G else self.G
+            self._t("appnp_bwd") if k == 0 else None
             L.seastar_gcn_bwd(g.handle, Gs_all, C, ld, self.nrm, 1.0 - a, None, "none", self.nrm, nxt, self.Gs[1 - cur])
+            self._t("appnp_bwd_end") if k == 0 else None
             G = nxt
             cur = 1 - cur
         L.seastar_axpby(n * ld, 1.0, G, 1.0, self.dH0)
@@ -446,11 +455,17 @@ class RGCN2:
         self.dZ1_all = e(Ra, self.ldh) if P > 1 else None
         self.timer = None
 
+    def _t(self, name):
+        if self.timer is not None:
+            self.timer(name)
+
     def forward(self):
         g, p, n = self.g, self.P, self.n
         self._X_all = self.comm.all_gather(self.X_all, self.X)
+        self._t("rgcn_fwd1")
         L.seastar_rgcn_fwd(g.handle, self._X_all, self.Fin, self.X.stride(0), p.p("W1"), self.Hd, None, p.p("b1"),
                            "relu", self.H1, self.ldh)
+        self._t("rgcn_fwd1_end")
         self._H1_all = self.comm.all_gather(self.H1_all, self.H1)
         L.seastar_rgcn_fwd(g.handle, self._H1_all, self.Hd, self.ldh, p.p("W2"), self.C, None, p.p("b2"), "none",
                            self.logits, self.ldc)
@@ -466,8 +481,10 @@ class RGCN2:
                               L.seastar_colsum_workspace(n, max(self.C, self.Hd))))
         L.seastar_colsum(self.dlog, n, self.C, self.ldc, p.g("b2"), ws, ws.numel())
         dlog_all = self.comm.all_gather(self.dlog_all, self.dlog)
+        self._t("rgcn_bwd2")
         L.seastar_rgcn_bwd(g.handle, self._H1_all, self.Hd, self.ldh, dlog_all, self.C, self.ldc, p.p("W2"), None,
                            self.H1, "relu", self.dZ1, p.g("W2"), ws, ws.numel())
+        self._t("rgcn_bwd2_end")
         L.seastar_colsum(self.dZ1, n, self.Hd, self.ldh, p.g("b1"), ws, ws.numel())
         dZ1_all = self.comm.all_gather(self.dZ1_all, self.dZ1)
         L.seastar_rgcn_bwd(g.handle, self._X_all, self.Fin, self.X.stride(0), dZ1_all, self.Hd, self.ldh, p.p("W1"),

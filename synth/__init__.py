@@ -196,3 +196,42 @@ def make_graph(cfg: Config):
     if cfg.typed:
         return powerlaw_directed_typed(cfg.N, cfg.E_dir, cfg.s, cfg.s, cfg.R, cfg.zipf_a, cfg.graph_seed)
     return powerlaw_sym(cfg.N, cfg.E_dir, cfg.s, cfg.graph_seed, cfg.self_loops)
+
+
+def _gcn_params(cfg: Config, fin: int, hid: int, C: int, base: int = 0) -> dict:
+    return {"W1": glorot(cfg.weight_seed(base + 1), fin, hid), "b1": np.zeros(hid, np.float32),
+            "W2": glorot(cfg.weight_seed(base + 2), hid, C), "b2": np.zeros(C, np.float32)}
+
+
+def _gat_params(cfg: Config, heads: int, hid: int) -> dict:
+    Wd, C = heads * hid, cfg.classes
+    return {"W1": glorot(cfg.weight_seed(11), cfg.F_in, Wd),
+            "al1": glorot(cfg.weight_seed(12), hid, 1, (heads, hid)),
+            "ar1": glorot(cfg.weight_seed(13), hid, 1, (heads, hid)),
+            "b1": np.zeros(Wd, np.float32),
+            "W2": glorot(cfg.weight_seed(14), Wd, C),
+            "al2": glorot(cfg.weight_seed(15), C, 1, (1, C)),
+            "ar2": glorot(cfg.weight_seed(16), C, 1, (1, C)),
+            "b2": np.zeros(C, np.float32)}
+
+
+def workload(name: str) -> dict:
+    """The complete seeded input set of one BASELINE config: graph, features, labels and the initial
+    parameters of every model the config trains (biases 0, as in DGL's init; Glorot weights).
+    Keys: cfg, indptr, indices, etypes (typed only), X [N, F_in] f32, labels [N] i64, and one
+    parameter dict per model name ("gcn", "gat", "appnp", "rgcn")."""
+    cfg = CONFIGS[name]
+    g = make_graph(cfg)
+    out = {"cfg": cfg, "indptr": g[0], "indices": g[1], "etypes": g[2] if cfg.typed else None,
+           "X": uniform(cfg.feat_seed, (cfg.N, cfg.F_in), -1.0, 1.0),
+           "labels": labels(cfg.label_seed, cfg.N, cfg.classes)}
+    models = cfg.model.split("+")
+    if "gcn" in models or "appnp" in models:
+        out[models[0] if "appnp" in models else "gcn"] = _gcn_params(cfg, cfg.F_in, cfg.hidden, cfg.classes)
+    if "gat" in models:
+        out["gat"] = _gat_params(cfg, cfg.heads, cfg.extra.get("gat_hidden", cfg.hidden))
+    if "rgcn" in models:
+        R, fin, hid, C = cfg.R, cfg.F_in, cfg.hidden, cfg.classes
+        out["rgcn"] = {"W1": glorot(cfg.weight_seed(1), fin, hid, (R, fin, hid)), "b1": np.zeros(hid, np.float32),
+                       "W2": glorot(cfg.weight_seed(2), hid, C, (R, hid, C)), "b2": np.zeros(C, np.float32)}
+    return out

@@ -72,8 +72,6 @@ def test_linear_fwd_tcgen05(env, M, K, N):
 @pytest.mark.parametrize("M,K,N", SHAPES)
 def test_linear_bwd(env, M, K, N):
     torch, L = env["torch"], env["L"]
-    if N > 64:
-        pytest.skip("bwd_weight supports Nout <= 64")
     X, W, dY = rnd(5, (M, K)), rnd(6, (K, N)), rnd(7, (M, N))
     rs = rnd(8, (M,), 0.5, 2.0)
     dX = torch.empty((M, K), device="cuda")
@@ -136,7 +134,7 @@ def test_colsum_axpby_adam(env):
 
 
 TC_TN_SHAPES = [(256, 32, 1), (1000, 602, 16), (5003, 602, 64), (3001, 64, 41), (300, 8710, 8), (4099, 100, 33),
-                (20000, 128, 32), (233, 602, 16)]
+                (20000, 128, 32), (233, 602, 16), (2000, 64, 70), (3000, 100, 130), (300, 40, 200)]
 
 
 @pytest.mark.parametrize("M,K,N", TC_TN_SHAPES)

@@ -6,7 +6,7 @@ import pytest
 import oracle
 import synth
 from conftest import rel_err
-import model_ref
+from oracle import model_ref
 
 pytestmark = pytest.mark.gpu
 TOL = 1e-5

@@ -7,7 +7,7 @@ import threading
 import numpy as np
 import pytest
 
-import model_ref
+from oracle import model_ref
 import synth
 from conftest import rel_err
 

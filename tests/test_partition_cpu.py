@@ -133,7 +133,7 @@ def _worker(rank, world, port, errfile):
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        import model_ref
+        from oracle import model_ref
         import synth
         from paper_conf_eurosys_wumcjlzcy21_b200 import partition as part
         from paper_conf_eurosys_wumcjlzcy21_b200.models import Comm
