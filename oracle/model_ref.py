@@ -23,7 +23,7 @@ def gcn2(ip, ix, X, lab, p, acts=None):
     dT = oracle.gcn_aggregate_T(ip, ix, dZ1, out_n, in_n)
     _, dW1, _ = oracle.linear_bwd(X, p["W1"], dT, need_dX=False, need_db=False)
     if acts is not None:
-        acts.update(H1=H1, logits=logits)
+        acts.update(H1=H1, logits=logits, Z1=Z1, dH1=dH1)
     return loss, {"W1": dW1, "b1": db1, "W2": dW2, "b2": db2}
 
 
@@ -31,8 +31,9 @@ def _gat_layer_fwd(ip, ix, Xin, W, al, ar, b, act, H, F):
     N = Xin.shape[0]
     T = oracle.linear_fwd(Xin, W).reshape(N, H, F)
     el, er = oracle.gat_attn_proj(T, al, ar)
-    A, _, _ = oracle.gat_fwd(ip, ix, T, el, er, 0.2)
+    A, lse, _ = oracle.gat_fwd(ip, ix, T, el, er, 0.2)
     Z = A.reshape(N, H * F) + b
+    _gat_layer_fwd.lse = lse          # exposed to callers that want it (acts); not part of the return value
     return T, el, er, Z, oracle.act_fwd(act, Z)
 
 
@@ -44,20 +45,29 @@ def _gat_layer_bwd(ip, ix, Xin, W, al, ar, T, el, er, Z, act, dY, H, F, need_dX)
     dTp, dal, dar = oracle.gat_attn_proj_bwd(T, al, ar, dl, dr)
     dTt = (dT + dTp).reshape(N, H * F)
     dX, dW, _ = oracle.linear_bwd(Xin, W, dTt, need_dX=need_dX, need_db=False)
+    _gat_layer_bwd.dZ = dZ
     return dX, dW, dal, dar, db
 
 
 def gat2(ip, ix, X, lab, p, heads, hidden, acts=None):
     C = p["W2"].shape[1]
     T1, el1, er1, Z1, Y1 = _gat_layer_fwd(ip, ix, X, p["W1"], p["al1"], p["ar1"], p["b1"], "elu", heads, hidden)
+    lse1 = _gat_layer_fwd.lse
     T2, el2, er2, Z2, Y2 = _gat_layer_fwd(ip, ix, Y1, p["W2"], p["al2"], p["ar2"], p["b2"], "none", 1, C)
+    lse2 = _gat_layer_fwd.lse
     loss, dY2 = oracle.softmax_xent(Y2, lab)
     dY1, dW2, dal2, dar2, db2 = _gat_layer_bwd(ip, ix, Y1, p["W2"], p["al2"], p["ar2"], T2, el2, er2, Z2, "none",
                                                dY2, 1, C, True)
+    dZ2 = _gat_layer_bwd.dZ
     _, dW1, dal1, dar1, db1 = _gat_layer_bwd(ip, ix, X, p["W1"], p["al1"], p["ar1"], T1, el1, er1, Z1, "elu", dY1,
                                              heads, hidden, False)
+    dZ1 = _gat_layer_bwd.dZ
     if acts is not None:
-        acts.update(Y1=Y1, Y2=Y2)
+        acts.update(Y1=Y1, Y2=Y2,
+                    layers=[dict(Xin=X, T=T1, el=el1, er=er1, A=Z1 - p["b1"], lse=lse1, dZ=dZ1, al=p["al1"],
+                                 ar=p["ar1"]),
+                            dict(Xin=Y1, T=T2, el=el2, er=er2, A=Z2 - p["b2"], lse=lse2, dZ=dZ2, al=p["al2"],
+                                 ar=p["ar2"])])
     return loss, {"W1": dW1, "al1": dal1, "ar1": dar1, "b1": db1, "W2": dW2, "al2": dal2, "ar2": dar2, "b2": db2}
 
 
@@ -72,7 +82,7 @@ def appnp(ip, ix, X, lab, p, K, alpha, acts=None):
     dZ1 = oracle.act_bwd("relu", Z1, dHh)
     _, dW1, db1 = oracle.linear_bwd(X, p["W1"], dZ1, need_dX=False)
     if acts is not None:
-        acts.update(Z=Z)
+        acts.update(Z=Z, Z1=Z1, dH1=dHh)
     return loss, {"W1": dW1, "b1": db1, "W2": dW2, "b2": db2}
 
 
@@ -86,5 +96,5 @@ def rgcn2(ip, ix, et, X, lab, p, acts=None):
     dZ1 = oracle.act_bwd("relu", Z1, dH1)
     _, dW1 = oracle.rgcn_bwd(ip, ix, et, X, p["W1"], dZ1, need_dX=False)
     if acts is not None:
-        acts.update(H1=H1, logits=Z2)
+        acts.update(H1=H1, logits=Z2, Z1=Z1, dH1=dH1)
     return loss, {"W1": dW1, "b1": dZ1.sum(0), "W2": dW2, "b2": db2}

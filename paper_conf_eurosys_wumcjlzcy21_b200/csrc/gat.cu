@@ -369,38 +369,80 @@ __global__ void k_gat_attn_proj(const float* __restrict__ T, int64_t M, int H, i
     if (er) er[i] = sr;
 }
 
-// thread per (v,h): dA = dY act'(Y), c = <dA, A>, record D[v] = [dA | (er, lse, c, nl2) per head]
-__global__ void k_gat_bwd_prep(int64_t M, int H, int F, int64_t ldt, const float* __restrict__ dY,
-                               const float* __restrict__ Y, int act, const float* __restrict__ A,
-                               const float* __restrict__ er, const float* __restrict__ lse, float* __restrict__ D,
-                               int64_t ldd, const float* __restrict__ B, const float* __restrict__ bsum,
-                               float* __restrict__ der) {
-    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (i >= M * H) return;
-    const int64_t v = i / H;
-    const int h = (int)(i % H);
-    const int64_t o = v * ldt + (int64_t)h * F;
+// warp per row v (coalesced row reads): dA = dY act'(Y), c = <dA, A>, record D[v] = [dA | (er, lse, c, nl2)
+// per head]; with the forward-saved factors also der_v = <dA_v, B_v> - c_v b_v.  c and der are carried in
+// fp64: der cancels down to the LeakyReLU-negative part of the softmax (|der| << |c|).  Per-head sums are
+// fixed xor trees (deterministic): segmented over the F lanes of a head when F divides 32, else one full
+// warp reduction per head.
+__device__ __forceinline__ double warp_sum_seg(double x, int width) {
+    for (int o = width >> 1; o; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+    return x;
+}
+
+__global__ void __launch_bounds__(256) k_gat_bwd_prep(int64_t M, int H, int F, int64_t ldt,
+                                                      const float* __restrict__ dY, const float* __restrict__ Y,
+                                                      int act, const float* __restrict__ A,
+                                                      const float* __restrict__ er, const float* __restrict__ lse,
+                                                      float* __restrict__ D, int64_t ldd, const float* __restrict__ B,
+                                                      const float* __restrict__ bsum, float* __restrict__ der) {
+    const int lane = threadIdx.x & 31;
+    const int64_t v = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (v >= M) return;
+    const int W = H * F;
+    const int64_t o = v * ldt;
     float* rec = D + v * ldd;
-    // c and der in fp64: der = <dA, B> - c b cancels down to the LeakyReLU-negative part of the softmax
-    // (|der| << |c|), so the two dot products are carried at double precision (F FMAs per (v,h))
-    double cdot = 0.0, bdot = 0.0;
-    for (int f = 0; f < F; ++f) {
-        float d = __ldg(dY + o + f);
-        if (act != SEASTAR_ACT_NONE) d *= act_grad_from_y(act, __ldg(Y + o + f));
-        rec[(int64_t)h * F + f] = d;
-        cdot = fma((double)d, (double)__ldg(A + o + f), cdot);
-        if (B) bdot = fma((double)d, (double)__ldg(B + o + f), bdot);
+    const bool seg = (32 % F) == 0;           // a head's columns are F consecutive lanes of one 32-column pass
+    double cdot = 0.0, bdot = 0.0;             // this lane's head (seg) -- valid after the reductions
+    double cacc[8], bacc[8];                   // non-seg, H <= 8: per-head partials of this lane
+#pragma unroll
+    for (int h = 0; h < 8; ++h) cacc[h] = bacc[h] = 0.0;
+    for (int j0 = 0; j0 < W; j0 += 32) {
+        const int j = j0 + lane;
+        double pc = 0.0, pb = 0.0;
+        if (j < W) {
+            float d = __ldg(dY + o + j);
+            if (act != SEASTAR_ACT_NONE) d *= act_grad_from_y(act, __ldg(Y + o + j));
+            rec[j] = d;
+            pc = (double)d * (double)__ldg(A + o + j);
+            if (B) pb = (double)d * (double)__ldg(B + o + j);
+        }
+        if (seg) {
+            pc = warp_sum_seg(pc, F);
+            pb = warp_sum_seg(pb, F);
+            // every lane of head hh's group now holds its sum; lane hh (the head's owner, H <= 32) takes it
+            for (int hh = j0 / F; hh < H && hh * F < j0 + 32; ++hh) {
+                const double xc = __shfl_sync(0xffffffffu, pc, hh * F - j0);
+                const double xb = __shfl_sync(0xffffffffu, pb, hh * F - j0);
+                if (lane == hh) { cdot = xc; bdot = xb; }
+            }
+        } else {
+            const int h = j < W ? j / F : 0;
+#pragma unroll
+            for (int hh = 0; hh < 8; ++hh)
+                if (hh == h) { cacc[hh] += pc; bacc[hh] += pb; }
+        }
     }
-    // der_v = sum_e a_e LReLU'(s_e) (g_e - c_v) = <dA_v, B_v> - c_v b_v   (B, b from the forward)
-    if (B) der[i] = (float)(bdot - cdot * (double)__ldg(bsum + i));
-    if (h == H - 1)   // zero the padding between dA and the aux block so vector loads read zeros
-        for (int64_t f = (int64_t)H * F; f < rec_aux_offset(H * F); ++f) rec[f] = 0.f;
-    float* aux = rec + rec_aux_offset(H * F) + 4 * h;
-    aux[0] = __ldg(er + i);
-    const float l = __ldg(lse + i);
-    aux[1] = l;
-    aux[2] = (float)cdot;
-    aux[3] = -l * kLog2e;   // nl2: a_e = ex2(LReLU(s_e) log2 e + nl2)
+    if (!seg) {
+#pragma unroll
+        for (int hh = 0; hh < 8; ++hh) {
+            if (hh >= H) break;
+            const double xc = warp_sum_seg(cacc[hh], 32);
+            const double xb = warp_sum_seg(bacc[hh], 32);
+            if (lane == hh) { cdot = xc; bdot = xb; }
+        }
+    }
+    // zero the padding between dA and the aux block so vector loads read zeros
+    for (int f = W + lane; f < rec_aux_offset(W); f += 32) rec[f] = 0.f;
+    if (lane < H) {
+        const int64_t i = v * H + lane;
+        if (B) der[i] = (float)(bdot - cdot * (double)__ldg(bsum + i));
+        float* aux = rec + rec_aux_offset(W) + 4 * lane;
+        aux[0] = __ldg(er + i);
+        const float l = __ldg(lse + i);
+        aux[1] = l;
+        aux[2] = (float)cdot;
+        aux[3] = -l * kLog2e;   // nl2: a_e = ex2(LReLU(s_e) log2 e + nl2)
+    }
 }
 
 // stage 1 of attn_proj_bwd: dT += del a_l + der a_r (in place) and per-block partial da_l, da_r
@@ -422,6 +464,7 @@ __global__ void __launch_bounds__(256) k_gat_attn_proj_bwd1(const float* __restr
         if (j < W) {
             const int h = j / F;
             const float al = __ldg(a_l + j), ar = __ldg(a_r + j);
+#pragma unroll 4
             for (int64_t r = r0 + ty; r < r1; r += 8) {
                 const float t = __ldg(T + r * ldt + j);
                 const float dl = del ? __ldg(del + r * H + h) : 0.f;
@@ -443,18 +486,8 @@ __global__ void __launch_bounds__(256) k_gat_attn_proj_bwd1(const float* __restr
     }
 }
 
-// stage 2: out[j] = sum_b part[b*stride + j] in block order
-__global__ void k_sum_partials(const float* __restrict__ part, int64_t nblk, int64_t stride, int64_t n,
-                               float* __restrict__ out) {
-    const int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (j >= n) return;
-    float x = 0.f;
-    for (int64_t b = 0; b < nblk; ++b) x += part[b * stride + j];
-    out[j] = x;
-}
-
 static int64_t proj_bwd_blocks(int64_t M) {
-    int64_t b = 2 * num_sms();
+    int64_t b = 8 * num_sms();
     if (M < b * 64) b = (M + 63) / 64;
     return b < 1 ? 1 : b;
 }
@@ -578,8 +611,8 @@ seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const 
     SS_TRY(check_device());
     const int64_t M = g->n_loc();
     if (M == 0) return SEASTAR_OK;
-    const int64_t n = M * H;
-    k_gat_bwd_prep<<<(unsigned)((n + 255) / 256), 256, 0, to_stream(stream)>>>(
+    SS_ARG(H <= 8 || (32 % F == 0 && H <= 32), "gat_bwd_prep: H > 8 needs F dividing 32 (and H <= 32)");
+    k_gat_bwd_prep<<<(unsigned)((M + 7) / 8), 256, 0, to_stream(stream)>>>(
         M, H, F, ldt, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, D_loc, seastar_gat_record_ld(H, F), B_loc, b_loc,
         der_loc);
     return check_launch("k_gat_bwd_prep");
@@ -656,8 +689,8 @@ seastar_status seastar_gat_attn_proj_bwd(const float* T, int64_t M, int32_t H, i
     const int64_t rpb = (M + nblk - 1) / nblk;
     float* part = static_cast<float*>(workspace);
     k_gat_attn_proj_bwd1<<<(unsigned)nblk, 256, 0, s>>>(T, M, H, F, ldt, a_l, a_r, del, der, dT, rpb > 0 ? rpb : 1, part);
-    k_sum_partials<<<(unsigned)((W + 255) / 256), 256, 0, s>>>(part, nblk, 2 * (int64_t)W, W, da_l);
-    k_sum_partials<<<(unsigned)((W + 255) / 256), 256, 0, s>>>(part + W, nblk, 2 * (int64_t)W, W, da_r);
+    reduce_splits(part, nblk, 2 * (int64_t)W, W, W, W, da_l, s);
+    reduce_splits(part + W, nblk, 2 * (int64_t)W, W, W, W, da_r, s);
     return check_launch("k_gat_attn_proj_bwd");
 }
 

@@ -1,6 +1,7 @@
 // gat_h1.cu -- single-head GAT edge kernels (H = 1, any F <= 128, e.g. the output layer F = #classes):
-// each lane owns VPL consecutive float4 chunks of the row, L lanes (<= 4) cover one edge, S = RL / L
-// edge slots per row group; g = <dA, T> by an L-lane xor reduction.  PAPER.md Fig. 2 L95-L123,
+// L lanes (<= 4) cover one edge and lane c owns the float4 chunks c, c + L, c + 2L, ... of the row
+// (interleaved, so the L lanes' q-th loads are one contiguous 16L-byte span: each gathered row costs
+// ~ceil(row bytes / 64) L1 wavefronts instead of one per lane-chunk), S = RL / L edge slots per row group; g = <dA, T> by an L-lane xor reduction.  PAPER.md Fig. 2 L95-L123,
 // §6.3.4 L461-L463.  Same branch-free inner loop as gat_hpl.cu: an out-of-range edge slot gathers
 // row 0 and gets weight 0; chunks past the row end are never loaded (per-lane constant predicate).
 #include "gat_common.cuh"
@@ -16,10 +17,10 @@ constexpr int h1_ub() { return (VPL <= 2 ? 4 : 2) < GAT_H1_UBMAX ? (VPL <= 2 ? 4
 // load the lane's chunks of a row; chunks at or past W are zero (never loaded).  Columns inside
 // the last partial chunk are loaded as stored (row padding): callers either zero the matching
 // factor (own rows) or only read padding that is zero by construction (D records).
-template <int VPL>
+template <int VPL, int L>
 __device__ __forceinline__ void load_lane_chunks(const float* p, const bool (&qv)[VPL], float4 (&x)[VPL]) {
 #pragma unroll
-    for (int q = 0; q < VPL; ++q) x[q] = qv[q] ? ldg4(p + 4 * q) : make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int q = 0; q < VPL; ++q) x[q] = qv[q] ? ldg4(p + 4 * L * q) : make_float4(0.f, 0.f, 0.f, 0.f);
 }
 
 // zero the columns >= nv of a chunk (nv in 0..4)
@@ -42,10 +43,10 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
     const int beg = valid ? __ldg(a.off + row) : 0;
     const int end = valid ? __ldg(a.off + row + 1) : 0;
     const int64_t v = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;
-    const int W = a.F, col0 = c * NV;
+    const int W = a.F, col0 = 4 * c;             // chunk q of this lane: columns col0 + 4 L q ..
     bool qv[VPL];
 #pragma unroll
-    for (int q = 0; q < VPL; ++q) qv[q] = col0 + 4 * q < W;
+    for (int q = 0; q < VPL; ++q) qv[q] = col0 + 4 * L * q < W;
     const float erv = valid ? __ldg(a.er + v) : 0.f;
     const float slope = a.slope;
     const float* Tc = a.T + col0;
@@ -69,7 +70,7 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
             for (int jj = 0; jj < UE; ++jj) {
                 const int k = (b * UE + jj) * S + slot;     // < RL
                 const int u = __shfl_sync(gmask, my, k, RL);
-                load_lane_chunks<VPL>(row_ptr(Tc, u, a.ld), qv, x[jj]);
+                load_lane_chunks<VPL, L>(row_ptr(Tc, u, a.ld), qv, x[jj]);
                 const float s = __ldg(a.el + u) + erv;
                 z[jj] = k < n ? lrelu(s, slope) : -INFINITY;
             }
@@ -137,7 +138,7 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
     float* pb = SB ? a.B + v * a.ld : nullptr;
 #pragma unroll
     for (int q = 0; q < VPL; ++q) {
-        const int col = col0 + 4 * q;
+        const int col = col0 + 4 * L * q;
         if (col >= W) continue;
         float o4[4], y4[4], b4[4];
 #pragma unroll
@@ -180,26 +181,26 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD) k_gat_bwd_h1(const GatBwdArgs
     const int beg = valid ? __ldg(a.off + row) : 0;
     const int end = valid ? __ldg(a.off + row + 1) : 0;
     const int64_t w = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;   // u (src-major) or v (der)
-    const int W = a.F, col0 = c * NV;
+    const int W = a.F, col0 = 4 * c;             // chunk q of this lane: columns col0 + 4 L q ..
     const int aux0 = rec_aux_offset(W);
     const float slope = a.slope;
     bool qv[VPL];
 #pragma unroll
-    for (int q = 0; q < VPL; ++q) qv[q] = valid && col0 + 4 * q < W;
+    for (int q = 0; q < VPL; ++q) qv[q] = valid && col0 + 4 * L * q < W;
     // own row, padding columns zeroed so gathered padding never enters g
     float4 own[VPL];
     float4 k4 = make_float4(0.f, 0.f, 0.f, 0.f);   // src-major: (el_u, -, -, -); der: (er, lse, c, nl2)_v
     if (!DER) {
-        load_lane_chunks<VPL>(a.T + w * a.ldt + col0, qv, own);
+        load_lane_chunks<VPL, L>(a.T + w * a.ldt + col0, qv, own);
         if (valid) k4.x = __ldg(a.el + w);
     } else {
-        load_lane_chunks<VPL>(a.D + w * a.ldd + col0, qv, own);
+        load_lane_chunks<VPL, L>(a.D + w * a.ldd + col0, qv, own);
         if (valid) k4 = ldg4(a.D + w * a.ldd + aux0);
     }
     int nvalid[VPL];   // valid columns of each chunk (0..4)
 #pragma unroll
     for (int q = 0; q < VPL; ++q) {
-        nvalid[q] = min(4, max(0, W - (col0 + 4 * q)));
+        nvalid[q] = min(4, max(0, W - (col0 + 4 * L * q)));
         own[q] = mask_tail(own[q], nvalid[q]);
     }
     const float* Gc = DER ? a.T + col0 : a.D + col0;           // gathered rows
@@ -222,7 +223,7 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD) k_gat_bwd_h1(const GatBwdArgs
             for (int jj = 0; jj < UE; ++jj) {
                 kk[jj] = (b * UE + jj) * S + slot;
                 const int o = __shfl_sync(gmask, my, kk[jj], RL);
-                load_lane_chunks<VPL>(row_ptr(Gc, o, gld), qv, x[jj]);
+                load_lane_chunks<VPL, L>(row_ptr(Gc, o, gld), qv, x[jj]);
                 if (!DER) {
                     e[jj] = ldg4(row_ptr(a.D + aux0, o, a.ldd));          // (er, lse, c, nl2)_v
                 } else {
@@ -280,7 +281,7 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD) k_gat_bwd_h1(const GatBwdArgs
     float* pd = a.dT + w * a.ldt;
 #pragma unroll
     for (int q = 0; q < VPL; ++q) {
-        const int col = col0 + 4 * q;
+        const int col = col0 + 4 * L * q;
         if (col >= W) continue;
         if (col + 4 <= W)
             *reinterpret_cast<float4*>(pd + col) = make_float4(acc[4 * q], acc[4 * q + 1], acc[4 * q + 2], acc[4 * q + 3]);

@@ -191,17 +191,6 @@ __global__ void __launch_bounds__(256) k_gemm_tn(const float* __restrict__ X, in
     }
 }
 
-// out[k * ldo + j] = sum_b part[b][k][j] (split order, fp64 accumulator) for one column chunk of width nc
-__global__ void k_sum_splits(const float* __restrict__ part, int64_t nsplit, int64_t K, int64_t nc,
-                             float* __restrict__ out, int64_t ldo) {
-    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    const int64_t n = K * nc;
-    if (i >= n) return;
-    double x = 0.0;
-    for (int64_t b = 0; b < nsplit; ++b) x += (double)part[b * n + i];
-    out[(i / nc) * ldo + (i % nc)] = (float)x;
-}
-
 static void tn_geometry(int64_t M, int64_t K, int64_t& ktiles, int64_t& nsplit, int64_t& rows_per_split) {
     ktiles = (K + 63) / 64;
     int64_t want = (2 * num_sms() + ktiles - 1) / ktiles;   // ~2 waves of blocks
@@ -300,9 +289,8 @@ seastar_status seastar_linear_bwd_weight(const float* X, int64_t M, int64_t K, i
         } else if (st != SEASTAR_OK) {
             return st;
         }
-        const int64_t n = K * nc;
-        k_sum_splits<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(part, ns, K, nc, dW + c0, Nout);
-        SS_TRY(check_launch("k_sum_splits"));
+        reduce_splits(part, ns, K * nc, K * nc, nc, Nout, dW + c0, s);
+        SS_TRY(check_launch("k_reduce_splits"));
     }
     if (db) {
         size_t off = ((seastar_linear_bwd_weight_workspace(M, K, Nout) - colsum_ws(M, Nout) - 512) + 255) & ~size_t(255);

@@ -37,12 +37,35 @@ __global__ void __launch_bounds__(256) k_colsum1(const float* __restrict__ X, in
     }
 }
 
-__global__ void k_colsum2(const float* __restrict__ part, int64_t nblk, int64_t F, float* __restrict__ out) {
-    const int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (j >= F) return;
-    float x = 0.f;
-    for (int64_t b = 0; b < nblk; ++b) x += part[b * F + j];
-    out[j] = x;
+__global__ void __launch_bounds__(256) k_reduce_splits(const float* __restrict__ part, int64_t nsplit, int64_t stride,
+                                                       int64_t n, int64_t nc, int64_t ldo, float* __restrict__ out) {
+    __shared__ double red[8][32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t i = (int64_t)blockIdx.x * 32 + lane;
+    double x = 0.0;
+    if (i < n) {
+        int64_t b = w;
+        for (; b + 24 < nsplit; b += 32) {      // 4 independent loads in flight per lane
+            const float a0 = __ldg(part + b * stride + i), a1 = __ldg(part + (b + 8) * stride + i);
+            const float a2 = __ldg(part + (b + 16) * stride + i), a3 = __ldg(part + (b + 24) * stride + i);
+            x += (double)a0; x += (double)a1; x += (double)a2; x += (double)a3;
+        }
+        for (; b < nsplit; b += 8) x += (double)__ldg(part + b * stride + i);
+    }
+    red[w][lane] = x;
+    __syncthreads();
+    if (w == 0 && i < n) {
+        double y = 0.0;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) y += red[k][lane];
+        out[(i / nc) * ldo + (i % nc)] = (float)y;
+    }
+}
+
+void reduce_splits(const float* part, int64_t nsplit, int64_t stride, int64_t n, int64_t nc, int64_t ldo, float* out,
+                   cudaStream_t s) {
+    if (n <= 0) return;
+    k_reduce_splits<<<(unsigned)((n + 31) / 32), 256, 0, s>>>(part, nsplit, stride, n, nc, ldo, out);
 }
 
 seastar_status colsum_impl(const float* X, int64_t M, int64_t F, int64_t ld, float* out, void* ws, size_t ws_bytes,
@@ -56,7 +79,7 @@ seastar_status colsum_impl(const float* X, int64_t M, int64_t F, int64_t ld, flo
     const int64_t rpb = M > 0 ? (M + nblk - 1) / nblk : 1;
     float* part = static_cast<float*>(ws);
     k_colsum1<<<(unsigned)nblk, 256, 0, s>>>(X, M, F, ld, rpb, part);
-    k_colsum2<<<(unsigned)((F + 255) / 256), 256, 0, s>>>(part, nblk, F, out);
+    reduce_splits(part, nblk, F, F, F, F, out, s);
     return check_launch("k_colsum");
 }
 
@@ -70,19 +93,43 @@ __global__ void __launch_bounds__(256) k_softmax_xent(const float* __restrict__ 
     float loss = 0.f;
     if (r < M) {
         const float* z = Z + r * ldz;
-        float m = -INFINITY;
-        for (int c = lane; c < C; c += 32) m = fmaxf(m, __ldg(z + c));
-        for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
-        float sum = 0.f;
-        for (int c = lane; c < C; c += 32) sum += expf(__ldg(z + c) - m);
-        for (int o = 16; o; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
-        const float lse = m + logf(sum);
         const int64_t lab = labels[r];
         const float inv = 1.f / (float)n_total;
-        if (dZ)
-            for (int c = lane; c < C; c += 32)
-                dZ[r * lddz + c] = (expf(__ldg(z + c) - lse) - (c == lab ? 1.f : 0.f)) * inv;
-        loss = lse - __ldg(z + lab);
+        if (C <= 128) {                       // the row stays in registers: one coalesced read
+            float zv[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) zv[k] = (lane + 32 * k < C) ? __ldg(z + lane + 32 * k) : -INFINITY;
+            float m = fmaxf(fmaxf(zv[0], zv[1]), fmaxf(zv[2], zv[3]));
+            for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+            float sum = 0.f;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) sum += (lane + 32 * k < C) ? expf(zv[k] - m) : 0.f;
+            for (int o = 16; o; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+            const float lse = m + logf(sum);
+            float zl = 0.f;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const int c = lane + 32 * k;
+                if (c < C) {
+                    if (dZ) dZ[r * lddz + c] = (expf(zv[k] - lse) - (c == lab ? 1.f : 0.f)) * inv;
+                    if (c == lab) zl = zv[k];
+                }
+            }
+            for (int o = 16; o; o >>= 1) zl += __shfl_xor_sync(0xffffffffu, zl, o);
+            loss = lse - zl;
+        } else {
+            float m = -INFINITY;
+            for (int c = lane; c < C; c += 32) m = fmaxf(m, __ldg(z + c));
+            for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+            float sum = 0.f;
+            for (int c = lane; c < C; c += 32) sum += expf(__ldg(z + c) - m);
+            for (int o = 16; o; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+            const float lse = m + logf(sum);
+            if (dZ)
+                for (int c = lane; c < C; c += 32)
+                    dZ[r * lddz + c] = (expf(__ldg(z + c) - lse) - (c == lab ? 1.f : 0.f)) * inv;
+            loss = lse - __ldg(z + lab);
+        }
     }
     if (lane == 0) wl[w] = loss;
     __syncthreads();
