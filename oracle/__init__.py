@@ -21,6 +21,8 @@ appnp_fwd/bwd              Z <- (1-a) n A n Z + a H0, K steps                   
 gat_attn_proj(_bwd)        e_u = f_u^T attn_u                                    Fig.2 L95-107
 gat_fwd / gat_bwd          LeakyReLU -> edge softmax -> weighted sum            Fig.2, Fig.3
 rgcn_norm/fwd/bwd          sum_r sum_{u in N_r(v)} 1/c_{v,r} h_u W_r           L465-475, [53]
+rgcn_basis_fwd/bwd         featureless input, W_r = sum_b a_rb V_b (NEXT-2)      L485, L1219-1227, [53]
+basis_combine(_bwd)        W_r = sum_b a_rb V_b for a dense layer (NEXT-2)       [53] (reading #27)
 softmax_xent, adam         DGL default training loop                             L481
 =========================  ===================================================  ==================
 
@@ -78,6 +80,8 @@ def _L():
             "orc_rgcn_norm": ([_I, _I, _P, _P, ctypes.c_int32, _P], None),
             "orc_rgcn_fwd": ([_I, _I, _P, _P, _P, _I, _I, _P, _P, _P, _P, _I, _P], None),
             "orc_rgcn_bwd": ([_I, _I, _P, _P, _P, ctypes.c_int32, _I, _I, _P, _P, _P, _P, _P, _P], None),
+            "orc_rgcn_basis_fwd": ([_I, _I, _P, _P, _P, _I, _I, _P, _P, _P, _P, _I, _P], None),
+            "orc_rgcn_basis_bwd": ([_I, _I, _P, _P, _P, ctypes.c_int32, _I, _I, _P, _P, _P, _P, _P, _P], None),
             "orc_softmax_xent": ([_I, _I, _P, _P, _P], _D),
             "orc_adam": ([_I, _P, _P, _P, _P, _D, _D, _D, _D, _I], None),
         }
@@ -350,6 +354,62 @@ def rgcn_bwd(indptr, indices, etypes, X, W, dA, norm=None, need_dX=True, need_dW
     _L().orc_rgcn_bwd(N, int(indptr[-1]), _p(indptr), _p(indices), _p(etypes), R, Fin, Fout, _p(X), _p(W),
                       _p(norm), _p(dA), _p(dX), _p(dW))
     return dX, dW
+
+
+# ------------------------------------------------------------------------------------------
+# NEXT-2: R-GCN with featureless input and basis decomposition (reading #27)
+# ------------------------------------------------------------------------------------------
+def rgcn_basis_fwd(indptr, indices, etypes, V, a, norm=None, rows=None):
+    """sum_{e in in(v)} norm_e sum_b a[type_e, b] V[src_e, b, :] ; V is [N, B, F], a is [R, B]."""
+    indptr, indices, etypes, V, a = _i64(indptr), _i64(indices), _i32(etypes), _f64(V), _f64(a)
+    N = indptr.size - 1
+    R, B = a.shape
+    assert V.shape[:2] == (N, B), V.shape
+    F = V.shape[2]
+    norm = rgcn_norm(indptr, etypes, R) if norm is None else _f64(norm)
+    rows = _i64(rows)
+    nrows = N if rows is None else rows.size
+    out = np.empty((nrows, F))
+    _L().orc_rgcn_basis_fwd(N, int(indptr[-1]), _p(indptr), _p(indices), _p(etypes), B, F, _p(V), _p(a),
+                            _p(norm), _p(rows), nrows, _p(out))
+    return out
+
+
+def rgcn_basis_bwd(indptr, indices, etypes, V, a, dA, norm=None, need_dV=True, need_da=True):
+    indptr, indices, etypes, V, a, dA = (_i64(indptr), _i64(indices), _i32(etypes), _f64(V), _f64(a),
+                                         _f64(dA))
+    N = indptr.size - 1
+    R, B = a.shape
+    F = V.shape[2]
+    norm = rgcn_norm(indptr, etypes, R) if norm is None else _f64(norm)
+    dV = np.empty((N, B, F)) if need_dV else None
+    da = np.empty((R, B)) if need_da else None
+    _L().orc_rgcn_basis_bwd(N, int(indptr[-1]), _p(indptr), _p(indices), _p(etypes), R, B, F, _p(V), _p(a),
+                            _p(norm), _p(dA), _p(dV), _p(da))
+    return dV, da
+
+
+def basis_combine(a, Vb):
+    """W[r] = sum_b a[r,b] Vb[b]   (a [R,B], Vb [B,Fin,Fout] -> W [R,Fin,Fout]); [53] Eq. 3."""
+    a, Vb = _f64(a), _f64(Vb)
+    R, B = a.shape
+    W = np.zeros((R,) + Vb.shape[1:])
+    for r in range(R):
+        for b in range(B):
+            W[r] += a[r, b] * Vb[b]
+    return W
+
+
+def basis_combine_bwd(a, Vb, dW):
+    """VJP of basis_combine: da[r,b] = <dW[r], Vb[b]>, dVb[b] = sum_r a[r,b] dW[r]."""
+    a, Vb, dW = _f64(a), _f64(Vb), _f64(dW)
+    R, B = a.shape
+    da = np.array([[float((dW[r] * Vb[b]).sum()) for b in range(B)] for r in range(R)])
+    dVb = np.zeros_like(Vb)
+    for b in range(B):
+        for r in range(R):
+            dVb[b] += a[r, b] * dW[r]
+    return da, dVb
 
 
 # ------------------------------------------------------------------------------------------

@@ -543,6 +543,75 @@ void orc_rgcn_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* in
 }
 
 /* ------------------------------------------------------------------------------------------ */
+/* NEXT-2: R-GCN as the paper ran it (Table 2/3 L485, L1219-L1227: aifb / mutag / bgs with a     */
+/* featureless input layer).  Layer of [53] with basis decomposition (reading #27):              */
+/*   W_r = sum_b a[r,b] V_b ; featureless input h_u = one-hot(u) => h_u W_r = W_r[u,:]            */
+/* V is stored [N, B, F] (V[u,b,:] = row u of basis b), a is [R, B].                             */
+/* ------------------------------------------------------------------------------------------ */
+
+/* out[r,:] = sum_{e in in(v)} norm[e] * W_{type(e)}[src(e),:],  W_t[u,:] = sum_b a[t,b] V[u,b,:] */
+void orc_rgcn_basis_fwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices,
+                        const int32_t* etypes, int64_t B, int64_t F, const double* V, const double* a,
+                        const double* norm, const int64_t* rows, int64_t nrows, double* out) {
+    (void)E;
+    if (!rows) nrows = N;
+    #pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t r = 0; r < nrows; ++r) {
+        int64_t v = rows ? rows[r] : r;
+        double* o = out + r * F;
+        for (int64_t f = 0; f < F; ++f) o[f] = 0.0;
+        for (int64_t e = indptr[v]; e < indptr[v + 1]; ++e) {
+            int64_t u = indices[e], t = etypes[e];
+            for (int64_t f = 0; f < F; ++f) {
+                double w = 0.0;                               /* W_t[u,f] */
+                for (int64_t b = 0; b < B; ++b) w += a[t * B + b] * V[(u * B + b) * F + f];
+                o[f] += norm[e] * w;
+            }
+        }
+    }
+}
+
+/* VJP of orc_rgcn_basis_fwd given dA = dL/d out (all N rows):
+ *   dV[u,b,:] = sum_{e in out(u)} norm[e] a[type(e),b] dA[dst(e),:]
+ *   da[t,b]   = sum_{e : type(e) = t} norm[e] <V[src(e),b,:], dA[dst(e),:]>      (both optional) */
+void orc_rgcn_basis_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices,
+                        const int32_t* etypes, int32_t R, int64_t B, int64_t F, const double* V,
+                        const double* a, const double* norm, const double* dA, double* dV, double* da) {
+    int64_t* dst = dst_of_edges(N, E, indptr);
+    if (dV) {
+        int64_t *optr, *oeid;
+        out_adjacency(N, E, indices, &optr, &oeid);
+        #pragma omp parallel for schedule(dynamic, 64)
+        for (int64_t u = 0; u < N; ++u) {
+            double* o = dV + u * B * F;
+            for (int64_t k = 0; k < B * F; ++k) o[k] = 0.0;
+            for (int64_t p = optr[u]; p < optr[u + 1]; ++p) {
+                int64_t e = oeid[p], v = dst[e], t = etypes[e];
+                for (int64_t b = 0; b < B; ++b)
+                    for (int64_t f = 0; f < F; ++f) o[b * F + f] += norm[e] * a[t * B + b] * dA[v * F + f];
+            }
+        }
+        free(optr); free(oeid);
+    }
+    if (da) {
+        #pragma omp parallel for schedule(dynamic, 1)
+        for (int32_t t = 0; t < R; ++t) {
+            for (int64_t b = 0; b < B; ++b) da[(int64_t)t * B + b] = 0.0;
+            for (int64_t e = 0; e < E; ++e) {
+                if (etypes[e] != t) continue;
+                int64_t u = indices[e], v = dst[e];
+                for (int64_t b = 0; b < B; ++b) {
+                    double d = 0.0;
+                    for (int64_t f = 0; f < F; ++f) d += V[(u * B + b) * F + f] * dA[v * F + f];
+                    da[(int64_t)t * B + b] += norm[e] * d;
+                }
+            }
+        }
+    }
+    free(dst);
+}
+
+/* ------------------------------------------------------------------------------------------ */
 /* training-step pieces around the hot path (DGL default training loop)         */
 /* ------------------------------------------------------------------------------------------ */
 
