@@ -302,6 +302,51 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
 size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out);
 
 /* ------------------------------------------------------------------------------------------ */
+/* NEXT-2: R-GCN as the paper ran it -- featureless input layer, basis decomposition            */
+/* (Table 2 L485 / Table 3 L1219-L1227 aifb, mutag, bgs; layer of [53]; DESIGN.md      */
+/* reading #26).  W_r = sum_b a[r,b] V_b ; featureless h_u = one-hot(u) => h_u W_r = sum_b a[r,b] V[u,b,:]. */
+/* ------------------------------------------------------------------------------------------ */
+/*
+ * Y[v] = act( sum_{e in in(v)} norm_e sum_b a[type(e),b] V_all[src(e), b*F : b*F+F] + loop[v] + bias )
+ *   V_all [N, B*F] ld ldv (dev; row u = the B basis rows of vertex u, basis-major; gathered by source
+ *   id, so a partitioned caller all-gathers it) ; a [R, B] (dev) ; norm_user [E] by user edge id or NULL
+ *   = the graph's 1/c_{v,r} ; loop_loc [n_loc, F] ld ldl or NULL (self-loop addend, e.g. W_0[v] of a
+ *   featureless self-loop) ; bias [F] or NULL ; Y_loc [n_loc, F] ld ldy.
+ *   F a power of two in [4, 128]; B*F <= 2048; R*B*4 <= 96 KB; ldv, ldy multiples of 4, pointers 16B aligned.
+ *   One warp per destination row, no atomics (bitwise deterministic).
+ */
+seastar_status seastar_rgcn_basis_fwd(seastar_graph g, const float* V_all, int64_t B, int64_t F, int64_t ldv,
+                                      const float* a, const float* norm_user, const float* loop_loc, int64_t ldl,
+                                      const float* bias, seastar_act act, float* Y_loc, int64_t ldy,
+                                      seastar_stream stream);
+/*
+ * VJP of seastar_rgcn_basis_fwd's pre-activation output given dA_all = dL/d(pre-activation) [N, F] ld ldd
+ * (gathered by destination id):
+ *   dV_loc[u, b*F + f] = sum_{e in out(u)} norm_e a[type(e),b] dA_all[dst(e), f]   (owned sources u;
+ *     source-major over the reverse CSR, no atomics) -- NULL to skip ;
+ *   da[r, b] = sum_{e: type(e)=r} norm_e <V_all[src(e), b*F : b*F+F], dA_all[dst(e), :]>  (over the
+ *     type-major view built at graph_create; per-task partials reduced per type in task order in
+ *     fp64; this rank's partial when partitioned) -- NULL to skip.
+ *   The self-loop and bias gradients are dA itself and its column sum (the caller's).
+ *   dV_loc [n_loc, B*F] ld ldv ; workspace: seastar_rgcn_basis_bwd_workspace() bytes when da != NULL.
+ */
+seastar_status seastar_rgcn_basis_bwd(seastar_graph g, const float* V_all, int64_t B, int64_t F, int64_t ldv,
+                                      const float* a, const float* norm_user, const float* dA_all, int64_t ldd,
+                                      float* dV_loc, float* da, void* workspace, size_t ws_bytes,
+                                      seastar_stream stream);
+size_t seastar_rgcn_basis_bwd_workspace(seastar_graph g, int64_t B);
+/*
+ * Basis combination for a dense R-GCN layer: W[r, k] = sum_b a[r,b] Vb[b, k] for k < K
+ * (a [R,B], Vb [B,K], W [R,K], all dev, contiguous; K = F_in*F_out of seastar_rgcn_fwd's W).
+ * fp64 accumulation in a fixed order.
+ */
+seastar_status seastar_basis_combine(const float* a, const float* Vb, int32_t R, int32_t B, int64_t K, float* W,
+                                     seastar_stream stream);
+/* its VJP: da[r,b] = <dW[r,:], Vb[b,:]>, dVb[b,k] = sum_r a[r,b] dW[r,k]; either output may be NULL */
+seastar_status seastar_basis_combine_bwd(const float* a, const float* Vb, const float* dW, int32_t R, int32_t B,
+                                         int64_t K, float* da, float* dVb, seastar_stream stream);
+
+/* ------------------------------------------------------------------------------------------ */
 /* training-step glue kept on the GPU (DGL default loop)                         */
 /* ------------------------------------------------------------------------------------------ */
 /*

@@ -98,3 +98,19 @@ def rgcn2(ip, ix, et, X, lab, p, acts=None):
     if acts is not None:
         acts.update(H1=H1, logits=Z2, Z1=Z1, dH1=dH1)
     return loss, {"W1": dW1, "b1": dZ1.sum(0), "W2": dW2, "b2": db2}
+
+
+def rgcnb2(ip, ix, et, lab, p, acts=None):
+    """NEXT-2 R-GCN (featureless input layer with bases, dense basis output layer; reading #26)."""
+    Z1 = oracle.rgcn_basis_fwd(ip, ix, et, p["V1"], p["a1"]) + p["b1"]
+    H1 = oracle.act_fwd("relu", Z1)
+    W2 = oracle.basis_combine(p["a2"], p["V2"])
+    Z2 = oracle.rgcn_fwd(ip, ix, et, H1, W2) + p["b2"]
+    loss, dZ2 = oracle.softmax_xent(Z2, lab)
+    dH1, dW2 = oracle.rgcn_bwd(ip, ix, et, H1, W2, dZ2)
+    da2, dV2 = oracle.basis_combine_bwd(p["a2"], p["V2"], dW2)
+    dZ1 = oracle.act_bwd("relu", Z1, dH1)
+    dV1, da1 = oracle.rgcn_basis_bwd(ip, ix, et, p["V1"], p["a1"], dZ1)
+    if acts is not None:
+        acts.update(H1=H1, logits=Z2, Z1=Z1, dH1=dH1)
+    return loss, {"V1": dV1, "a1": da1, "b1": dZ1.sum(0), "V2": dV2, "a2": da2, "b2": dZ2.sum(0)}

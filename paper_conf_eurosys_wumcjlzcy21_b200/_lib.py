@@ -77,6 +77,11 @@ _SIGS = {
     "seastar_rgcn_fwd": ([_P, _P, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
     "seastar_rgcn_bwd": ([_P, _P, _I64, _I64, _P, _I64, _I64, _P, _P, _P, _I32, _P, _P, _P, _SZ, _P], _ST),
     "seastar_rgcn_bwd_workspace": ([_P, _I64, _I64], _SZ),
+    "seastar_rgcn_basis_fwd": ([_P, _P, _I64, _I64, _I64, _P, _P, _P, _I64, _P, _I32, _P, _I64, _P], _ST),
+    "seastar_rgcn_basis_bwd": ([_P, _P, _I64, _I64, _I64, _P, _P, _P, _I64, _P, _P, _P, _SZ, _P], _ST),
+    "seastar_rgcn_basis_bwd_workspace": ([_P, _I64], _SZ),
+    "seastar_basis_combine": ([_P, _P, _I32, _I32, _I64, _P, _P], _ST),
+    "seastar_basis_combine_bwd": ([_P, _P, _P, _I32, _I32, _I64, _P, _P, _P], _ST),
     "seastar_softmax_xent": ([_P, _I64, _I64, _I32, _I64, _P, _P, _P, _I64, _P, _SZ, _P], _ST),
     "seastar_softmax_xent_workspace": ([_I64], _SZ),
     "seastar_colsum": ([_P, _I64, _I64, _I64, _P, _P, _SZ, _P], _ST),
@@ -298,6 +303,33 @@ def seastar_rgcn_bwd(g, X_all, F_in, ldx, dA_all, F_out, ldd, W, norm_user, Yact
     _call("seastar_rgcn_bwd", g, _dptr(X_all, "X"), F_in, ldx, _dptr(dA_all, "dA"), F_out, ldd, _dptr(W, "W"),
           _dptr(norm_user, "norm"), _dptr(Yact_loc, "Yact"), _act(act), _dptr(dX_loc, "dX"), _dptr(dW, "dW"),
           _dptr(workspace, "workspace"), ws_bytes, _stream(stream))
+
+
+# ----------------------------------------------------------------------------------- R-GCN, featureless + bases (NEXT-2)
+def seastar_rgcn_basis_fwd(g, V_all, B, F, ldv, a, norm_user, loop_loc, ldl, bias, act, Y_loc, ldy,
+                           stream=None) -> None:
+    _call("seastar_rgcn_basis_fwd", g, _dptr(V_all, "V"), B, F, ldv, _dptr(a, "a"), _dptr(norm_user, "norm"),
+          _dptr(loop_loc, "loop"), ldl, _dptr(bias, "bias"), _act(act), _dptr(Y_loc, "Y"), ldy, _stream(stream))
+
+
+def seastar_rgcn_basis_bwd_workspace(g, B) -> int:
+    return int(load().seastar_rgcn_basis_bwd_workspace(g, B))
+
+
+def seastar_rgcn_basis_bwd(g, V_all, B, F, ldv, a, norm_user, dA_all, ldd, dV_loc, da, workspace, ws_bytes,
+                           stream=None) -> None:
+    _call("seastar_rgcn_basis_bwd", g, _dptr(V_all, "V"), B, F, ldv, _dptr(a, "a"), _dptr(norm_user, "norm"),
+          _dptr(dA_all, "dA"), ldd, _dptr(dV_loc, "dV"), _dptr(da, "da"), _dptr(workspace, "workspace"), ws_bytes,
+          _stream(stream))
+
+
+def seastar_basis_combine(a, Vb, R, B, K, W, stream=None) -> None:
+    _call("seastar_basis_combine", _dptr(a, "a"), _dptr(Vb, "Vb"), R, B, K, _dptr(W, "W"), _stream(stream))
+
+
+def seastar_basis_combine_bwd(a, Vb, dW, R, B, K, da, dVb, stream=None) -> None:
+    _call("seastar_basis_combine_bwd", _dptr(a, "a"), _dptr(Vb, "Vb"), _dptr(dW, "dW"), R, B, K, _dptr(da, "da"),
+          _dptr(dVb, "dVb"), _stream(stream))
 
 
 # ----------------------------------------------------------------------------------- glue

@@ -176,6 +176,11 @@ size_t l2_persist_bytes();
 void reduce_splits(const float* part, int64_t nsplit, int64_t stride, int64_t n, int64_t nc, int64_t ldo, float* out,
                    cudaStream_t s);   // device set-aside for persisting lines (configured on first use), 0 if none
 
+// out[s * width + e] = sum_{t in [seg_off[s], seg_off[s+1])} part[t * width + e] for s < nseg, e < width:
+// deterministic fp64 segmented column sums (fixed task-to-thread assignment and merge order), one
+// block per (segment, 32 columns).  Used for the per-type reduction of R-GCN task partials.
+void seg_reduce_cols(const float* part, const int32_t* seg_off, int nseg, int width, float* out, cudaStream_t s);
+
 template <typename... KArgs, typename... Args>
 inline void launch_k(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
     cudaLaunchConfig_t cfg = {};

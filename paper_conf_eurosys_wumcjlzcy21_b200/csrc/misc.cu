@@ -158,19 +158,42 @@ __global__ void k_axpby(int64_t n, float a, const float* __restrict__ x, float b
     if (i < n) y[i] = a * x[i] + (b == 0.f ? 0.f : b * y[i]);
 }
 
-__global__ void k_adam(float* __restrict__ p, const float* __restrict__ g, float* __restrict__ m,
-                       float* __restrict__ v, int64_t n, float lr, float b1, float b2, float eps,
-                       const int32_t* __restrict__ step) {
-    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (i >= n) return;
+__device__ __forceinline__ void adam1(float& p, float g, float& m, float& v, float lr, float b1, float b2, float eps,
+                                      float c1, float c2) {
+    m = b1 * m + (1.f - b1) * g;
+    v = b2 * v + (1.f - b2) * g * g;
+    p -= lr * (m / c1) / (sqrtf(v / c2) + eps);
+}
+
+// grid-stride, 128-bit accesses (7 x 16 B per 4 parameters); the bias corrections are computed once per thread
+__global__ void __launch_bounds__(256) k_adam(float* __restrict__ p, const float* __restrict__ g, float* __restrict__ m,
+                                              float* __restrict__ v, int64_t n, float lr, float b1, float b2, float eps,
+                                              const int32_t* __restrict__ step, int vec) {
     const int t = *step;
     const float c1 = 1.f - powf(b1, (float)t), c2 = 1.f - powf(b2, (float)t);
-    const float gi = g[i];
-    const float mi = b1 * m[i] + (1.f - b1) * gi;
-    const float vi = b2 * v[i] + (1.f - b2) * gi * gi;
-    m[i] = mi;
-    v[i] = vi;
-    p[i] -= lr * (mi / c1) / (sqrtf(vi / c2) + eps);
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t i0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    int64_t done = 0;
+    if (vec) {
+        const int64_t n4 = n >> 2;
+        float4* p4 = reinterpret_cast<float4*>(p);
+        float4* m4 = reinterpret_cast<float4*>(m);
+        float4* v4 = reinterpret_cast<float4*>(v);
+        const float4* g4 = reinterpret_cast<const float4*>(g);
+        for (int64_t i = i0; i < n4; i += stride) {
+            float4 pp = p4[i], mm = m4[i], vv = v4[i];
+            const float4 gg = __ldcs(g4 + i);
+            adam1(pp.x, gg.x, mm.x, vv.x, lr, b1, b2, eps, c1, c2);
+            adam1(pp.y, gg.y, mm.y, vv.y, lr, b1, b2, eps, c1, c2);
+            adam1(pp.z, gg.z, mm.z, vv.z, lr, b1, b2, eps, c1, c2);
+            adam1(pp.w, gg.w, mm.w, vv.w, lr, b1, b2, eps, c1, c2);
+            p4[i] = pp;
+            __stcs(m4 + i, mm);
+            __stcs(v4 + i, vv);
+        }
+        done = n4 << 2;
+    }
+    for (int64_t i = done + i0; i < n; i += stride) adam1(p[i], g[i], m[i], v[i], lr, b1, b2, eps, c1, c2);
 }
 
 __global__ void k_step_inc(int32_t* c) { *c += 1; }
@@ -222,8 +245,12 @@ seastar_status seastar_adam(float* param, const float* grad, float* m, float* v,
     SS_ARG(param && grad && m && v && step && n >= 0, "adam: bad argument");
     SS_TRY(check_device());
     if (n == 0) return SEASTAR_OK;
-    k_adam<<<(unsigned)((n + 255) / 256), 256, 0, to_stream(stream)>>>(param, grad, m, v, n, lr, beta1, beta2, eps,
-                                                                        step);
+    const int vec = aligned16(param) && aligned16(grad) && aligned16(m) && aligned16(v);
+    int64_t blocks = ((vec ? (n + 3) / 4 : n) + 255) / 256;
+    const int64_t cap = 8 * (int64_t)num_sms();
+    if (blocks > cap) blocks = cap;
+    if (blocks < 1) blocks = 1;
+    k_adam<<<(unsigned)blocks, 256, 0, to_stream(stream)>>>(param, grad, m, v, n, lr, beta1, beta2, eps, step, vec);
     return check_launch("k_adam");
 }
 

@@ -49,7 +49,10 @@ __device__ void stage_w(const RgcnRowArgs& a, float* Ws) {
     }
 }
 
-template <int L, int RL>
+// WPR = 1: RL lanes per row (rows of degree < 1024).  WPR > 1 (hub rows, degree >= 1024): one CTA of WPR
+// warps per row, warp w owns the contiguous edge slice w/WPR of the row (a type run cut at a slice border is
+// flushed through W_r by both warps -- linear, so exact), per-warp outputs merged in warp order.
+template <int L, int RL, int WPR>
 __global__ void __launch_bounds__(512) k_rgcn_rows(const RgcnRowArgs a) {
     extern __shared__ float4 smem4[];
     float* Ws = reinterpret_cast<float*>(smem4);
@@ -65,11 +68,20 @@ __global__ void __launch_bounds__(512) k_rgcn_rows(const RgcnRowArgs a) {
     const unsigned smask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << ((lane / L) * L));
     const int Fop = (a.Fo + 3) & ~3;
     const int Cg = (a.Fg + 3) / 4, Co = (a.Fo + 3) / 4;
-    const int gpb = blockDim.x / RL;
+    const int gpb = WPR > 1 ? 1 : blockDim.x / RL;
     const int64_t ngroups = (int64_t)gridDim.x * gpb;
+    const int warp = threadIdx.x >> 5;
+    __shared__ float red[WPR > 1 ? WPR : 1][64];
 
-    for (int64_t row = a.row_begin + (int64_t)blockIdx.x * gpb + threadIdx.x / RL; row < a.row_end; row += ngroups) {
-        const int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+    for (int64_t row = a.row_begin + (int64_t)blockIdx.x * gpb + (WPR > 1 ? 0 : threadIdx.x / RL); row < a.row_end;
+         row += ngroups) {
+        int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+        if (WPR > 1) {
+            const int64_t n = end - beg;
+            const int b0 = beg + (int)(n * warp / WPR);
+            end = beg + (int)(n * (warp + 1) / WPR);
+            beg = b0;
+        }
         const int64_t v = (int64_t)__ldg(a.perm + row) - a.vbase;
         float out[4] = {0.f, 0.f, 0.f, 0.f};
         float g[4] = {0.f, 0.f, 0.f, 0.f};
@@ -157,6 +169,21 @@ __global__ void __launch_bounds__(512) k_rgcn_rows(const RgcnRowArgs a) {
         for (int o = L; o < RL; o <<= 1)
 #pragma unroll
             for (int q = 0; q < 4; ++q) out[q] += __shfl_xor_sync(gmask, out[q], o, RL);
+        if (WPR > 1) {
+            if (slot == 0 && c < Co)
+#pragma unroll
+                for (int q = 0; q < 4; ++q) red[warp][4 * c + q] = out[q];
+            __syncthreads();
+            if (warp == 0 && slot == 0 && c < Co)
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    float t = red[0][4 * c + q];
+                    for (int w = 1; w < WPR; ++w) t += red[w][4 * c + q];
+                    out[q] = t;
+                }
+            __syncthreads();
+            if (warp != 0) continue;
+        }
         if (slot == 0 && c < Co) {
             float* po = a.out + v * a.ldo + 4 * c;
 #pragma unroll
@@ -182,100 +209,143 @@ struct RgcnDwArgs {
     float* part;
 };
 
-// warp per task: dW_r partial (Fin x Fout entries, NPL per lane) in registers
+// one CTA (8 warps) per task of one type: warp w owns the contiguous edge slice w/8 of the task (its first
+// run found by binary search over run_off; a run cut at a slice border contributes its two parts
+// g1 (x) dA_v + g2 (x) dA_v, which is exact), keeps its dW_r partial (Fin x Fout, NPL per lane) in registers,
+// and the 8 partials are summed in warp order into part[task] (deterministic, no atomics).
 template <int L, int NPL>
 __global__ void __launch_bounds__(256) k_rgcn_dw(const RgcnDwArgs a) {
-    constexpr int S = 32 / L;
-    __shared__ float sg[8][64];
-    __shared__ float sd[8][64];
+    constexpr int S = 32 / L, WARPS = 8;
+    __shared__ float sg[WARPS][64];
+    __shared__ float sd[WARPS][64];
+    extern __shared__ float red[];                 // [WARPS][Fin * Fout]
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int slot = lane / L, c = lane % L;
     const int Cg = (a.Fin + 3) / 4;
     const int FF = a.Fin * a.Fout;
-    const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t t = blockIdx.x * (int64_t)(blockDim.x >> 5) + w; t < a.n_tasks; t += nwarps) {
+    for (int64_t t = blockIdx.x; t < a.n_tasks; t += gridDim.x) {
         float acc[NPL];
 #pragma unroll
         for (int i = 0; i < NPL; ++i) acc[i] = 0.f;
         const int r0 = __ldg(a.task_run + t), r1 = __ldg(a.task_run + t + 1);
-        for (int run = r0; run < r1; ++run) {
-            const int es = __ldg(a.run_off + run), ee = __ldg(a.run_off + run + 1);
-            const int64_t v = __ldg(a.run_dst + run);
-            float g[4] = {0.f, 0.f, 0.f, 0.f};
-            for (int k = es + slot; k < ee; k += S) {
-                if (c < Cg) {
-                    const int u = __ldg(a.src + k);
-                    const float wgt = a.norm_user ? __ldg(a.norm_user + __ldg(a.eid + k)) : __ldg(a.norm + k);
-                    const float4 x = ldg4(a.X + (int64_t)u * a.ldx + 4 * c);
-                    g[0] = fmaf(wgt, x.x, g[0]); g[1] = fmaf(wgt, x.y, g[1]);
-                    g[2] = fmaf(wgt, x.z, g[2]); g[3] = fmaf(wgt, x.w, g[3]);
+        const int es = __ldg(a.run_off + r0), ee = __ldg(a.run_off + r1);
+        const int64_t n = ee - es;
+        const int k0 = es + (int)(n * w / WARPS), k1 = es + (int)(n * (w + 1) / WARPS);
+        if (k0 < k1) {
+            int lo = r0, hi = r1 - 1;                  // last run with run_off <= k0
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (__ldg(a.run_off + mid) <= k0) lo = mid; else hi = mid - 1;
+            }
+            int run = lo;
+            for (int k = k0; k < k1; ++run) {
+                const int rend = min(__ldg(a.run_off + run + 1), k1);
+                const int64_t v = __ldg(a.run_dst + run);
+                float g[4] = {0.f, 0.f, 0.f, 0.f};
+                for (int kk = k + slot; kk < rend; kk += S) {
+                    if (c < Cg) {
+                        const int u = __ldg(a.src + kk);
+                        const float wgt = a.norm_user ? __ldg(a.norm_user + __ldg(a.eid + kk)) : __ldg(a.norm + kk);
+                        const float4 x = ldg4(a.X + (int64_t)u * a.ldx + 4 * c);
+                        g[0] = fmaf(wgt, x.x, g[0]); g[1] = fmaf(wgt, x.y, g[1]);
+                        g[2] = fmaf(wgt, x.z, g[2]); g[3] = fmaf(wgt, x.w, g[3]);
+                    }
                 }
+#pragma unroll
+                for (int o = L; o < 32; o <<= 1)
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) g[q] += __shfl_xor_sync(0xffffffffu, g[q], o);
+                if (slot == 0 && c < Cg)
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        if (4 * c + q < a.Fin) sg[w][4 * c + q] = g[q];
+                for (int j = lane; j < a.Fout; j += 32) sd[w][j] = __ldg(a.dA + v * a.ldd + j);
+                __syncwarp();
+#pragma unroll
+                for (int i = 0; i < NPL; ++i) {
+                    const int e = lane + 32 * i;
+                    if (e < FF) acc[i] = fmaf(sg[w][e / a.Fout], sd[w][e % a.Fout], acc[i]);
+                }
+                __syncwarp();
+                k = rend;
             }
-#pragma unroll
-            for (int o = L; o < 32; o <<= 1)
-#pragma unroll
-                for (int q = 0; q < 4; ++q) g[q] += __shfl_xor_sync(0xffffffffu, g[q], o);
-            if (slot == 0 && c < Cg)
-#pragma unroll
-                for (int q = 0; q < 4; ++q)
-                    if (4 * c + q < a.Fin) sg[w][4 * c + q] = g[q];
-            for (int j = lane; j < a.Fout; j += 32) sd[w][j] = __ldg(a.dA + v * a.ldd + j);
-            __syncwarp();
-#pragma unroll
-            for (int i = 0; i < NPL; ++i) {
-                const int e = lane + 32 * i;
-                if (e < FF) acc[i] = fmaf(sg[w][e / a.Fout], sd[w][e % a.Fout], acc[i]);
-            }
-            __syncwarp();
         }
-        float* p = a.part + t * FF;
 #pragma unroll
         for (int i = 0; i < NPL; ++i) {
             const int e = lane + 32 * i;
-            if (e < FF) p[e] = acc[i];
+            if (e < FF) red[w * FF + e] = acc[i];
         }
+        __syncthreads();
+        for (int e = threadIdx.x; e < FF; e += blockDim.x) {
+            float x = red[e];
+#pragma unroll
+            for (int w2 = 1; w2 < WARPS; ++w2) x += red[w2 * FF + e];
+            a.part[t * FF + e] = x;
+        }
+        __syncthreads();
     }
 }
 
-// dW[r][e] = sum over the tasks of type r (task order) of part[task][e]
-__global__ void k_rgcn_dw_reduce(const float* __restrict__ part, const int32_t* __restrict__ type_task, int R, int FF,
-                                 float* __restrict__ dW) {
-    const int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (idx >= (int64_t)R * FF) return;
-    const int r = (int)(idx / FF), e = (int)(idx % FF);
-    float x = 0.f;
-    for (int t = type_task[r]; t < type_task[r + 1]; ++t) x += part[(int64_t)t * FF + e];
-    dW[idx] = x;
+__global__ void __launch_bounds__(256) k_seg_reduce_cols(const float* __restrict__ part,
+                                                          const int32_t* __restrict__ seg_off, int width,
+                                                          float* __restrict__ out) {
+    __shared__ double red[8][32];
+    const int sgi = blockIdx.y, lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int e = blockIdx.x * 32 + lane;
+    const int t0 = __ldg(seg_off + sgi), t1 = __ldg(seg_off + sgi + 1);
+    double x = 0.0;
+    if (e < width) {
+#pragma unroll 4
+        for (int t = t0 + w; t < t1; t += 8) x += (double)__ldg(part + (int64_t)t * width + e);
+    }
+    red[w][lane] = x;
+    __syncthreads();
+    if (w == 0 && e < width) {
+        double y = red[0][lane];
+#pragma unroll
+        for (int k = 1; k < 8; ++k) y += red[k][lane];
+        out[(int64_t)sgi * width + e] = (float)y;
+    }
 }
 
-template <int L, int RL>
+void seg_reduce_cols(const float* part, const int32_t* seg_off, int nseg, int width, float* out, cudaStream_t s) {
+    if (nseg <= 0 || width <= 0) return;
+    k_seg_reduce_cols<<<dim3((unsigned)((width + 31) / 32), (unsigned)nseg), 256, 0, s>>>(part, seg_off, width, out);
+}
+
+template <int L, int RL, int WPR = 1>
 static seastar_status launch_rows(const RgcnRowArgs& a, size_t smem, cudaStream_t s) {
     if (a.row_end <= a.row_begin) return SEASTAR_OK;
     static bool attr_set = false;
     if (!attr_set) {
-        SS_CUDA(cudaFuncSetAttribute(k_rgcn_rows<L, RL>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+        SS_CUDA(cudaFuncSetAttribute(k_rgcn_rows<L, RL, WPR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     227 * 1024 - (int)sizeof(float) * 64 * WPR));
         attr_set = true;
     }
     int per_sm = 0;
-    SS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rgcn_rows<L, RL>, 512, smem));
+    SS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rgcn_rows<L, RL, WPR>, 512, smem));
     if (per_sm < 1) {
         set_error("rgcn: W (%zu bytes) does not fit in shared memory", smem);
         return SEASTAR_ERR_UNSUPPORTED;
     }
     const int64_t groups = a.row_end - a.row_begin;
     int64_t blocks = (int64_t)per_sm * num_sms();
-    const int64_t need = (groups + (512 / RL) - 1) / (512 / RL);
+    const int gpb = WPR > 1 ? 1 : 512 / RL;
+    const int64_t need = (groups + gpb - 1) / gpb;
     if (blocks > need) blocks = need;
-    launch_k(k_rgcn_rows<L, RL>, dim3((unsigned)blocks), dim3(512), smem, s, a);
+    launch_k(k_rgcn_rows<L, RL, WPR>, dim3((unsigned)blocks), dim3(512), smem, s, a);
     return check_launch("k_rgcn_rows");
 }
 
 template <int L>
 static seastar_status launch_buckets(const IndexSet& x, RgcnRowArgs a, size_t smem, cudaStream_t s) {
+    const int64_t hub = x.bucket_rows[0];     // degree >= 1024: a 16-warp CTA per row
     const int64_t split = x.bucket_rows[1];   // rows with degree >= 32 get a warp with 32/L slots
-    RgcnRowArgs hi = a, lo = a;
-    hi.row_begin = 0; hi.row_end = split;
+    RgcnRowArgs hb = a, hi = a, lo = a;
+    hb.row_begin = 0; hb.row_end = hub;
+    hi.row_begin = hub; hi.row_end = split;
     lo.row_begin = split; lo.row_end = x.n_rows;
+    SS_TRY((launch_rows<L, 32, 16>(hb, smem, s)));
     SS_TRY((launch_rows<L, 32>(hi, smem, s)));
     constexpr int RLo = L < 4 ? 4 : L;
     return launch_rows<L, RLo>(lo, smem, s);
@@ -363,13 +433,19 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
             d.X = X_all; d.ldx = ldx; d.dA = dA_all; d.ldd = ldd; d.Fin = (int)F_in; d.Fout = (int)F_out;
             d.part = static_cast<float*>(workspace);
             ScopedL2Window win(X_all, (size_t)g->N * ldx * sizeof(float));
-            int64_t blocks = (g->tm.n_tasks + 7) / 8;
-            const int64_t cap = 16 * (int64_t)num_sms();
-            if (blocks > cap) blocks = cap;
             const int Cg = (int)((F_in + 3) / 4);
             const int L = pow2_ceil(Cg);
             const int npl = pow2_ceil((FF + 31) / 32);
-#define RGCN_DW(LL, NN) launch_k(k_rgcn_dw<LL, NN>, dim3((unsigned)blocks), dim3(256), 0, s, d)
+            const size_t smem_r = (size_t)8 * FF * sizeof(float);
+            int64_t blocks = 0;
+#define RGCN_DW(LL, NN)                                                                                  \
+    do {                                                                                                 \
+        int per_sm = 0;                                                                                  \
+        SS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rgcn_dw<LL, NN>, 256, smem_r)); \
+        blocks = (int64_t)(per_sm > 0 ? per_sm : 1) * num_sms();                                         \
+        if (blocks > g->tm.n_tasks) blocks = g->tm.n_tasks;                                              \
+        launch_k(k_rgcn_dw<LL, NN>, dim3((unsigned)blocks), dim3(256), smem_r, s, d);                    \
+    } while (0)
 #define RGCN_DW_L(LL)                                                   \
     switch (npl) {                                                      \
         case 1: RGCN_DW(LL, 1); break;                                  \
@@ -389,10 +465,8 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
 #undef RGCN_DW_L
 #undef RGCN_DW
             SS_TRY(check_launch("k_rgcn_dw"));
-            const int64_t n = (int64_t)g->R * FF;
-            k_rgcn_dw_reduce<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(static_cast<float*>(workspace),
-                                                                          g->tm.type_task, g->R, FF, dW);
-            SS_TRY(check_launch("k_rgcn_dw_reduce"));
+            seg_reduce_cols(static_cast<float*>(workspace), g->tm.type_task, g->R, FF, dW, s);
+            SS_TRY(check_launch("k_seg_reduce_cols"));
         } else {
             SS_CUDA(cudaMemsetAsync(dW, 0, sizeof(float) * (size_t)g->R * FF, s));
         }

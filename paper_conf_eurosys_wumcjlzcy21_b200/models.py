@@ -496,3 +496,124 @@ class RGCN2:
         self.backward()
         self.P.adam(self.lr)
         return loss
+
+
+class RGCNBasis2:
+    """2-layer R-GCN as the paper trained it on aifb / mutag / bgs (Table 2, Table 3
+    L1219-L1227; DGL's entity-classification defaults): a featureless input layer
+    h_u W_r = sum_b a1[r,b] V1[u,b,:] (ReLU), a dense output layer W2_r = sum_b a2[r,b] V2[b] (identity),
+    normaliser 1/c_{v,r}, no self-loop, softmax cross-entropy.  SURVEY.md §8(f) NEXT-2, reading #26.
+
+    Parameters: V1 [N, B1, Hd] (row-partitioned like the vertices: each rank owns and updates the rows of
+    its vertices, gathered for the forward; never all-reduced), a1 [R, B1], b1 [Hd], V2 [B2, Hd, C],
+    a2 [R, B2], b2 [C] (replicated, one flat all-reduced buffer)."""
+
+    def __init__(self, g: Graph, labels_loc, params: dict, lr=0.01, comm: Comm | None = None,
+                 n_pad_rows: int | None = None):
+        self.g, self.lab, self.lr = g, labels_loc, lr
+        self.comm = comm or Comm()
+        dev = labels_loc.device
+        self.n = g.n_loc
+        self.rows_all = n_pad_rows if n_pad_rows is not None else g.N
+        self.R, self.B1 = params["a1"].shape
+        self.B2, self.Hd, self.C = params["V2"].shape
+        Vn = params["V1"]
+        assert Vn.shape[1:] == (self.B1, self.Hd)
+        n = _local_rows(self)
+        self.ldv = self.B1 * self.Hd
+        V1_loc = np.zeros((n, self.B1, self.Hd), np.float32)     # padded rows stay 0 (never read)
+        if Vn.shape[0] == g.N:                                    # whole table given: take the owned rows
+            Vn = Vn[g.row_begin:g.row_begin + self.n]
+        assert Vn.shape[0] == self.n, "V1 must cover all N vertices or exactly the owned rows"
+        V1_loc[:self.n] = Vn
+        self.E = _Params({"V1": (n, self.ldv)}, {"V1": V1_loc.reshape(n, self.ldv)}, dev)
+        shp = {"a1": params["a1"].shape, "b1": (self.Hd,), "V2": params["V2"].shape, "a2": params["a2"].shape,
+               "b2": (self.C,)}
+        self.P = _Params(shp, {k: params[k] for k in shp}, dev)
+        self.ldh, self.ldc = _ld(self.Hd), _ld(self.C)
+        e = lambda r, c: torch.zeros((r, c), device=dev)
+        self.H1, self.dZ1 = e(n, self.ldh), e(n, self.ldh)
+        self.logits, self.dlog = e(n, self.ldc), e(n, self.ldc)
+        self.W2 = torch.zeros((self.R, self.Hd, self.C), device=dev)
+        self.dW2 = torch.zeros_like(self.W2)
+        self.loss = torch.zeros(1, device=dev)
+        self.ws = _Ws(dev)
+        P, Ra = self.comm.world, self.rows_all
+        self.V1_all = e(Ra, self.ldv) if P > 1 else None
+        self.H1_all = e(Ra, self.ldh) if P > 1 else None
+        self.dlog_all = e(Ra, self.ldc) if P > 1 else None
+        self.dZ1_all = e(Ra, self.ldh) if P > 1 else None
+        self.timer = None
+
+    def _t(self, name):
+        if self.timer is not None:
+            self.timer(name)
+
+    def grad(self, k):
+        return self.E.g(k)[:self.n].reshape(self.n, self.B1, self.Hd) if k == "V1" else self.P.g(k)
+
+    def param(self, k):
+        return self.E.p(k)[:self.n].reshape(self.n, self.B1, self.Hd) if k == "V1" else self.P.p(k)
+
+    def forward(self):
+        g, p, n = self.g, self.P, self.n
+        self._V1_all = self.comm.all_gather(self.V1_all, self.E.p("V1"))
+        self._t("rgcnb_fwd1")
+        L.seastar_rgcn_basis_fwd(g.handle, self._V1_all, self.B1, self.Hd, self.ldv, p.p("a1"), None, None, 0,
+                                 p.p("b1"), "relu", self.H1, self.ldh)
+        self._t("rgcnb_fwd1_end")
+        L.seastar_basis_combine(p.p("a2"), p.p("V2"), self.R, self.B2, self.Hd * self.C, self.W2)
+        self._H1_all = self.comm.all_gather(self.H1_all, self.H1)
+        L.seastar_rgcn_fwd(g.handle, self._H1_all, self.Hd, self.ldh, self.W2, self.C, None, p.p("b2"), "none",
+                           self.logits, self.ldc)
+        ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
+        L.seastar_softmax_xent(self.logits, n, self.g.N, self.C, self.ldc, self.lab, self.loss, self.dlog, self.ldc,
+                               ws, ws.numel())
+        return self.loss
+
+    def backward(self):
+        g, p, n = self.g, self.P, self.n
+        ws = self.ws.need(max(L.seastar_rgcn_bwd_workspace(g.handle, self.Hd, self.C),
+                              L.seastar_rgcn_basis_bwd_workspace(g.handle, self.B1),
+                              L.seastar_colsum_workspace(n, max(self.C, self.Hd))))
+        L.seastar_colsum(self.dlog, n, self.C, self.ldc, p.g("b2"), ws, ws.numel())
+        dlog_all = self.comm.all_gather(self.dlog_all, self.dlog)
+        L.seastar_rgcn_bwd(g.handle, self._H1_all, self.Hd, self.ldh, dlog_all, self.C, self.ldc, self.W2, None,
+                           self.H1, "relu", self.dZ1, self.dW2, ws, ws.numel())
+        L.seastar_basis_combine_bwd(p.p("a2"), p.p("V2"), self.dW2, self.R, self.B2, self.Hd * self.C, p.g("a2"),
+                                    p.g("V2"))
+        L.seastar_colsum(self.dZ1, n, self.Hd, self.ldh, p.g("b1"), ws, ws.numel())
+        dZ1_all = self.comm.all_gather(self.dZ1_all, self.dZ1)
+        self._t("rgcnb_bwd1")
+        L.seastar_rgcn_basis_bwd(g.handle, self._V1_all, self.B1, self.Hd, self.ldv, p.p("a1"), None, dZ1_all,
+                                 self.ldh, self.E.g("V1"), p.g("a1"), ws, ws.numel())
+        self._t("rgcnb_bwd1_end")
+        self.comm.all_reduce(self.P.grad)      # V1's gradient rows are owned: no reduction
+
+    def epoch(self):
+        loss = self.forward()
+        self.backward()
+        self.P.adam(self.lr)
+        self.E.adam(self.lr)
+        return loss
+
+
+class CapturedEpoch:
+    """One model's training epoch captured once in a CUDA graph and replayed (the launch-bound small
+    configs spend more time issuing ~20 C-ABI calls from Python than in the kernels).  Every call of an
+    epoch is stream-ordered and allocation-free once the model's buffers exist (seastar.h conventions),
+    so the captured graph is exactly the eager epoch; ``epoch()`` replays it and returns the model's
+    (static) loss tensor.  Run the eager epoch at least once before capturing (it sizes the workspaces)."""
+
+    def __init__(self, model):
+        self.model = model
+        self.graph = torch.cuda.CUDAGraph()
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.graph(self.graph, stream=s):
+            self.loss = model.epoch()
+        torch.cuda.current_stream().wait_stream(s)
+
+    def epoch(self):
+        self.graph.replay()
+        return self.loss

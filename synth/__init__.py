@@ -185,6 +185,15 @@ CONFIGS = {
     # configs[3]: R-GCN, AM-shaped (1.9M V, 5.7M E, 133 relations), dense synthetic X 16 -> 16 -> 11
     "am_rgcn": Config("am_rgcn", 1_900_000, 5_700_000, 0.60, 16, 16, 11, "rgcn", self_loops=False,
                       typed=True, R=133, zipf_a=1.0, cfg_id=4),
+    # NEXT-2: R-GCN as the paper ran it, Table 2 L485 shapes (aifb 8,285 V / 58,086 E /
+    # 90 relations; mutag 23,644 / 148,454 / 46; bgs 333,845 / 1,832,398 / 206), featureless input, hidden 16,
+    # DGL entity-classification defaults: bases = R (aifb), 30 (mutag), 40 (bgs); classes 4 / 2 / 2
+    "aifb_rgcnb": Config("aifb_rgcnb", 8285, 58086, 0.60, 0, 16, 4, "rgcnb", self_loops=False, typed=True, R=90,
+                         cfg_id=6, extra={"bases": 90}),
+    "mutag_rgcnb": Config("mutag_rgcnb", 23644, 148454, 0.60, 0, 16, 2, "rgcnb", self_loops=False, typed=True,
+                          R=46, cfg_id=7, extra={"bases": 30}),
+    "bgs_rgcnb": Config("bgs_rgcnb", 333845, 1832398, 0.60, 0, 16, 2, "rgcnb", self_loops=False, typed=True,
+                        R=206, cfg_id=8, extra={"bases": 40}),
     # configs[4]: GCN and GAT full-graph training, Reddit-shaped (232,965 V, 114,615,892 E incl. self-loops)
     "reddit": Config("reddit", 232_965, 114_615_892 - 232_965, 0.35, 602, 16, 41, "gcn+gat", heads=8,
                      cfg_id=5, extra={"gat_hidden": 8}),
@@ -234,4 +243,10 @@ def workload(name: str) -> dict:
         R, fin, hid, C = cfg.R, cfg.F_in, cfg.hidden, cfg.classes
         out["rgcn"] = {"W1": glorot(cfg.weight_seed(1), fin, hid, (R, fin, hid)), "b1": np.zeros(hid, np.float32),
                        "W2": glorot(cfg.weight_seed(2), hid, C, (R, hid, C)), "b2": np.zeros(C, np.float32)}
+    if "rgcnb" in models:
+        R, hid, C, B = cfg.R, cfg.hidden, cfg.classes, cfg.extra["bases"]
+        out["rgcnb"] = {"V1": glorot(cfg.weight_seed(1), cfg.N, hid, (cfg.N, B, hid)),
+                        "a1": glorot(cfg.weight_seed(2), R, B, (R, B)), "b1": np.zeros(hid, np.float32),
+                        "V2": glorot(cfg.weight_seed(3), hid, C, (B, hid, C)),
+                        "a2": glorot(cfg.weight_seed(4), R, B, (R, B)), "b2": np.zeros(C, np.float32)}
     return out

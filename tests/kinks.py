@@ -77,6 +77,22 @@ def relu_rgcn(ip, ix, et, R, X, Z1, dH1, shapes):
     return env, int(r.size)
 
 
+def relu_rgcnb(ip, ix, et, R, V1, a1, Z1, dH1, shapes):
+    """NEXT-2 featureless basis layer: flipping (r, j) adds dH1[r, j] * norm_e * a1[t_e, b] to dV1[src_e, b, j]
+    and dH1[r, j] * norm_e * V1[src_e, b, j] to da1[t_e, b] for every in-edge e of r."""
+    r, j = _ambiguous(Z1, np.diff(ip) == 0)
+    env = {k: np.zeros(s) for k, s in shapes.items()}
+    if r.size:
+        norm = oracle.rgcn_norm(ip, et, R)
+        w = np.abs(dH1[r, j])
+        np.add.at(env["b1"], j, w)
+        for k in range(r.size):
+            for e in range(ip[r[k]], ip[r[k] + 1]):
+                env["V1"][ix[e], :, j[k]] += w[k] * norm[e] * np.abs(a1[et[e]])
+                env["a1"][et[e], :] += w[k] * norm[e] * np.abs(V1[ix[e], :, j[k]])
+    return env, int(r.size)
+
+
 def gat_layer(ip, ix, L, H, F, slope=0.2, chunk=8_000_000):
     """Envelope for the flipped layer's own parameters (W, al, ar) from ambiguous edge scores."""
     el, er = L["el"], L["er"]

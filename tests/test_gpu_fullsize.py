@@ -70,8 +70,9 @@ def check_step(model, loss_ref, grads_ref, acts, envelope=None, n_ambiguous=0):
     for name, (got, ref) in acts.items():
         errs[name] = rel_err(got().cpu().numpy(), ref)
     excess, width = {}, {}
+    grad = getattr(model, "grad", model.P.g)
     for k, ref in grads_ref.items():
-        got = model.P.g(k).cpu().numpy().astype(np.float64)
+        got = grad(k).cpu().numpy().astype(np.float64)
         ref = ref.reshape(got.shape)
         errs["d" + k] = rel_err(got, ref)
         if k in envelope:
@@ -192,3 +193,21 @@ def test_am_rgcn2_step(env):
     loss, grads = model_ref.rgcn2(ip, ix, et, X, lab, f64(w["rgcn"]), acts)
     env, na = kinks.relu_rgcn(ip, ix, et, cfg.R, X, acts["Z1"], acts["dH1"], {k: grads[k].shape for k in ("W1", "b1")})
     check_step(m, loss, grads, {"H1": (lambda: m.H1[:, :cfg.hidden], acts["H1"])}, env, na)
+
+
+# ---------------------------------------------------------------------------------------------
+# NEXT-2: R-GCN as the paper ran it (featureless input, bases), Table 2 shapes
+# ---------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("name", ["aifb_rgcnb", "mutag_rgcnb", "bgs_rgcnb"])
+def test_rgcnb2_step(env, name):
+    w = workload(name)
+    ip, ix, et, lab = w["indptr"], w["indices"], w["etypes"], w["labels"]
+    cfg = w["cfg"]
+    g = env["Graph"](ip, ix, et, num_etypes=cfg.R, rgcn_norm=True)
+    m = env["models"].RGCNBasis2(g, env["torch"].from_numpy(lab).cuda(), w["rgcnb"])
+    acts = {}
+    p = f64(w["rgcnb"])
+    loss, grads = model_ref.rgcnb2(ip, ix, et, lab, p, acts)
+    envl, na = kinks.relu_rgcnb(ip, ix, et, cfg.R, p["V1"], p["a1"], acts["Z1"], acts["dH1"],
+                                {k: grads[k].shape for k in ("V1", "a1", "b1")})
+    check_step(m, loss, grads, {"H1": (lambda: m.H1[:, :cfg.hidden], acts["H1"])}, envl, na)

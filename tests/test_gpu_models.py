@@ -29,8 +29,9 @@ def check(model, loss_ref, grads_ref):
     loss = model.forward()
     model.backward()
     assert abs(loss.item() - loss_ref) <= TOL * abs(loss_ref)
+    grad = getattr(model, "grad", model.P.g)
     for k, ref in grads_ref.items():
-        got = model.P.g(k).cpu().numpy()
+        got = grad(k).cpu().numpy()
         assert rel_err(got, ref.reshape(got.shape)) <= TOL, k
 
 
@@ -78,3 +79,18 @@ def test_rgcn2(env):
     g = env["Graph"](ip, ix, et, num_etypes=R, rgcn_norm=True)
     m = env["models"].RGCN2(g, dev(env, X), dev(env, lab), p)
     check(m, *model_ref.rgcn2(ip, ix, et, X, lab, {k: v.astype(np.float64) for k, v in p.items()}))
+
+
+def test_rgcnb2(env):
+    """NEXT-2: featureless input layer with bases + dense basis output layer (aifb-like shape, B < R)."""
+    N, R, B1, B2, Hd, C = 2500, 30, 12, 6, 16, 4
+    ip, ix, et = synth.powerlaw_directed_typed(N, 18000, 0.6, 0.6, R, 1.0, 35)
+    lab = synth.labels(36, N, C)
+    p = {"V1": synth.uniform(37, (N, B1, Hd), -0.5, 0.5), "a1": synth.uniform(38, (R, B1)),
+         "b1": synth.uniform(39, (Hd,), -0.1, 0.1), "V2": synth.uniform(40, (B2, Hd, C), -0.5, 0.5),
+         "a2": synth.uniform(41, (R, B2)), "b2": synth.uniform(42, (C,), -0.1, 0.1)}
+    g = env["Graph"](ip, ix, et, num_etypes=R, rgcn_norm=True)
+    m = env["models"].RGCNBasis2(g, dev(env, lab), p)
+    check(m, *model_ref.rgcnb2(ip, ix, et, lab, {k: v.astype(np.float64) for k, v in p.items()}))
+    m.epoch()
+    assert not np.array_equal(m.param("V1").cpu().numpy(), p["V1"])

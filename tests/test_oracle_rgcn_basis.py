@@ -86,3 +86,21 @@ def test_basis_combine():
     f = lambda: (oracle.basis_combine(a, Vb) * dW).sum()
     assert rel_err(da, fd_grad(f, a)) < 1e-8
     assert rel_err(dVb, fd_grad(f, Vb)) < 1e-8
+
+
+def test_rgcnb2_model_fd():
+    """The NEXT-2 model composition (oracle/model_ref.rgcnb2): every gradient against central differences
+    of its loss."""
+    from oracle import model_ref
+    import synth
+    indptr, indices, et = small_graph(15, N=9, E=30, R=3)
+    N, R, B1, B2, Hd, C = 9, 3, 2, 2, 3, 2
+    lab = synth.labels(1, N, C)
+    p = {"V1": rnd(20, N, B1, Hd), "a1": rnd(21, R, B1), "b1": rnd(22, Hd) * 0.1, "V2": rnd(23, B2, Hd, C),
+         "a2": rnd(24, R, B2), "b2": rnd(25, C) * 0.1}
+    acts = {}
+    loss, grads = model_ref.rgcnb2(indptr, indices, et, lab, p, acts)
+    assert np.abs(acts["Z1"]).min() > 1e-4          # no ReLU kink within the FD step
+    for k in p:
+        fd = fd_grad(lambda: model_ref.rgcnb2(indptr, indices, et, lab, p)[0], p[k])
+        assert rel_err(grads[k], fd) < 1e-7, k
