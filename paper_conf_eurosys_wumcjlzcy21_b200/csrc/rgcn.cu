@@ -52,8 +52,8 @@ __device__ void stage_w(const RgcnRowArgs& a, float* Ws) {
 // WPR = 1: RL lanes per row (rows of degree < 1024).  WPR > 1 (hub rows, degree >= 1024): one CTA of WPR
 // warps per row, warp w owns the contiguous edge slice w/WPR of the row (a type run cut at a slice border is
 // flushed through W_r by both warps -- linear, so exact), per-warp outputs merged in warp order.
-template <int L, int RL, int WPR>
-__global__ void __launch_bounds__(512) k_rgcn_rows(const RgcnRowArgs a) {
+template <int L, int RL, int WPR, int BS = 512>
+__global__ void __launch_bounds__(BS) k_rgcn_rows(const RgcnRowArgs a) {
     extern __shared__ float4 smem4[];
     float* Ws = reinterpret_cast<float*>(smem4);
     stage_w(a, Ws);
@@ -286,6 +286,94 @@ __global__ void __launch_bounds__(256) k_rgcn_dw(const RgcnDwArgs a) {
     }
 }
 
+// Narrow layers (F_in <= 16, F_out <= 16: every R-GCN config): a group of L lanes (lane c holds input
+// features 4c..4c+3) owns a contiguous edge slice of the task -- 8 warps x 32/L groups per task -- and
+// keeps its whole dW_r partial (4 x 4*FO4 per lane) in registers: per edge one float4 gather and 4 FMAs,
+// per run one dA row and the 4 x F_out outer-product FMAs; no shuffles or shared memory inside the edge
+// loop.  Groups are merged by a fixed xor tree, warps in warp order (deterministic).
+template <int L, int FO4>
+__global__ void __launch_bounds__(256) k_rgcn_dw_g(const RgcnDwArgs a) {
+    constexpr int S = 32 / L, WARPS = 8, G = WARPS * S, FO = 4 * FO4;
+    extern __shared__ float red[];                 // [WARPS][Fin * Fout]
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int slot = lane / L, c = lane % L;
+    const int Cg = (a.Fin + 3) / 4;
+    const int FF = a.Fin * a.Fout;
+    for (int64_t t = blockIdx.x; t < a.n_tasks; t += gridDim.x) {
+        float acc[4][FO];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int j = 0; j < FO; ++j) acc[i][j] = 0.f;
+        const int r0 = __ldg(a.task_run + t), r1 = __ldg(a.task_run + t + 1);
+        const int es = __ldg(a.run_off + r0), ee = __ldg(a.run_off + r1);
+        const int64_t n = ee - es;
+        const int q = w * S + slot;
+        const int k0 = es + (int)(n * q / G), k1 = es + (int)(n * (q + 1) / G);
+        if (k0 < k1) {                                 // group-uniform
+            int lo = r0, hi = r1 - 1;                  // last run with run_off <= k0
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (__ldg(a.run_off + mid) <= k0) lo = mid; else hi = mid - 1;
+            }
+            int run = lo, rend = __ldg(a.run_off + run + 1);
+            float g[4] = {0.f, 0.f, 0.f, 0.f};
+            auto flush = [&]() {
+                const float* dp = a.dA + (int64_t)__ldg(a.run_dst + run) * a.ldd;
+                float d[FO];
+#pragma unroll
+                for (int j4 = 0; j4 < FO4; ++j4) {
+                    const float4 d4 = ldg4(dp + 4 * j4);
+                    d[4 * j4] = d4.x; d[4 * j4 + 1] = d4.y; d[4 * j4 + 2] = d4.z; d[4 * j4 + 3] = d4.w;
+                }
+#pragma unroll
+                for (int j = 0; j < FO; ++j)
+                    if (j >= a.Fout) d[j] = 0.f;       // the row padding is never read into a result
+#pragma unroll
+                for (int i = 0; i < 4; ++i)
+#pragma unroll
+                    for (int j = 0; j < FO; ++j) acc[i][j] = fmaf(g[i], d[j], acc[i][j]);
+            };
+            for (int k = k0; k < k1; ++k) {
+                if (k == rend) {
+                    flush();
+                    ++run;
+                    rend = __ldg(a.run_off + run + 1);
+                    g[0] = g[1] = g[2] = g[3] = 0.f;
+                }
+                if (c < Cg) {
+                    const int u = __ldg(a.src + k);
+                    const float wgt = a.norm_user ? __ldg(a.norm_user + __ldg(a.eid + k)) : __ldg(a.norm + k);
+                    const float4 x = ldg4(a.X + (int64_t)u * a.ldx + 4 * c);
+                    g[0] = fmaf(wgt, x.x, g[0]); g[1] = fmaf(wgt, x.y, g[1]);
+                    g[2] = fmaf(wgt, x.z, g[2]); g[3] = fmaf(wgt, x.w, g[3]);
+                }
+            }
+            flush();
+        }
+#pragma unroll
+        for (int o = L; o < 32; o <<= 1)
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+#pragma unroll
+                for (int j = 0; j < FO; ++j) acc[i][j] += __shfl_xor_sync(0xffffffffu, acc[i][j], o);
+        if (slot == 0 && c < Cg)
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+#pragma unroll
+                for (int j = 0; j < FO; ++j)
+                    if (4 * c + i < a.Fin && j < a.Fout) red[w * FF + (4 * c + i) * a.Fout + j] = acc[i][j];
+        __syncthreads();
+        for (int e = threadIdx.x; e < FF; e += blockDim.x) {
+            float x = red[e];
+#pragma unroll
+            for (int w2 = 1; w2 < WARPS; ++w2) x += red[w2 * FF + e];
+            a.part[t * FF + e] = x;
+        }
+        __syncthreads();
+    }
+}
+
 __global__ void __launch_bounds__(256) k_seg_reduce_cols(const float* __restrict__ part,
                                                           const int32_t* __restrict__ seg_off, int width,
                                                           float* __restrict__ out) {
@@ -313,27 +401,29 @@ void seg_reduce_cols(const float* part, const int32_t* seg_off, int nseg, int wi
     k_seg_reduce_cols<<<dim3((unsigned)((width + 31) / 32), (unsigned)nseg), 256, 0, s>>>(part, seg_off, width, out);
 }
 
-template <int L, int RL, int WPR = 1>
+// BS: 1024-thread CTAs for the narrow (L <= 4, <= 64 registers) row kernels, so that a W table too large for two
+// CTAs per SM (AM: 133 x 16 x 16 fp32 = 136 KB) still leaves 32 warps per SM to hide the gather latency
+template <int L, int RL, int WPR = 1, int BS = (WPR == 1 && L <= 4 ? 1024 : 512)>
 static seastar_status launch_rows(const RgcnRowArgs& a, size_t smem, cudaStream_t s) {
     if (a.row_end <= a.row_begin) return SEASTAR_OK;
     static bool attr_set = false;
     if (!attr_set) {
-        SS_CUDA(cudaFuncSetAttribute(k_rgcn_rows<L, RL, WPR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        SS_CUDA(cudaFuncSetAttribute(k_rgcn_rows<L, RL, WPR, BS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      227 * 1024 - (int)sizeof(float) * 64 * WPR));
         attr_set = true;
     }
     int per_sm = 0;
-    SS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rgcn_rows<L, RL, WPR>, 512, smem));
+    SS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rgcn_rows<L, RL, WPR, BS>, BS, smem));
     if (per_sm < 1) {
         set_error("rgcn: W (%zu bytes) does not fit in shared memory", smem);
         return SEASTAR_ERR_UNSUPPORTED;
     }
     const int64_t groups = a.row_end - a.row_begin;
     int64_t blocks = (int64_t)per_sm * num_sms();
-    const int gpb = WPR > 1 ? 1 : 512 / RL;
+    const int gpb = WPR > 1 ? 1 : BS / RL;
     const int64_t need = (groups + gpb - 1) / gpb;
     if (blocks > need) blocks = need;
-    launch_k(k_rgcn_rows<L, RL, WPR>, dim3((unsigned)blocks), dim3(512), smem, s, a);
+    launch_k(k_rgcn_rows<L, RL, WPR, BS>, dim3((unsigned)blocks), dim3(BS), smem, s, a);
     return check_launch("k_rgcn_rows");
 }
 
@@ -455,13 +545,38 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
         case 16: RGCN_DW(LL, 16); break;                                \
         default: RGCN_DW(LL, 32); break;                                \
     }
-            switch (L) {
-                case 1: RGCN_DW_L(1); break;
-                case 2: RGCN_DW_L(2); break;
-                case 4: RGCN_DW_L(4); break;
-                case 8: RGCN_DW_L(8); break;
-                default: RGCN_DW_L(16); break;
+#define RGCN_DWG(LL, F4)                                                                                \
+    do {                                                                                                  \
+        int per_sm = 0;                                                                                   \
+        SS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rgcn_dw_g<LL, F4>, 256, smem_r)); \
+        blocks = (int64_t)(per_sm > 0 ? per_sm : 1) * num_sms();                                          \
+        if (blocks > g->tm.n_tasks) blocks = g->tm.n_tasks;                                               \
+        launch_k(k_rgcn_dw_g<LL, F4>, dim3((unsigned)blocks), dim3(256), smem_r, s, d);                   \
+    } while (0)
+#define RGCN_DWG_L(LL)                   \
+    switch ((F_out + 3) / 4) {           \
+        case 1: RGCN_DWG(LL, 1); break;  \
+        case 2: RGCN_DWG(LL, 2); break;  \
+        case 3: RGCN_DWG(LL, 3); break;  \
+        default: RGCN_DWG(LL, 4); break; \
+    }
+            if (F_in <= 16 && F_out <= 16) {
+                switch (L) {
+                    case 1: RGCN_DWG_L(1); break;
+                    case 2: RGCN_DWG_L(2); break;
+                    default: RGCN_DWG_L(4); break;
+                }
+            } else {
+                switch (L) {
+                    case 1: RGCN_DW_L(1); break;
+                    case 2: RGCN_DW_L(2); break;
+                    case 4: RGCN_DW_L(4); break;
+                    case 8: RGCN_DW_L(8); break;
+                    default: RGCN_DW_L(16); break;
+                }
             }
+#undef RGCN_DWG_L
+#undef RGCN_DWG
 #undef RGCN_DW_L
 #undef RGCN_DW
             SS_TRY(check_launch("k_rgcn_dw"));
