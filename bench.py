@@ -329,11 +329,18 @@ def main():
         return
 
     import torch
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # SEASTAR_DIST_BACKEND=gloo runs the partitioned path with several ranks sharing the visible GPUs
+    # (collectives staged through host memory): a functional check of the N > 1 path on a 1-GPU box
+    backend = os.environ.get("SEASTAR_DIST_BACKEND", "nccl")
+    local_dev = local % torch.cuda.device_count() if backend == "gloo" else local
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "gloo":
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
     from paper_conf_eurosys_wumcjlzcy21_b200.graph import Graph
     from paper_conf_eurosys_wumcjlzcy21_b200 import partition
@@ -376,7 +383,7 @@ def main():
         for m in models.values():
             m.epoch()
 
-    clocks = Clocks(local)       # sampled from the warm-up on, so the short timed region has samples under load
+    clocks = Clocks(local_dev)   # sampled from the warm-up on, so the short timed region has samples under load
     clocks.start()
     for _ in range(args.warmup):
         step()

@@ -22,7 +22,8 @@ gat_attn_proj(_bwd)        e_u = f_u^T attn_u                                   
 gat_fwd / gat_bwd          LeakyReLU -> edge softmax -> weighted sum            Fig.2, Fig.3
 rgcn_norm/fwd/bwd          sum_r sum_{u in N_r(v)} 1/c_{v,r} h_u W_r           L465-475, [53]
 rgcn_basis_fwd/bwd         featureless input, W_r = sum_b a_rb V_b (NEXT-2)      L485, L1219-1227, [53]
-basis_combine(_bwd)        W_r = sum_b a_rb V_b for a dense layer (NEXT-2)       [53] (reading #27)
+basis_combine(_bwd)        W_r = sum_b a_rb V_b for a dense layer (NEXT-2)       [53] (reading #26)
+dropout_mask               counter-based keep mask x 1/(1-p) (NEXT-3)            L361, L481 (reading #27)
 softmax_xent, adam         DGL default training loop                             L481
 =========================  ===================================================  ==================
 
@@ -82,6 +83,8 @@ def _L():
             "orc_rgcn_bwd": ([_I, _I, _P, _P, _P, ctypes.c_int32, _I, _I, _P, _P, _P, _P, _P, _P], None),
             "orc_rgcn_basis_fwd": ([_I, _I, _P, _P, _P, _I, _I, _P, _P, _P, _P, _I, _P], None),
             "orc_rgcn_basis_bwd": ([_I, _I, _P, _P, _P, ctypes.c_int32, _I, _I, _P, _P, _P, _P, _P, _P], None),
+            "orc_sm64": ([ctypes.c_uint64], ctypes.c_uint64),
+            "orc_dropout_keep": ([ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32, _I, _I, ctypes.c_float, _P], None),
             "orc_softmax_xent": ([_I, _I, _P, _P, _P], _D),
             "orc_adam": ([_I, _P, _P, _P, _P, _D, _D, _D, _D, _I], None),
         }
@@ -410,6 +413,21 @@ def basis_combine_bwd(a, Vb, dW):
         for r in range(R):
             dVb[b] += a[r, b] * dW[r]
     return da, dVb
+
+
+# ------------------------------------------------------------------------------------------
+# NEXT-3: reproducible dropout (reading #27)
+# ------------------------------------------------------------------------------------------
+def sm64(z):
+    return int(_L().orc_sm64(int(z) & 0xFFFFFFFFFFFFFFFF))
+
+
+def dropout_mask(seed, site, step, M, F, p, row0=0):
+    """[M, F] fp64 inverted-dropout multiplier: keep(seed, site, step, (row0 + r) * F + f) / (1 - p), else 0."""
+    p32 = float(np.float32(p))
+    keep = np.empty(M * F, np.uint8)
+    _L().orc_dropout_keep(int(seed), int(site), int(step), int(row0) * int(F), M * F, p32, _p(keep))
+    return keep.reshape(M, F).astype(np.float64) / (1.0 - p32)
 
 
 # ------------------------------------------------------------------------------------------

@@ -8,16 +8,27 @@ import numpy as np
 import oracle  # noqa: F401  (package of the oracle functions composed here)
 
 
-def gcn2(ip, ix, X, lab, p, acts=None):
+def _mask(drop, site, M, F):
+    """NEXT-3 inverted-dropout multiplier for one dropout site (all ones when drop is None or p = 0).
+    drop = dict(p=..., seed=..., step=...); sites: GCN 1 = hidden; GAT 1 = X, 2 = hidden."""
+    if not drop or drop["p"] == 0.0:
+        return None
+    return oracle.dropout_mask(drop["seed"], site, drop["step"], M, F, drop["p"])
+
+
+def gcn2(ip, ix, X, lab, p, acts=None, drop=None):
     in_n, out_n = oracle.degree_norms(ip, ix)
     T = oracle.linear_fwd(X, p["W1"])
     Z1 = oracle.gcn_aggregate(ip, ix, T, out_n, in_n) + p["b1"]
     H1 = oracle.act_fwd("relu", Z1)
-    P2 = oracle.gcn_aggregate(ip, ix, H1, out_n, in_n)
+    m1 = _mask(drop, 1, *H1.shape)
+    P2 = oracle.gcn_aggregate(ip, ix, H1 if m1 is None else H1 * m1, out_n, in_n)
     logits = oracle.linear_fwd(P2, p["W2"], p["b2"])
     loss, dlog = oracle.softmax_xent(logits, lab)
     dP2, dW2, db2 = oracle.linear_bwd(P2, p["W2"], dlog)
     dH1 = oracle.gcn_aggregate_T(ip, ix, dP2, out_n, in_n)
+    if m1 is not None:
+        dH1 = dH1 * m1
     dZ1 = oracle.act_bwd("relu", Z1, dH1)
     db1 = dZ1.sum(0)
     dT = oracle.gcn_aggregate_T(ip, ix, dZ1, out_n, in_n)
@@ -49,24 +60,30 @@ def _gat_layer_bwd(ip, ix, Xin, W, al, ar, T, el, er, Z, act, dY, H, F, need_dX)
     return dX, dW, dal, dar, db
 
 
-def gat2(ip, ix, X, lab, p, heads, hidden, acts=None):
+def gat2(ip, ix, X, lab, p, heads, hidden, acts=None, drop=None):
     C = p["W2"].shape[1]
-    T1, el1, er1, Z1, Y1 = _gat_layer_fwd(ip, ix, X, p["W1"], p["al1"], p["ar1"], p["b1"], "elu", heads, hidden)
+    m0 = _mask(drop, 1, *X.shape)                    # feat_drop on the layer-1 input
+    Xd = X if m0 is None else X * m0
+    T1, el1, er1, Z1, Y1 = _gat_layer_fwd(ip, ix, Xd, p["W1"], p["al1"], p["ar1"], p["b1"], "elu", heads, hidden)
     lse1 = _gat_layer_fwd.lse
-    T2, el2, er2, Z2, Y2 = _gat_layer_fwd(ip, ix, Y1, p["W2"], p["al2"], p["ar2"], p["b2"], "none", 1, C)
+    m1 = _mask(drop, 2, *Y1.shape)                   # feat_drop on the layer-2 input
+    Y1d = Y1 if m1 is None else Y1 * m1
+    T2, el2, er2, Z2, Y2 = _gat_layer_fwd(ip, ix, Y1d, p["W2"], p["al2"], p["ar2"], p["b2"], "none", 1, C)
     lse2 = _gat_layer_fwd.lse
     loss, dY2 = oracle.softmax_xent(Y2, lab)
-    dY1, dW2, dal2, dar2, db2 = _gat_layer_bwd(ip, ix, Y1, p["W2"], p["al2"], p["ar2"], T2, el2, er2, Z2, "none",
+    dY1, dW2, dal2, dar2, db2 = _gat_layer_bwd(ip, ix, Y1d, p["W2"], p["al2"], p["ar2"], T2, el2, er2, Z2, "none",
                                                dY2, 1, C, True)
+    if m1 is not None:
+        dY1 = dY1 * m1
     dZ2 = _gat_layer_bwd.dZ
-    _, dW1, dal1, dar1, db1 = _gat_layer_bwd(ip, ix, X, p["W1"], p["al1"], p["ar1"], T1, el1, er1, Z1, "elu", dY1,
+    _, dW1, dal1, dar1, db1 = _gat_layer_bwd(ip, ix, Xd, p["W1"], p["al1"], p["ar1"], T1, el1, er1, Z1, "elu", dY1,
                                              heads, hidden, False)
     dZ1 = _gat_layer_bwd.dZ
     if acts is not None:
         acts.update(Y1=Y1, Y2=Y2,
-                    layers=[dict(Xin=X, T=T1, el=el1, er=er1, A=Z1 - p["b1"], lse=lse1, dZ=dZ1, al=p["al1"],
+                    layers=[dict(Xin=Xd, T=T1, el=el1, er=er1, A=Z1 - p["b1"], lse=lse1, dZ=dZ1, al=p["al1"],
                                  ar=p["ar1"]),
-                            dict(Xin=Y1, T=T2, el=el2, er=er2, A=Z2 - p["b2"], lse=lse2, dZ=dZ2, al=p["al2"],
+                            dict(Xin=Y1d, T=T2, el=el2, er=er2, A=Z2 - p["b2"], lse=lse2, dZ=dZ2, al=p["al2"],
                                  ar=p["ar2"])])
     return loss, {"W1": dW1, "al1": dal1, "ar1": dar1, "b1": db1, "W2": dW2, "al2": dal2, "ar2": dar2, "b2": db2}
 

@@ -612,6 +612,29 @@ void orc_rgcn_basis_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64
 }
 
 /* ------------------------------------------------------------------------------------------ */
+/* NEXT-3: reproducible dropout ("further processed using a Dropout layer"; DGL    */
+/* default configs, L481).  Counter-based mask, reading #27:                          */
+/*   key   = sm64(seed ^ sm64((site << 32) | step))                                             */
+/*   keep(i) <=> (sm64(key ^ i) >> 40) >= thr,  thr = round(p * 2^24)                            */
+/* with sm64 = Vigna's splitmix64 output function; i = global element index row * F + col.      */
+/* ------------------------------------------------------------------------------------------ */
+static uint64_t sm64(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+uint64_t orc_sm64(uint64_t z) { return sm64(z); }
+
+/* mask[i] = keep(idx0 + i) ? 1 : 0 for i < n; p is the fp32 drop probability */
+void orc_dropout_keep(uint64_t seed, uint32_t site, int32_t step, int64_t idx0, int64_t n, float p, uint8_t* mask) {
+    const uint64_t key = sm64(seed ^ sm64(((uint64_t)site << 32) | (uint32_t)step));
+    const uint32_t thr = (uint32_t)llround((double)p * 16777216.0);
+    for (int64_t i = 0; i < n; ++i) mask[i] = (uint8_t)((sm64(key ^ (uint64_t)(idx0 + i)) >> 40) >= thr);
+}
+
+/* ------------------------------------------------------------------------------------------ */
 /* training-step pieces around the hot path (DGL default training loop)         */
 /* ------------------------------------------------------------------------------------------ */
 

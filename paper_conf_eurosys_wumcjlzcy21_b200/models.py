@@ -36,26 +36,58 @@ def _local_rows(m) -> int:
 
 
 class Comm:
-    """Row-partition plumbing.  P = 1: every gather is the identity (no copies)."""
+    """Row-partition plumbing.  P = 1: every gather is the identity (no copies).
 
-    def __init__(self, world: int = 1, rank: int = 0, group=None):
+    The collectives are NCCL's (``torch.distributed`` with the nccl backend).  When the process group
+    is gloo (``staged=True``; used to run the partitioned path with several ranks on ONE GPU, e.g. on a
+    single-GPU test box) the same calls are staged through host memory with identical shapes."""
+
+    def __init__(self, world: int = 1, rank: int = 0, group=None, staged: bool | None = None):
         self.world, self.rank, self.group = world, rank, group
+        if staged is None:
+            staged = world > 1 and torch.distributed.get_backend(group) == "gloo"
+        self.staged = staged
+
+    @staticmethod
+    def _rows(t: torch.Tensor) -> torch.Tensor:
+        """A column slice [:, :F] of a row-padded buffer -> the full padded rows (same storage)."""
+        if t.is_contiguous():
+            return t
+        assert t.dim() == 2 and t.stride(1) == 1, "gathered tables are row-major"
+        return torch.as_strided(t, (t.shape[0], t.stride(0)), (t.stride(0), 1))
 
     def all_gather(self, out_all: torch.Tensor, loc: torch.Tensor):
         if self.world == 1:
             return loc
-        torch.distributed.all_gather_into_tensor(out_all, loc, group=self.group)
+        loc = self._rows(loc)
+        assert out_all.is_contiguous() and out_all.numel() == loc.numel() * self.world, (out_all.shape, loc.shape)
+        if self.staged:
+            parts = [torch.empty(loc.shape, dtype=loc.dtype) for _ in range(self.world)]
+            torch.distributed.all_gather(parts, loc.cpu(), group=self.group)
+            out_all.view(self.world, *loc.shape).copy_(torch.stack(parts))
+        else:
+            torch.distributed.all_gather_into_tensor(out_all, loc, group=self.group)
         return out_all
 
     def reduce_scatter(self, out_loc: torch.Tensor, part_all: torch.Tensor):
         if self.world == 1:
             return part_all
-        torch.distributed.reduce_scatter_tensor(out_loc, part_all, group=self.group)
+        if self.staged:
+            h = part_all.cpu()
+            torch.distributed.all_reduce(h, group=self.group)
+            out_loc.copy_(h.view(self.world, *out_loc.shape)[self.rank])
+        else:
+            torch.distributed.reduce_scatter_tensor(out_loc, part_all, group=self.group)
         return out_loc
 
     def all_reduce(self, flat: torch.Tensor):
         if self.world > 1:
-            torch.distributed.all_reduce(flat, group=self.group)
+            if self.staged:
+                h = flat.cpu()
+                torch.distributed.all_reduce(h, group=self.group)
+                flat.copy_(h)
+            else:
+                torch.distributed.all_reduce(flat, group=self.group)
 
 
 class _Params:

@@ -149,3 +149,36 @@ def test_rgcn_partitioned(env):
     assert abs(sum(r[0] for r in res) - rl) <= TOL * abs(rl)
     for k in rg:
         assert rel_err(res[0][1][k], rg[k].reshape(res[0][1][k].shape)) <= TOL, k
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_rgcnb_partitioned(env, P):
+    """NEXT-2 model: V1 row-partitioned with the vertices (dV rows owned, never all-reduced), V1 all-gathered."""
+    torch, models, part, Graph = env["torch"], env["models"], env["part"], env["Graph"]
+    N, R, B1, B2, Hd, C = 2003, 14, 6, 4, 16, 3
+    ip, ix, et = synth.powerlaw_directed_typed(N, 12000, 0.6, 0.6, R, 1.0, 53)
+    lab = synth.labels(37, N, C)
+    p = {"V1": synth.uniform(38, (N, B1, Hd), -0.5, 0.5), "a1": synth.uniform(39, (R, B1)),
+         "b1": synth.uniform(40, (Hd,), -0.1, 0.1), "V2": synth.uniform(41, (B2, Hd, C), -0.5, 0.5),
+         "a2": synth.uniform(42, (R, B2)), "b2": synth.uniform(43, (C,), -0.1, 0.1)}
+
+    def build(r, comm):
+        torch.cuda.set_device(0)
+        rb, re = part.row_range(N, P, r)
+        g = Graph(ip, ix, et, num_etypes=R, row_begin=rb, row_end=re, rgcn_norm=True)
+        m = models.RGCNBasis2(g, torch.from_numpy(lab[rb:re]).cuda(), p, comm=comm,
+                              n_pad_rows=part.gathered_rows(N, P))
+        l = m.forward().item()
+        m.backward()
+        torch.cuda.synchronize()
+        return l, {k: m.grad(k).cpu().numpy().copy() for k in p}, rb, re
+
+    res = run_ranks(P, build)
+    rl, rg = model_ref.rgcnb2(ip, ix, et, lab, {k: v.astype(np.float64) for k, v in p.items()})
+    assert abs(sum(r[0] for r in res) - rl) <= TOL * abs(rl)
+    for k in rg:
+        if k == "V1":       # owned rows of each rank, concatenated
+            got = np.concatenate([r[1]["V1"] for r in res], 0)
+        else:
+            got = res[0][1][k]
+        assert rel_err(got, rg[k].reshape(got.shape)) <= TOL, k
