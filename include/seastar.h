@@ -372,6 +372,19 @@ seastar_status seastar_axpby(int64_t n, float a, const float* x, float b, float*
  */
 seastar_status seastar_adam(float* param, const float* grad, float* m, float* v, int64_t n, float lr, float beta1,
                             float beta2, float eps, const int32_t* step, seastar_stream stream);
+/*
+ * NEXT-3: reproducible inverted dropout ("a Dropout layer"; DGL default configs L481;
+ * DESIGN.md reading #27).  Y[r,f] = keep(i) ? X[r,f] / (1 - p) : 0 with i = (row0 + r) * F + f (the
+ * element's GLOBAL index, so a row-partitioned caller passes row0 = row_begin and reproduces the
+ * single-GPU mask) and
+ *   key = sm64(seed ^ sm64((site << 32) | step)),  keep(i) <=> (sm64(key ^ i) >> 40) >= round(p * 2^24),
+ * sm64 = splitmix64's output function.  `step` (dev int32, e.g. the Adam step counter) or NULL (= 0) is
+ * read on the device, so a captured CUDA graph draws a fresh mask every epoch.  The mask is a pure
+ * function of (seed, site, step, i): the backward is the same call on dY.  X [M,F] ld ldx, Y [M,F] ld
+ * ldy (dev; Y == X allowed when ldy == ldx).  0 <= p < 1.
+ */
+seastar_status seastar_dropout(const float* X, int64_t M, int64_t F, int64_t ldx, int64_t row0, float p, uint64_t seed,
+                               uint32_t site, const int32_t* step, float* Y, int64_t ldy, seastar_stream stream);
 /* *counter += 1 on the device */
 seastar_status seastar_step_inc(int32_t* counter, seastar_stream stream);
 

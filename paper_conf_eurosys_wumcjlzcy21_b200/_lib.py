@@ -80,6 +80,7 @@ _SIGS = {
     "seastar_rgcn_basis_fwd": ([_P, _P, _I64, _I64, _I64, _P, _P, _P, _I64, _P, _I32, _P, _I64, _P], _ST),
     "seastar_rgcn_basis_bwd": ([_P, _P, _I64, _I64, _I64, _P, _P, _P, _I64, _P, _P, _P, _SZ, _P], _ST),
     "seastar_rgcn_basis_bwd_workspace": ([_P, _I64], _SZ),
+    "seastar_dropout": ([_P, _I64, _I64, _I64, _I64, _F, ctypes.c_uint64, ctypes.c_uint32, _P, _P, _I64, _P], _ST),
     "seastar_basis_combine": ([_P, _P, _I32, _I32, _I64, _P, _P], _ST),
     "seastar_basis_combine_bwd": ([_P, _P, _P, _I32, _I32, _I64, _P, _P, _P], _ST),
     "seastar_softmax_xent": ([_P, _I64, _I64, _I32, _I64, _P, _P, _P, _I64, _P, _SZ, _P], _ST),
@@ -330,6 +331,12 @@ def seastar_basis_combine(a, Vb, R, B, K, W, stream=None) -> None:
 def seastar_basis_combine_bwd(a, Vb, dW, R, B, K, da, dVb, stream=None) -> None:
     _call("seastar_basis_combine_bwd", _dptr(a, "a"), _dptr(Vb, "Vb"), _dptr(dW, "dW"), R, B, K, _dptr(da, "da"),
           _dptr(dVb, "dVb"), _stream(stream))
+
+
+# ----------------------------------------------------------------------------------- dropout (NEXT-3)
+def seastar_dropout(X, M, F, ldx, row0, p, seed, site, step, Y, ldy, stream=None) -> None:
+    _call("seastar_dropout", _dptr(X, "X"), M, F, ldx, row0, p, seed, site, _dptr(step, "step"), _dptr(Y, "Y"), ldy,
+          _stream(stream))
 
 
 # ----------------------------------------------------------------------------------- glue

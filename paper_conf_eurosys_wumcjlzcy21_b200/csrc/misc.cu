@@ -4,6 +4,7 @@
 #include <math.h>
 
 #include "common.cuh"
+#include <cmath>
 
 namespace seastar {
 
@@ -198,6 +199,30 @@ __global__ void __launch_bounds__(256) k_adam(float* __restrict__ p, const float
 
 __global__ void k_step_inc(int32_t* c) { *c += 1; }
 
+// NEXT-3 dropout (reading #27): splitmix64 output function, counter = global element index
+__device__ __forceinline__ uint64_t sm64(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+__global__ void __launch_bounds__(256) k_dropout(const float* X, int64_t M, uint32_t F, int64_t ldx, int64_t row0,
+                                                 uint32_t thr, float scale, uint64_t seed, uint32_t site,
+                                                 const int32_t* __restrict__ step, float* Y, int64_t ldy) {
+    const uint32_t st = step ? (uint32_t)*step : 0u;
+    const uint64_t key = sm64(seed ^ sm64(((uint64_t)site << 32) | st));
+    const uint64_t n = (uint64_t)M * F;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += stride) {
+        const uint64_t r = n <= 0xFFFFFFFFull ? (uint64_t)((uint32_t)i / F) : i / F;
+        const uint64_t f = i - r * F;
+        const bool keep = (sm64(key ^ ((uint64_t)(row0 + (int64_t)r) * F + f)) >> 40) >= thr;
+        const float x = X[r * ldx + f];
+        Y[r * ldy + f] = keep ? x * scale : 0.f;
+    }
+}
+
 }  // namespace seastar
 
 using namespace seastar;
@@ -252,6 +277,25 @@ seastar_status seastar_adam(float* param, const float* grad, float* m, float* v,
     if (blocks < 1) blocks = 1;
     k_adam<<<(unsigned)blocks, 256, 0, to_stream(stream)>>>(param, grad, m, v, n, lr, beta1, beta2, eps, step, vec);
     return check_launch("k_adam");
+}
+
+seastar_status seastar_dropout(const float* X, int64_t M, int64_t F, int64_t ldx, int64_t row0, float p, uint64_t seed,
+                               uint32_t site, const int32_t* step, float* Y, int64_t ldy, seastar_stream stream) {
+    SS_ARG(X && Y, "dropout: NULL argument");
+    SS_ARG(M >= 0 && F >= 1 && F <= 0xFFFFFFFFll && ldx >= F && ldy >= F && row0 >= 0, "dropout: bad sizes");
+    SS_ARG(p >= 0.f && p < 1.f, "dropout: need 0 <= p < 1 (got %g)", (double)p);
+    SS_ARG(X != Y || ldx == ldy, "dropout: in place needs ldx == ldy");
+    SS_TRY(check_device());
+    if (M == 0) return SEASTAR_OK;
+    const uint32_t thr = (uint32_t)llround((double)p * 16777216.0);
+    const float scale = (float)(1.0 / (1.0 - (double)p));
+    const int64_t n = M * F;
+    int64_t blocks = (n + 255) / 256;
+    const int64_t cap = 16 * (int64_t)num_sms();
+    if (blocks > cap) blocks = cap;
+    k_dropout<<<(unsigned)blocks, 256, 0, to_stream(stream)>>>(X, M, (uint32_t)F, ldx, row0, thr, scale, seed, site, step,
+                                                              Y, ldy);
+    return check_launch("k_dropout");
 }
 
 seastar_status seastar_step_inc(int32_t* counter, seastar_stream stream) {

@@ -151,8 +151,9 @@ class GCN2:
     next-layer norm into the backward aggregation's epilogue."""
 
     def __init__(self, g: Graph, X_loc: torch.Tensor, labels_loc: torch.Tensor, params: dict, lr=0.01,
-                 comm: Comm | None = None, n_pad_rows: int | None = None):
+                 comm: Comm | None = None, n_pad_rows: int | None = None, dropout: float = 0.0, seed: int = 0):
         self.g, self.X, self.lab, self.lr = g, X_loc, labels_loc, lr
+        self.drop_p, self.drop_seed = float(dropout), int(seed)     # NEXT-3: dropout on the hidden layer (DGL: 0.5)
         self.comm = comm or Comm()
         dev = X_loc.device
         self.n = g.n_loc
@@ -199,6 +200,8 @@ class GCN2:
         L.seastar_gcn_fwd(g.handle, T1_all, H, H, self.dst_n, p.p("b1"), "relu", 0.0, None, self.H1, self.src_n,
                           self.H1s)
         self._t("gcn_fwd1_end")
+        if self.drop_p > 0:      # layer-2 input src_n * drop(H1): the mask commutes with the row scale
+            L.seastar_dropout(self.H1s, n, H, H, g.row_begin, self.drop_p, self.drop_seed, 1, p.step, self.H1s, H)
         H1s_all = self.comm.all_gather(self.H1s_all, self.H1s)
         L.seastar_gcn_fwd(g.handle, H1s_all, H, H, self.dst_n, None, "none", 0.0, None, self.P2)
         _linear(self.ws, self.P2, n, H, H, p.p("W2"), C, p.p("b2"), None, "none", self.logits, self.ldc)
@@ -219,6 +222,9 @@ class GCN2:
         self._t("gcn_bwd2")
         L.seastar_gcn_bwd(g.handle, dP2_all, H, H, self.src_n, 1.0, self.H1, "relu", self.dst_n, self.dA1, self.dP1)
         self._t("gcn_bwd2_end")
+        if self.drop_p > 0:      # d drop(H1) -> dH1: the same mask, commuting with relu' and the dst_n scale
+            for t in (self.dA1, self.dP1):
+                L.seastar_dropout(t, n, H, H, g.row_begin, self.drop_p, self.drop_seed, 1, p.step, t, H)
         L.seastar_colsum(self.dA1, n, H, H, p.g("b1"), ws, ws.numel())
         dP1_all = self.comm.all_gather(self.dP1_all, self.dP1)
         L.seastar_gcn_bwd(g.handle, dP1_all, H, H, self.src_n, 1.0, None, "none", None, self.dT1, None)
@@ -243,8 +249,9 @@ class GAT2:
 
     def __init__(self, g: Graph, X_loc: torch.Tensor, labels_loc: torch.Tensor, params: dict, heads: int,
                  hidden: int, lr=0.005, slope=0.2, comm: Comm | None = None, n_pad_rows: int | None = None,
-                 save_der_factors: bool = True):
+                 save_der_factors: bool = True, dropout: float = 0.0, seed: int = 0):
         self.g, self.X, self.lab, self.lr, self.slope = g, X_loc, labels_loc, lr, slope
+        self.drop_p, self.drop_seed = float(dropout), int(seed)     # NEXT-3: feat_drop on both layer inputs
         self.save_B = save_der_factors
         self.comm = comm or Comm()
         dev = X_loc.device
@@ -271,6 +278,11 @@ class GAT2:
         self.del1, self.del2 = e(n, heads), e(n, 1)
         self.der1, self.der2 = e(n, heads), e(n, 1)
         self.dY1 = e(n, self.ld1)
+        if self.drop_p > 0:      # dropped layer inputs (kept for the weight gradients)
+            self.Xd = e(n, X_loc.stride(0))[:, :self.Fin]
+            self.Y1d = e(n, self.ld1)
+        else:
+            self.Xd, self.Y1d = X_loc, self.Y1
         self.B1, self.bs1 = (e(n, self.ld1), e(n, heads)) if self.save_B else (None, None)
         self.B2, self.bs2 = (e(n, self.ld2), e(n, 1)) if self.save_B else (None, None)
         self.loss = torch.zeros(1, device=dev)
@@ -292,7 +304,10 @@ class GAT2:
     def forward(self):
         g, p, n = self.g, self.P, self.n
         H, F, W, C = self.H1, self.F1, self.W1w, self.C
-        _linear(self.ws, self.X, n, self.Fin, self.X.stride(0), p.p("W1"), W, None, None, "none", self.T1,
+        if self.drop_p > 0:
+            L.seastar_dropout(self.X, n, self.Fin, self.X.stride(0), g.row_begin, self.drop_p, self.drop_seed, 1,
+                              p.step, self.Xd, self.Xd.stride(0))
+        _linear(self.ws, self.Xd, n, self.Fin, self.Xd.stride(0), p.p("W1"), W, None, None, "none", self.T1,
                              self.ld1)
         L.seastar_gat_attn_proj(self.T1, n, H, F, self.ld1, p.p("al1"), p.p("ar1"), self.el1, self.er1)
         T1_all = self.comm.all_gather(self.T1_all, self.T1)
@@ -302,7 +317,10 @@ class GAT2:
         L.seastar_gat_fwd(g.handle, T1_all, el1_all, self.er1, H, F, self.ld1, self.slope, p.p("b1"), "elu", self.A1,
                           self.Y1, self.lse1, self.B1, self.bs1)
         self._t("gat_fwd1_end")
-        _linear(self.ws, self.Y1, n, W, self.ld1, p.p("W2"), C, None, None, "none", self.T2, self.ld2)
+        if self.drop_p > 0:
+            L.seastar_dropout(self.Y1, n, W, self.ld1, g.row_begin, self.drop_p, self.drop_seed, 2, p.step, self.Y1d,
+                              self.ld1)
+        _linear(self.ws, self.Y1d, n, W, self.ld1, p.p("W2"), C, None, None, "none", self.T2, self.ld2)
         L.seastar_gat_attn_proj(self.T2, n, 1, C, self.ld2, p.p("al2"), p.p("ar2"), self.el2, self.er2)
         T2_all = self.comm.all_gather(self.T2_all, self.T2)
         el2_all = self.comm.all_gather(self.el2_all, self.el2)
@@ -341,14 +359,17 @@ class GAT2:
                         p.p("ar2"), p.g("al2"), p.g("ar2"), p.g("b2"), "2", self.B2, self.bs2)
         ws = self.ws.need(max(L.seastar_linear_bwd_weight_workspace(n, W, C),
                               L.seastar_linear_bwd_weight_workspace(n, self.Fin, W)))
-        L.seastar_linear_bwd_weight(self.Y1, n, W, self.ld1, self.dT2, C, self.ld2, p.g("W2"), None, ws, ws.numel())
+        L.seastar_linear_bwd_weight(self.Y1d, n, W, self.ld1, self.dT2, C, self.ld2, p.g("W2"), None, ws, ws.numel())
         L.seastar_linear_bwd_data(self.dT2, n, C, self.ld2, p.p("W2"), W, None, None, "none", self.dY1, self.ld1)
+        if self.drop_p > 0:
+            L.seastar_dropout(self.dY1, n, W, self.ld1, self.g.row_begin, self.drop_p, self.drop_seed, 2, p.step,
+                              self.dY1, self.ld1)
         self._layer_bwd(self.T1, self.ld1, self.el1, self.er1, self.A1, self.Y1, self.lse1, self.dY1, "elu", H, F,
                         self.D1, self.D1_all, self.dT1, self.del1, self.der1, self._gathered1, p.p("al1"),
                         p.p("ar1"), p.g("al1"), p.g("ar1"), p.g("b1"), "1", self.B1, self.bs1)
         ws = self.ws.need(L.seastar_linear_bwd_weight_workspace(n, self.Fin, W))
-        L.seastar_linear_bwd_weight(self.X, n, self.Fin, self.X.stride(0), self.dT1, W, self.ld1, p.g("W1"), None, ws,
-                                    ws.numel())
+        L.seastar_linear_bwd_weight(self.Xd, n, self.Fin, self.Xd.stride(0), self.dT1, W, self.ld1, p.g("W1"), None,
+                                    ws, ws.numel())
         self.comm.all_reduce(self.P.grad)
 
     def epoch(self):

@@ -1,0 +1,130 @@
+"""NEXT-3 parity: seastar_dropout (counter-based inverted dropout) against the oracle's mask -- identical keep
+decisions (bit-exact, integer work), values within fp32 rounding -- and the dropout-composed GCN2 / GAT2
+training steps (single GPU and row-partitioned) against the oracle compositions."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from conftest import rel_err
+from oracle import model_ref
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-5
+
+
+@pytest.fixture(scope="module")
+def env():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
+    from paper_conf_eurosys_wumcjlzcy21_b200 import models, partition
+    from paper_conf_eurosys_wumcjlzcy21_b200.graph import Graph
+    return dict(torch=torch, L=L, models=models, part=partition, Graph=Graph)
+
+
+@pytest.mark.parametrize("M,F,ld,p,row0,step", [(1000, 16, 16, 0.5, 0, 0), (777, 602, 604, 0.6, 123, 7),
+                                                (5, 3, 4, 0.1, 0, 1), (2048, 41, 44, 0.9, 4096, 123456),
+                                                (300, 64, 64, 0.0, 0, 3)])
+def test_dropout_kernel(env, M, F, ld, p, row0, step):
+    torch, L = env["torch"], env["L"]
+    X = synth.uniform(1, (M, F), 0.5, 1.5)                      # nonzero, so Y == 0 <=> dropped
+    Xp = np.full((M, ld), np.nan, np.float32)
+    Xp[:, :F] = X
+    Xd = torch.from_numpy(Xp).cuda()
+    Y = torch.full((M, ld), float("nan"), device="cuda")
+    st = torch.tensor([step], dtype=torch.int32, device="cuda")
+    L.seastar_dropout(Xd, M, F, ld, row0, p, 0xABCDEF12345, 3, st, Y, ld)
+    mask = oracle.dropout_mask(0xABCDEF12345, 3, step, M, F, p, row0=row0)
+    y = Y.cpu().numpy()
+    assert np.array_equal(y[:, :F] != 0, mask > 0)              # identical keep decisions
+    assert rel_err(y[:, :F], X * mask) <= 1e-6
+    assert np.isnan(y[:, F:]).all()                             # padding never written
+    # in place, and the backward is the same call
+    L.seastar_dropout(Xd, M, F, ld, row0, p, 0xABCDEF12345, 3, st, Xd, ld)
+    assert torch.equal(Xd[:, :F], Y[:, :F])
+
+
+def test_dropout_fresh_mask_per_step_under_graph_replay(env):
+    torch, L = env["torch"], env["L"]
+    M, F = 512, 16
+    X = torch.ones((M, F), device="cuda")
+    Y = torch.empty_like(X)
+    st = torch.zeros(1, dtype=torch.int32, device="cuda")
+    g = torch.cuda.CUDAGraph()
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.graph(g, stream=s):
+        L.seastar_dropout(X, M, F, F, 0, 0.5, 42, 1, st, Y, F)
+        L.seastar_step_inc(st)
+    torch.cuda.current_stream().wait_stream(s)
+    for step in range(3):
+        g.replay()
+        torch.cuda.synchronize()
+        assert np.array_equal(Y.cpu().numpy() != 0, oracle.dropout_mask(42, 1, step, M, F, 0.5) > 0)
+
+
+def _check(m, loss_ref, grads_ref):
+    loss = m.forward()
+    m.backward()
+    assert abs(loss.item() - loss_ref) <= TOL * abs(loss_ref)
+    for k, ref in grads_ref.items():
+        got = m.P.g(k).cpu().numpy()
+        assert rel_err(got, ref.reshape(got.shape)) <= TOL, k
+
+
+def test_gcn2_dropout(env):
+    torch, models, Graph = env["torch"], env["models"], env["Graph"]
+    ip, ix = synth.powerlaw_sym(2000, 16000, 0.6, 61)
+    N, Fin, H, C = 2000, 120, 16, 7
+    X, lab = synth.uniform(1, (N, Fin)), synth.labels(2, N, C)
+    p = {"W1": synth.glorot(3, Fin, H), "b1": synth.uniform(4, (H,), -0.1, 0.1),
+         "W2": synth.glorot(5, H, C), "b2": synth.uniform(6, (C,), -0.1, 0.1)}
+    m = models.GCN2(Graph(ip, ix), torch.from_numpy(X).cuda(), torch.from_numpy(lab).cuda(), p, dropout=0.5, seed=99)
+    _check(m, *model_ref.gcn2(ip, ix, X, lab, {k: v.astype(np.float64) for k, v in p.items()},
+                              drop={"p": 0.5, "seed": 99, "step": 0}))
+
+
+def test_gat2_dropout(env):
+    torch, models, Graph = env["torch"], env["models"], env["Graph"]
+    ip, ix = synth.powerlaw_sym(1500, 12000, 0.6, 62)
+    N, Fin, heads, hid, C = 1500, 100, 8, 8, 41
+    X, lab = synth.uniform(11, (N, Fin)), synth.labels(12, N, C)
+    p = {"W1": synth.glorot(13, Fin, heads * hid), "al1": synth.uniform(14, (heads, hid), -0.5, 0.5),
+         "ar1": synth.uniform(15, (heads, hid), -0.5, 0.5), "b1": synth.uniform(16, (heads * hid,), -0.1, 0.1),
+         "W2": synth.glorot(17, heads * hid, C), "al2": synth.uniform(18, (1, C), -0.5, 0.5),
+         "ar2": synth.uniform(19, (1, C), -0.5, 0.5), "b2": synth.uniform(20, (C,), -0.1, 0.1)}
+    Xp = torch.zeros((N, 100), device="cuda")
+    Xp.copy_(torch.from_numpy(X))
+    m = models.GAT2(Graph(ip, ix), Xp, torch.from_numpy(lab).cuda(), p, heads, hid, dropout=0.6, seed=7)
+    _check(m, *model_ref.gat2(ip, ix, X, lab, {k: v.astype(np.float64) for k, v in p.items()}, heads, hid,
+                              drop={"p": 0.6, "seed": 7, "step": 0}))
+
+
+def test_gcn2_dropout_partitioned(env):
+    """Masks are keyed by the global element index: P = 2 ranks reproduce the single-GPU step."""
+    from test_gpu_partition import run_ranks
+    torch, models, part, Graph = env["torch"], env["models"], env["part"], env["Graph"]
+    P, N, Fin, H, C = 2, 1801, 60, 16, 5
+    ip, ix = synth.powerlaw_sym(N, 14000, 0.5, 63)
+    X, lab = synth.uniform(21, (N, Fin)), synth.labels(22, N, C)
+    p = {"W1": synth.glorot(23, Fin, H), "b1": synth.uniform(24, (H,), -0.1, 0.1),
+         "W2": synth.glorot(25, H, C), "b2": synth.uniform(26, (C,), -0.1, 0.1)}
+
+    def build(r, comm):
+        torch.cuda.set_device(0)
+        rb, re = part.row_range(N, P, r)
+        m = models.GCN2(Graph(ip, ix, row_begin=rb, row_end=re), torch.from_numpy(X[rb:re]).cuda(),
+                        torch.from_numpy(lab[rb:re]).cuda(), p, comm=comm, n_pad_rows=part.gathered_rows(N, P),
+                        dropout=0.5, seed=5)
+        l = m.forward().item()
+        m.backward()
+        torch.cuda.synchronize()
+        return l, {k: m.P.g(k).cpu().numpy().copy() for k in p}
+
+    res = run_ranks(P, build)
+    rl, rg = model_ref.gcn2(ip, ix, X, lab, {k: v.astype(np.float64) for k, v in p.items()},
+                            drop={"p": 0.5, "seed": 5, "step": 0})
+    assert abs(sum(r[0] for r in res) - rl) <= TOL * abs(rl)
+    for k in rg:
+        assert rel_err(res[0][1][k], rg[k].reshape(res[0][1][k].shape)) <= TOL, k
