@@ -40,7 +40,11 @@ struct AggArgs {
 template <int VEC, int L, int RL, int NB>
 __global__ void __launch_bounds__(256) k_aggregate(const AggArgs a) {
     constexpr int S = RL / L;                    // edge slots per row group
+#ifdef GCN_UB_FIXED
+    constexpr int UB = GCN_UB_FIXED < 32 / L ? GCN_UB_FIXED : 32 / L;
+#else
     constexpr int UB = (L < 4 ? L : 4);          // gathers per lane per index chunk and batch
+#endif
     const int lane = threadIdx.x & 31;
     const int gl = lane % RL;                    // lane within the row group
     const int slot = gl / L;
@@ -169,7 +173,10 @@ static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s) {
         const int64_t blocks = (rows + (threads / 32) - 1) / (threads / 32);
         // NB = 1: measured on Reddit F=16, NB=2 (66 regs) is 18% slower than NB=1 (48 regs): occupancy
         // buys more memory-level parallelism than deeper per-lane batches
-        launch_k(k_aggregate<VEC, L, 32, 1>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        // narrow rows (L < 4 chunk lanes, F <= 8) take 4/L index chunks per iteration so every lane still has
+        // 4 gathers in flight: F = 8 0.75 -> 0.50 ms, F = 1..4 0.54 -> 0.46 ms on Reddit (tools/ab_gcn.sh)
+        constexpr int NBW = L >= 4 ? 1 : 4 / L;
+        launch_k(k_aggregate<VEC, L, 32, NBW>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
     } else {
         constexpr int RL = L < 4 ? 4 : L;   // at least 4 lanes per row group keeps index loads useful
         const int64_t per_block = threads / RL;
