@@ -484,23 +484,30 @@ def main():
             Xh, Xd = torch.from_numpy(X[rb:re]).pin_memory(), X_loc
         else:
             Xh, Xd = torch.from_numpy(lab[rb:re]).pin_memory(), lab_loc
-        loss_h = torch.empty(len(models), dtype=torch.float32).pin_memory()
+        loss_h = torch.empty((args.steps, len(models)), dtype=torch.float32).pin_memory()
+        from paper_conf_eurosys_wumcjlzcy21_b200.models import PrefetchedInput
         if world > 1:
             torch.distributed.barrier()
         torch.cuda.synchronize()
-        e_ms = []
-        for _ in range(args.steps):
-            flush.zero_()
-            a = torch.cuda.Event(enable_timing=True)
-            b = torch.cuda.Event(enable_timing=True)
-            a.record(stream)
-            Xd.copy_(Xh, non_blocking=True)
+        flush.zero_()
+        # K steps in one timed region: step t+1's host->device input copy (side stream) overlaps step t's
+        # kernels; every step's losses are copied device->host; the region ends when the last loss is on
+        # the host
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        feed = PrefetchedInput(Xh, Xd)
+        feed.prefetch()
+        for t in range(args.steps):
+            feed.consume()
+            if t + 1 < args.steps:
+                feed.prefetch()
             for i, m in enumerate(runners.values()):
-                loss_h[i:i + 1].copy_(m.epoch(), non_blocking=True)
-            b.record(stream)
-            b.synchronize()
-            _ = loss_h.tolist()
-            e_ms.append(a.elapsed_time(b))
+                loss_h[t, i:i + 1].copy_(m.epoch(), non_blocking=True)
+        b.record(stream)
+        b.synchronize()
+        _ = loss_h.tolist()
+        e_ms = [a.elapsed_time(b)]
         tot = sum(e_ms)
         if world > 1:
             t = torch.tensor([tot], device=dev)
@@ -508,7 +515,9 @@ def main():
             tot = t.item()
         e2e = {"value": edges_per_step / (tot / args.steps / 1e3), "unit": "edges/s",
                "h2d_bytes_per_step": int(Xh.numel() * Xh.element_size()) * world, "d2h_bytes_per_step": 4 * len(models) * world,
-               "ms_per_step": tot / args.steps}
+               "ms_per_step": tot / args.steps,
+               "pipelining": "input rows of step t+1 copied host->device on a side stream during step t "
+                             "(models.PrefetchedInput); losses copied device->host every step"}
 
     # ---- CPU oracle baseline (rank 0, N = 1 only) ----
     cpu = None

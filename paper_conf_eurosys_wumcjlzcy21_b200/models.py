@@ -670,3 +670,31 @@ class CapturedEpoch:
     def epoch(self):
         self.graph.replay()
         return self.loss
+
+
+class PrefetchedInput:
+    """A step's input rows streamed host -> device one step ahead (a DataLoader-style prefetch): the pinned
+    host rows are copied into a device staging buffer on a side stream while the previous step's kernels
+    run, and moved into the model's input buffer (a device-to-device copy) at the start of the step that
+    consumes them.  ``prefetch()`` issues the next copy, ``consume()`` makes the current stream wait for it."""
+
+    def __init__(self, host_pinned: torch.Tensor, dest: torch.Tensor):
+        assert host_pinned.is_pinned() and dest.is_cuda and host_pinned.shape == dest.shape
+        self.h, self.dest = host_pinned, dest
+        self.stage = torch.empty(host_pinned.shape, dtype=host_pinned.dtype, device=dest.device)
+        self.cs = torch.cuda.Stream(device=dest.device)
+        self.ready = torch.cuda.Event()
+        self.free = torch.cuda.Event()
+        self.free.record(torch.cuda.current_stream())
+
+    def prefetch(self):
+        self.cs.wait_event(self.free)                 # the staging buffer has been consumed
+        with torch.cuda.stream(self.cs):
+            self.stage.copy_(self.h, non_blocking=True)
+            self.ready.record(self.cs)
+
+    def consume(self):
+        cur = torch.cuda.current_stream()
+        cur.wait_event(self.ready)
+        self.dest.copy_(self.stage)
+        self.free.record(cur)
