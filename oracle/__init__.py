@@ -76,8 +76,8 @@ def _L():
             "orc_gcn_aggregate": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P], None),
             "orc_gcn_aggregate_T": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P], None),
             "orc_gat_attn_proj": ([_I, _I, _I, _P, _P, _P, _P, _P], None),
-            "orc_gat_fwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _I, _P, _P, _P], None),
-            "orc_gat_bwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _P, _I, _P, _P, _P], None),
+            "orc_gat_fwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _I, _P, _P, _P, _P], None),
+            "orc_gat_bwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _P, _I, _P, _P, _P, _P], None),
             "orc_rgcn_norm": ([_I, _I, _P, _P, ctypes.c_int32, _P], None),
             "orc_rgcn_fwd": ([_I, _I, _P, _P, _P, _I, _I, _P, _P, _P, _P, _I, _P], None),
             "orc_rgcn_bwd": ([_I, _I, _P, _P, _P, ctypes.c_int32, _I, _I, _P, _P, _P, _P, _P, _P], None),
@@ -291,9 +291,10 @@ def gat_attn_proj_bwd(T, a_l, a_r, del_, der):
     return dT, da_l, da_r
 
 
-def gat_fwd(indptr, indices, T, el, er, slope=0.2, rows=None, want_alpha=False):
-    """Returns (A [nrows,H,F], lse [nrows,H], alpha [E,H] or None)."""
-    indptr, indices, T, el, er = _i64(indptr), _i64(indices), _f64(T), _f64(el), _f64(er)
+def gat_fwd(indptr, indices, T, el, er, slope=0.2, rows=None, want_alpha=False, mask=None):
+    """Returns (A [nrows,H,F], lse [nrows,H], alpha [E,H] or None).  mask: [E,H] attention-dropout
+    multiplier by user edge id (NEXT-3), A = sum_e alpha_e mask_e T_u."""
+    indptr, indices, T, el, er, mask = _i64(indptr), _i64(indices), _f64(T), _f64(el), _f64(er), _f64(mask)
     N = indptr.size - 1
     E = int(indptr[-1])
     _, H, F = T.shape
@@ -303,13 +304,14 @@ def gat_fwd(indptr, indices, T, el, er, slope=0.2, rows=None, want_alpha=False):
     lse = np.empty((nrows, H))
     alpha = np.empty((E, H)) if want_alpha else None
     _L().orc_gat_fwd(N, E, _p(indptr), _p(indices), H, F, _p(T), _p(el), _p(er), slope, _p(rows), nrows,
-                     _p(A), _p(lse), _p(alpha))
+                     _p(A), _p(lse), _p(alpha), _p(mask))
     return A, lse, alpha
 
 
-def gat_bwd(indptr, indices, T, el, er, dA, slope=0.2, rows=None):
-    """Returns (dT [nrows,H,F], del [nrows,H], der [N,H])."""
+def gat_bwd(indptr, indices, T, el, er, dA, slope=0.2, rows=None, mask=None):
+    """Returns (dT [nrows,H,F], del [nrows,H], der [N,H]).  mask: as in gat_fwd."""
     indptr, indices, T, el, er, dA = _i64(indptr), _i64(indices), _f64(T), _f64(el), _f64(er), _f64(dA)
+    mask = _f64(mask)
     N = indptr.size - 1
     _, H, F = T.shape
     rows = _i64(rows)
@@ -318,7 +320,7 @@ def gat_bwd(indptr, indices, T, el, er, dA, slope=0.2, rows=None):
     dl = np.empty((nrows, H))
     dr = np.empty((N, H))
     _L().orc_gat_bwd(N, int(indptr[-1]), _p(indptr), _p(indices), H, F, _p(T), _p(el), _p(er), slope, _p(dA),
-                     _p(rows), nrows, _p(dT), _p(dl), _p(dr))
+                     _p(rows), nrows, _p(dT), _p(dl), _p(dr), _p(mask))
     return dT, dl, dr
 
 

@@ -10,7 +10,8 @@ import oracle  # noqa: F401  (package of the oracle functions composed here)
 
 def _mask(drop, site, M, F):
     """NEXT-3 inverted-dropout multiplier for one dropout site (all ones when drop is None or p = 0).
-    drop = dict(p=..., seed=..., step=...); sites: GCN 1 = hidden; GAT 1 = X, 2 = hidden."""
+    drop = dict(p=..., seed=..., step=...[, attn_p=...]); sites: GCN 1 = hidden; GAT 1 = X, 2 = hidden, 3 / 4 =
+    layer-1 / layer-2 attention (E x H, by user edge id)."""
     if not drop or drop["p"] == 0.0:
         return None
     return oracle.dropout_mask(drop["seed"], site, drop["step"], M, F, drop["p"])
@@ -38,21 +39,21 @@ def gcn2(ip, ix, X, lab, p, acts=None, drop=None):
     return loss, {"W1": dW1, "b1": db1, "W2": dW2, "b2": db2}
 
 
-def _gat_layer_fwd(ip, ix, Xin, W, al, ar, b, act, H, F):
+def _gat_layer_fwd(ip, ix, Xin, W, al, ar, b, act, H, F, mask=None):
     N = Xin.shape[0]
     T = oracle.linear_fwd(Xin, W).reshape(N, H, F)
     el, er = oracle.gat_attn_proj(T, al, ar)
-    A, lse, _ = oracle.gat_fwd(ip, ix, T, el, er, 0.2)
+    A, lse, _ = oracle.gat_fwd(ip, ix, T, el, er, 0.2, mask=mask)
     Z = A.reshape(N, H * F) + b
     _gat_layer_fwd.lse = lse          # exposed to callers that want it (acts); not part of the return value
     return T, el, er, Z, oracle.act_fwd(act, Z)
 
 
-def _gat_layer_bwd(ip, ix, Xin, W, al, ar, T, el, er, Z, act, dY, H, F, need_dX):
+def _gat_layer_bwd(ip, ix, Xin, W, al, ar, T, el, er, Z, act, dY, H, F, need_dX, mask=None):
     N = Xin.shape[0]
     dZ = oracle.act_bwd(act, Z, dY)
     db = dZ.sum(0)
-    dT, dl, dr = oracle.gat_bwd(ip, ix, T, el, er, dZ.reshape(N, H, F), 0.2)
+    dT, dl, dr = oracle.gat_bwd(ip, ix, T, el, er, dZ.reshape(N, H, F), 0.2, mask=mask)
     dTp, dal, dar = oracle.gat_attn_proj_bwd(T, al, ar, dl, dr)
     dTt = (dT + dTp).reshape(N, H * F)
     dX, dW, _ = oracle.linear_bwd(Xin, W, dTt, need_dX=need_dX, need_db=False)
@@ -64,20 +65,24 @@ def gat2(ip, ix, X, lab, p, heads, hidden, acts=None, drop=None):
     C = p["W2"].shape[1]
     m0 = _mask(drop, 1, *X.shape)                    # feat_drop on the layer-1 input
     Xd = X if m0 is None else X * m0
-    T1, el1, er1, Z1, Y1 = _gat_layer_fwd(ip, ix, Xd, p["W1"], p["al1"], p["ar1"], p["b1"], "elu", heads, hidden)
+    E = int(ip[-1])
+    ad = {"p": drop["attn_p"], "seed": drop["seed"], "step": drop["step"]} if drop and drop.get("attn_p") else None
+    a1, a2 = _mask(ad, 3, E, heads), _mask(ad, 4, E, 1)   # attn_drop, by (user edge id, head)
+    T1, el1, er1, Z1, Y1 = _gat_layer_fwd(ip, ix, Xd, p["W1"], p["al1"], p["ar1"], p["b1"], "elu", heads, hidden,
+                                          a1)
     lse1 = _gat_layer_fwd.lse
     m1 = _mask(drop, 2, *Y1.shape)                   # feat_drop on the layer-2 input
     Y1d = Y1 if m1 is None else Y1 * m1
-    T2, el2, er2, Z2, Y2 = _gat_layer_fwd(ip, ix, Y1d, p["W2"], p["al2"], p["ar2"], p["b2"], "none", 1, C)
+    T2, el2, er2, Z2, Y2 = _gat_layer_fwd(ip, ix, Y1d, p["W2"], p["al2"], p["ar2"], p["b2"], "none", 1, C, a2)
     lse2 = _gat_layer_fwd.lse
     loss, dY2 = oracle.softmax_xent(Y2, lab)
     dY1, dW2, dal2, dar2, db2 = _gat_layer_bwd(ip, ix, Y1d, p["W2"], p["al2"], p["ar2"], T2, el2, er2, Z2, "none",
-                                               dY2, 1, C, True)
+                                               dY2, 1, C, True, a2)
     if m1 is not None:
         dY1 = dY1 * m1
     dZ2 = _gat_layer_bwd.dZ
     _, dW1, dal1, dar1, db1 = _gat_layer_bwd(ip, ix, Xd, p["W1"], p["al1"], p["ar1"], T1, el1, er1, Z1, "elu", dY1,
-                                             heads, hidden, False)
+                                             heads, hidden, False, a1)
     dZ1 = _gat_layer_bwd.dZ
     if acts is not None:
         acts.update(Y1=Y1, Y2=Y2,

@@ -359,9 +359,11 @@ static inline double lrelu(double x, double slope) { return x > 0.0 ? x : slope 
  *   A[v,h,:] = sum_u a_uv T[u,h,:];  lse[v,h] = log sum exp(e_uv)  (-inf for an empty row)
  * alpha (optional): alpha[e*H + h] for every edge, by edge id.
  */
+/* mask (optional, NEXT-3 attention dropout, reading #27): [E, H] multiplier of the attention weight of edge e
+ * (user edge id) in the aggregation, A = sum_e a_e mask_e T_u (the softmax itself is not masked) */
 void orc_gat_fwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices, int64_t H, int64_t F,
                  const double* T, const double* el, const double* er, double slope,
-                 const int64_t* rows, int64_t nrows, double* A, double* lse, double* alpha) {
+                 const int64_t* rows, int64_t nrows, double* A, double* lse, double* alpha, const double* mask) {
     (void)E;
     if (!rows) nrows = N;
     #pragma omp parallel for schedule(dynamic, 64)
@@ -383,7 +385,8 @@ void orc_gat_fwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* ind
                 int64_t u = indices[e];
                 double al = exp(lrelu(el[u * H + h] + er[v * H + h], slope) - m) / S;
                 if (alpha) alpha[e * H + h] = al;
-                for (int64_t f = 0; f < F; ++f) a[f] += al * T[(u * H + h) * F + f];
+                const double mk = mask ? mask[e * H + h] : 1.0;
+                for (int64_t f = 0; f < F; ++f) a[f] += al * mk * T[(u * H + h) * F + f];
             }
             lse[r * H + h] = m + log(S);
         }
@@ -398,10 +401,12 @@ void orc_gat_fwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* ind
  *   der[v,h]  = sum_{e in in(v)} ds_e
  * Pass 1 (all v) computes per-(v,h) softmax statistics and der; pass 2 evaluates the source-side
  * sums for `rows` (NULL => all).  dT/del are [nrows,...]; der is [N,H].
+ * With the optional attention-dropout mask of orc_gat_fwd, dA_e/d a_e = mask_e g_e: g_e is replaced by
+ * mask_e g_e in the Jacobian and dT[u] gets a_e mask_e dA[dst].
  */
 void orc_gat_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices, int64_t H, int64_t F,
                  const double* T, const double* el, const double* er, double slope, const double* dA,
-                 const int64_t* rows, int64_t nrows, double* dT, double* del, double* der) {
+                 const int64_t* rows, int64_t nrows, double* dT, double* del, double* der, const double* mask) {
     double* mx = (double*)malloc(sizeof(double) * (size_t)(N * H > 0 ? N * H : 1));
     double* sm = (double*)malloc(sizeof(double) * (size_t)(N * H > 0 ? N * H : 1));
     double* gb = (double*)malloc(sizeof(double) * (size_t)(N * H > 0 ? N * H : 1));
@@ -420,6 +425,7 @@ void orc_gat_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* ind
                 double al = exp(lrelu(el[u * H + h] + er[v * H + h], slope) - m) / S;
                 double g = 0.0;
                 for (int64_t f = 0; f < F; ++f) g += dA[(v * H + h) * F + f] * T[(u * H + h) * F + f];
+                if (mask) g *= mask[e * H + h];
                 gbar += al * g;
             }
             for (int64_t e = indptr[v]; e < indptr[v + 1]; ++e) {
@@ -428,6 +434,7 @@ void orc_gat_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* ind
                 double al = exp(lrelu(s, slope) - m) / S;
                 double g = 0.0;
                 for (int64_t f = 0; f < F; ++f) g += dA[(v * H + h) * F + f] * T[(u * H + h) * F + f];
+                if (mask) g *= mask[e * H + h];
                 dsum += al * (g - gbar) * (s > 0.0 ? 1.0 : slope);
             }
             mx[v * H + h] = m; sm[v * H + h] = S; gb[v * H + h] = gbar;
@@ -449,10 +456,11 @@ void orc_gat_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* ind
                 int64_t v = dst[oeid[p]];
                 double s = el[u * H + h] + er[v * H + h];
                 double al = exp(lrelu(s, slope) - mx[v * H + h]) / sm[v * H + h];
+                const double mk = mask ? mask[oeid[p] * H + h] : 1.0;
                 double g = 0.0;
                 for (int64_t f = 0; f < F; ++f) g += dA[(v * H + h) * F + f] * T[(u * H + h) * F + f];
-                dl += al * (g - gb[v * H + h]) * (s > 0.0 ? 1.0 : slope);
-                for (int64_t f = 0; f < F; ++f) o[f] += al * dA[(v * H + h) * F + f];
+                dl += al * (mk * g - gb[v * H + h]) * (s > 0.0 ? 1.0 : slope);
+                for (int64_t f = 0; f < F; ++f) o[f] += al * mk * dA[(v * H + h) * F + f];
             }
             del[r * H + h] = dl;
         }

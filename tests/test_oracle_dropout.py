@@ -81,7 +81,34 @@ def test_gcn2_and_gat2_with_dropout_fd():
           "W2": synth.uniform(17, (heads * hid, C)).astype(np.float64),
           "al2": synth.uniform(18, (1, C)).astype(np.float64), "ar2": synth.uniform(19, (1, C)).astype(np.float64),
           "b2": synth.uniform(20, (C,)).astype(np.float64) * .1}
-    _, g = model_ref.gat2(ip, ix, X, lab, pa, heads, hid, None, drop)
-    for k in pa:
-        fd = fd_grad(lambda: model_ref.gat2(ip, ix, X, lab, pa, heads, hid, None, drop)[0], pa[k])
-        assert rel_err(g[k], fd) < 1e-6, k
+    for d in (drop, dict(drop, attn_p=0.4), dict(drop, p=0.0, attn_p=0.6)):
+        _, g = model_ref.gat2(ip, ix, X, lab, pa, heads, hid, None, d)
+        for k in pa:
+            fd = fd_grad(lambda: model_ref.gat2(ip, ix, X, lab, pa, heads, hid, None, d)[0], pa[k])
+            assert rel_err(g[k], fd) < 1e-6, (d, k)
+
+
+def test_gat_attention_mask_layer():
+    """gat_fwd / gat_bwd with an attention mask: all-ones is the unmasked layer, all-zeros gives A = 0 and no T
+    gradient, and the masked layer's gradients match central differences."""
+    import synth
+    from conftest import rel_err
+    from test_oracle_layers import fd_grad, small_graph
+    ip, ix = small_graph(22, N=9, E=36)
+    N, H, F, E = 9, 2, 3, 36
+    T = synth.uniform(1, (N, H, F)).astype(np.float64)
+    el, er = synth.uniform(2, (N, H)).astype(np.float64), synth.uniform(3, (N, H)).astype(np.float64)
+    A0, l0, _ = oracle.gat_fwd(ip, ix, T, el, er)
+    A1, l1, _ = oracle.gat_fwd(ip, ix, T, el, er, mask=np.ones((E, H)))
+    np.testing.assert_array_equal(A0, A1)
+    np.testing.assert_array_equal(l0, l1)
+    Az, lz, _ = oracle.gat_fwd(ip, ix, T, el, er, mask=np.zeros((E, H)))
+    assert np.all(Az == 0) and np.array_equal(lz, l0)           # the softmax itself is not masked
+    mask = oracle.dropout_mask(9, 3, 0, E, H, 0.5)
+    R = synth.uniform(4, (N, H, F)).astype(np.float64)
+    f = lambda: (oracle.gat_fwd(ip, ix, T, el, er, mask=mask)[0] * R).sum()
+    dT, dl, dr = oracle.gat_bwd(ip, ix, T, el, er, R, mask=mask)
+    assert rel_err(dT, fd_grad(f, T)) < 1e-8
+    # del / der are the gradients w.r.t. el (source side) and er (destination side)
+    assert rel_err(dl, fd_grad(f, el)) < 1e-8
+    assert rel_err(dr, fd_grad(f, er)) < 1e-8
