@@ -44,6 +44,16 @@ extern "C" {
 #define SEASTAR_ABI_VERSION 1
 
 typedef struct seastar_graph_s* seastar_graph;   /* opaque, immutable after create */
+/* NEXT-3 dropout descriptor (reading #27): drop probability p (0 <= p < 1), the mask's site id
+ * and seed, and a device int32 step counter (or NULL = 0) read on the device so a captured CUDA graph draws a
+ * fresh mask every epoch.  keep(i) <=> (sm64(key ^ i) >> 40) >= round(p * 2^24),
+ * key = sm64(seed ^ sm64((site << 32) | step)), sm64 = splitmix64's output function. */
+typedef struct {
+    float p;
+    uint32_t site;
+    uint64_t seed;
+    const int32_t* step;
+} seastar_dropout_spec;
 typedef void* seastar_stream;                     /* cudaStream_t */
 
 typedef enum {
@@ -223,7 +233,10 @@ seastar_status seastar_gat_attn_proj(const float* T, int64_t M, int32_t H, int32
 seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float* el_all, const float* er_loc,
                                int32_t H, int32_t F, int64_t ldt, float slope, const float* bias, seastar_act act,
                                float* A_loc, float* Y_loc, float* lse_loc, float* B_loc, float* b_loc,
-                               seastar_stream stream);
+                               const seastar_dropout_spec* attn_drop, seastar_stream stream);
+/* (attn_drop: NULL, or NEXT-3 attention dropout -- see seastar_dropout_spec; the aggregation uses
+ *  a_e * m_e with m_e = keep(eid * H + h) / (1 - p), the softmax and lse are not masked.  With p > 0 the
+ *  generic chunked kernels run (H*F <= 128).  gat_bwd and gat_der must get the same spec.) */
 /* leading dimension (floats) of the packed per-destination backward record D: round_up(H*F, 4) + 4*H */
 int64_t seastar_gat_record_ld(int32_t H, int32_t F);
 /*
@@ -247,7 +260,7 @@ seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const 
  */
 seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float* el_loc, const float* D_all,
                                int32_t H, int32_t F, int64_t ldt, float slope, float* dT_loc, float* del_loc,
-                               seastar_stream stream);
+                               const seastar_dropout_spec* attn_drop, seastar_stream stream);
 /*
  * Fused destination-major pass over the forward CSR: der_loc[v,h] = sum_{e in in(v)} ds_e with ds_e
  * recomputed from the gathered T_all / el_all rows and v's own record D_loc[v] (no E x H array is
@@ -256,7 +269,8 @@ seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float*
  * der_loc [n_loc,H].
  */
 seastar_status seastar_gat_der(seastar_graph g, const float* T_all, const float* el_all, const float* D_loc,
-                               int32_t H, int32_t F, int64_t ldt, float slope, float* der_loc, seastar_stream stream);
+                               int32_t H, int32_t F, int64_t ldt, float slope, float* der_loc,
+                               const seastar_dropout_spec* attn_drop, seastar_stream stream);
 /*
  * Backward of seastar_gat_attn_proj over M rows:  dT[u,h,:] += del[u,h] a_l[h,:] + der[u,h] a_r[h,:];
  * da_l = sum_u del[u,h] T[u,h,:];  da_r = sum_u der[u,h] T[u,h,:]   (deterministic, via workspace of

@@ -67,11 +67,11 @@ _SIGS = {
     "seastar_gcn_fwd": ([_P, _P, _I64, _I64, _P, _P, _I32, _F, _P, _P, _P, _P, _P], _ST),
     "seastar_gcn_bwd": ([_P, _P, _I64, _I64, _P, _F, _P, _I32, _P, _P, _P, _P], _ST),
     "seastar_gat_attn_proj": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P], _ST),
-    "seastar_gat_fwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _I32, _P, _P, _P, _P, _P, _P], _ST),
+    "seastar_gat_fwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _I32, _P, _P, _P, _P, _P, _P, _P], _ST),
     "seastar_gat_record_ld": ([_I32, _I32], _I64),
     "seastar_gat_bwd_prep": ([_P, _P, _P, _I32, _P, _P, _P, _I32, _I32, _I64, _P, _P, _P, _P, _P], _ST),
-    "seastar_gat_bwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P, _P], _ST),
-    "seastar_gat_der": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P], _ST),
+    "seastar_gat_bwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P, _P, _P], _ST),
+    "seastar_gat_der": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P, _P], _ST),
     "seastar_gat_attn_proj_bwd": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P, _P, _P, _P, _SZ, _P], _ST),
     "seastar_gat_attn_proj_bwd_workspace": ([_I64, _I32, _I32], _SZ),
     "seastar_rgcn_fwd": ([_P, _P, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
@@ -250,11 +250,27 @@ def seastar_gat_attn_proj(T, M, H, F, ldt, a_l, a_r, el, er, stream=None) -> Non
           _dptr(el, "el"), _dptr(er, "er"), _stream(stream))
 
 
+class seastar_dropout_spec(ctypes.Structure):
+    """NEXT-3 dropout descriptor (include/seastar.h): p, site, seed, device step counter (or NULL)."""
+    _fields_ = [("p", ctypes.c_float), ("site", ctypes.c_uint32), ("seed", ctypes.c_uint64), ("step", ctypes.c_void_p)]
+
+
+def dropout_spec(p, site, seed, step=None):
+    """A seastar_dropout_spec (None when p == 0); step: a device int32 tensor (e.g. the Adam step counter)."""
+    if not p:
+        return None
+    return seastar_dropout_spec(float(p), int(site), int(seed), _dptr(step, "step"))
+
+
+def _spec(d):
+    return ctypes.addressof(d) if d is not None else None
+
+
 def seastar_gat_fwd(g, T_all, el_all, er_loc, H, F, ldt, slope, bias, act, A_loc, Y_loc, lse_loc, B_loc=None,
-                    b_loc=None, stream=None) -> None:
+                    b_loc=None, stream=None, attn_drop=None) -> None:
     _call("seastar_gat_fwd", g, _dptr(T_all, "T"), _dptr(el_all, "el"), _dptr(er_loc, "er"), H, F, ldt,
           float(slope), _dptr(bias, "bias"), _act(act), _dptr(A_loc, "A"), _dptr(Y_loc, "Y"), _dptr(lse_loc, "lse"),
-          _dptr(B_loc, "B"), _dptr(b_loc, "b"), _stream(stream))
+          _dptr(B_loc, "B"), _dptr(b_loc, "b"), _spec(attn_drop), _stream(stream))
 
 
 def seastar_gat_record_ld(H, F) -> int:
@@ -268,14 +284,14 @@ def seastar_gat_bwd_prep(g, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, H, F, ld
           _dptr(b_loc, "b"), _dptr(der_loc, "der"), _stream(stream))
 
 
-def seastar_gat_bwd(g, T_loc, el_loc, D_all, H, F, ldt, slope, dT_loc, del_loc, stream=None) -> None:
+def seastar_gat_bwd(g, T_loc, el_loc, D_all, H, F, ldt, slope, dT_loc, del_loc, stream=None, attn_drop=None) -> None:
     _call("seastar_gat_bwd", g, _dptr(T_loc, "T"), _dptr(el_loc, "el"), _dptr(D_all, "D"), H, F, ldt, float(slope),
-          _dptr(dT_loc, "dT"), _dptr(del_loc, "del"), _stream(stream))
+          _dptr(dT_loc, "dT"), _dptr(del_loc, "del"), _spec(attn_drop), _stream(stream))
 
 
-def seastar_gat_der(g, T_all, el_all, D_loc, H, F, ldt, slope, der_loc, stream=None) -> None:
+def seastar_gat_der(g, T_all, el_all, D_loc, H, F, ldt, slope, der_loc, stream=None, attn_drop=None) -> None:
     _call("seastar_gat_der", g, _dptr(T_all, "T"), _dptr(el_all, "el"), _dptr(D_loc, "D"), H, F, ldt, float(slope),
-          _dptr(der_loc, "der"), _stream(stream))
+          _dptr(der_loc, "der"), _spec(attn_drop), _stream(stream))
 
 
 def seastar_gat_attn_proj_bwd_workspace(M, H, F) -> int:

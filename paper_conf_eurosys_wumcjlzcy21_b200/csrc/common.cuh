@@ -1,5 +1,6 @@
 // common.cuh -- shared internals of libseastar.so (sm_100a).  Not part of the ABI.
 #pragma once
+#include <cmath>
 
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -149,6 +150,24 @@ __device__ __forceinline__ float act_grad_from_y(int act, float y) {
 }
 
 inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+// NEXT-3 dropout generator (reading #27): splitmix64's output function; a mask element keeps
+// iff (sm64(key ^ i) >> 40) >= thr with key = sm64(seed ^ sm64((site << 32) | step))
+__device__ __forceinline__ uint64_t sm64(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+__device__ __forceinline__ uint64_t drop_key(uint64_t seed, uint32_t site, const int32_t* step) {
+    const uint32_t st = step ? (uint32_t)__ldg(step) : 0u;
+    return sm64(seed ^ sm64(((uint64_t)site << 32) | st));
+}
+__device__ __forceinline__ float drop_mult(uint64_t key, uint64_t i, uint32_t thr, float scale) {
+    return (sm64(key ^ i) >> 40) >= thr ? scale : 0.f;
+}
+inline uint32_t drop_threshold(float p) { return (uint32_t)llround((double)p * 16777216.0); }
+inline float drop_scale(float p) { return (float)(1.0 / (1.0 - (double)p)); }
 
 // ----------------------------------------------------------------------------------------------
 // L2 residency of the gathered table.  Every edge of a graph kernel gathers a row of one table

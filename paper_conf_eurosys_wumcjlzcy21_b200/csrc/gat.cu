@@ -58,6 +58,8 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
     const float erv = (valid && active) ? __ldg(a.er + v * a.H + h) : 0.f;
 
     const bool SB = a.B != nullptr;     // fallback path: runtime flag
+    const bool DROP = a.deid != nullptr;
+    const uint64_t dkey = DROP ? drop_key(a.dseed, a.dsite, a.dstep) : 0ull;
     float m = -INFINITY, ssum = 0.f, acc[VEC], pacc[VEC], psum = 0.f;
 #pragma unroll
     for (int i = 0; i < VEC; ++i) acc[i] = pacc[i] = 0.f;
@@ -70,14 +72,17 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
 #pragma unroll
         for (int j0 = 0; j0 < L; j0 += UB) {
             if (j0 * S >= n) break;
-            float z[UB], val[UB][VEC];
+            float z[UB], val[UB][VEC], mk[UB];
 #pragma unroll
             for (int jj = 0; jj < UB; ++jj) {
                 const int k = (j0 + jj) * S + slot;
                 const int u = __shfl_sync(gmask, my, k & (RL - 1), RL);
+                mk[jj] = 1.f;
                 if (k < n && active) {
                     z[jj] = lrelu(__ldg(a.el + (int64_t)u * a.H + h) + erv, a.slope);
                     load_vec<VEC>(a.T + (int64_t)u * a.ld + col, val[jj]);
+                    if (DROP)
+                        mk[jj] = drop_mult(dkey, (uint64_t)__ldg(a.deid + base + k) * a.H + h, a.dthr, a.dscale);
                 } else {
                     z[jj] = -INFINITY;
 #pragma unroll
@@ -98,10 +103,11 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
                 ssum += p;
                 const float pp = (SB && z[jj] > 0.f) ? p : 0.f;
                 psum += pp;
+                const float pm = p * mk[jj], ppm = pp * mk[jj];     // attention dropout: weights only
 #pragma unroll
                 for (int i = 0; i < VEC; ++i) {
-                    acc[i] = fmaf(p, val[jj][i], acc[i]);
-                    pacc[i] = fmaf(pp, val[jj][i], pacc[i]);
+                    acc[i] = fmaf(pm, val[jj][i], acc[i]);
+                    pacc[i] = fmaf(ppm, val[jj][i], pacc[i]);
                 }
             }
             m = mb;
@@ -194,6 +200,8 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
     float acc[VEC], dl = 0.f;
 #pragma unroll
     for (int i = 0; i < VEC; ++i) acc[i] = 0.f;
+    const bool DROP = a.deid != nullptr;
+    const uint64_t dkey = DROP ? drop_key(a.dseed, a.dsite, a.dstep) : 0ull;
 
     int nxt = (gl < end - beg) ? __ldcs(a.nbr + beg + gl) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += RL) {
@@ -237,9 +245,12 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
                 if (k < n && active) {
                     const float s = elu + er[jj];
                     const float al = expf(lrelu(s, a.slope) - lse[jj]);
-                    dl += al * (g - cv[jj]) * (s > 0.f ? 1.f : a.slope);
+                    const float mk =
+                        DROP ? drop_mult(dkey, (uint64_t)__ldg(a.deid + base + k) * a.H + h, a.dthr, a.dscale) : 1.f;
+                    dl += al * (mk * g - cv[jj]) * (s > 0.f ? 1.f : a.slope);
+                    const float alm = al * mk;
 #pragma unroll
-                    for (int i = 0; i < VEC; ++i) acc[i] = fmaf(al, dA[jj][i], acc[i]);
+                    for (int i = 0; i < VEC; ++i) acc[i] = fmaf(alm, dA[jj][i], acc[i]);
                 }
             }
         }
@@ -296,6 +307,8 @@ __global__ void __launch_bounds__(256) k_gat_der(const GatBwdArgs a) {
     for (int i = 0; i < VEC; ++i)
         if (!(valid && active) || col + i >= W) d[i] = 0.f;
     float dr = 0.f;
+    const bool DROP = a.deid != nullptr;
+    const uint64_t dkey = DROP ? drop_key(a.dseed, a.dsite, a.dstep) : 0ull;
     int nxt = (gl < end - beg) ? __ldcs(a.nbr + beg + gl) : 0;   // index prefetch (gcn.cu)
     for (int base = beg; base < end; base += RL) {
         const int n = min(RL, end - base);
@@ -336,7 +349,9 @@ __global__ void __launch_bounds__(256) k_gat_der(const GatBwdArgs a) {
                 if (k < n && active) {
                     const float s = elu[jj] + erv;
                     const float al = expf(lrelu(s, a.slope) - lsev);
-                    dr += al * (g - cvv) * (s > 0.f ? 1.f : a.slope);
+                    const float mk =
+                        DROP ? drop_mult(dkey, (uint64_t)__ldg(a.deid + base + k) * a.H + h, a.dthr, a.dscale) : 1.f;
+                    dr += al * (mk * g - cvv) * (s > 0.f ? 1.f : a.slope);
                 }
             }
         }
@@ -571,7 +586,7 @@ seastar_status seastar_gat_attn_proj(const float* T, int64_t M, int32_t H, int32
 seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float* el_all, const float* er_loc,
                                int32_t H, int32_t F, int64_t ldt, float slope, const float* bias, seastar_act act,
                                float* A_loc, float* Y_loc, float* lse_loc, float* B_loc, float* b_loc,
-                               seastar_stream stream) {
+                               const seastar_dropout_spec* attn_drop, seastar_stream stream) {
     SS_ARG(g && T_all && el_all && er_loc && A_loc && Y_loc && lse_loc, "gat_fwd: NULL argument");
     SS_ARG((B_loc == nullptr) == (b_loc == nullptr), "gat_fwd: pass both B_loc and b_loc or neither");
     SS_ARG(!B_loc || (aligned16(B_loc) == aligned16(A_loc)), "gat_fwd: B_loc must be aligned like A_loc");
@@ -587,8 +602,10 @@ seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float*
     a.H = H; a.F = F; a.ld = ldt; a.slope = slope; a.bias = bias; a.act = act;
     a.A = A_loc; a.Y = Y_loc; a.lse = lse_loc; a.B = B_loc; a.bsum = b_loc;
     a.row_begin = 0; a.row_end = g->fwd.n_rows;
-    if (launch_gat_fwd_hpl(a, s)) return check_launch("k_gat_fwd_hpl");
-    if (launch_gat_fwd_h1(a, g->fwd.bucket_rows[1], g->fwd.n_rows, s)) return check_launch("k_gat_fwd_h1");
+    SS_ARG(!attn_drop || (attn_drop->p >= 0.f && attn_drop->p < 1.f), "gat_fwd: need 0 <= attn_drop->p < 1");
+    set_attn_drop(a, attn_drop, g->fwd.eid);
+    if (!a.deid && launch_gat_fwd_hpl(a, s)) return check_launch("k_gat_fwd_hpl");
+    if (!a.deid && launch_gat_fwd_h1(a, g->fwd.bucket_rows[1], g->fwd.n_rows, s)) return check_launch("k_gat_fwd_h1");
     const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_all) && aligned16(A_loc) &&
                       aligned16(Y_loc);
     const int VEC = vec4 ? 4 : 1;
@@ -620,7 +637,7 @@ seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const 
 
 seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float* el_loc, const float* D_all,
                                int32_t H, int32_t F, int64_t ldt, float slope, float* dT_loc, float* del_loc,
-                               seastar_stream stream) {
+                               const seastar_dropout_spec* attn_drop, seastar_stream stream) {
     SS_ARG(g && T_loc && el_loc && D_all && dT_loc && del_loc, "gat_bwd: NULL argument");
     SS_ARG(ldt < (int64_t(1) << 31), "gat_bwd: ldt must be < 2^31");
     SS_ARG(H >= 1 && F >= 1 && ldt >= (int64_t)H * F, "gat_bwd: bad sizes");
@@ -634,8 +651,11 @@ seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float*
     a.dT = dT_loc; a.del = del_loc;
     ScopedL2Window win(D_all, (size_t)g->N * a.ldd * sizeof(float));
     a.row_begin = 0; a.row_end = g->rev.n_rows;
-    if (launch_gat_bwd_hpl(a, s)) return check_launch("k_gat_bwd_hpl");
-    if (launch_gat_bwd_h1(a, g->rev.bucket_rows[1], g->rev.n_rows, false, s)) return check_launch("k_gat_bwd_h1");
+    SS_ARG(!attn_drop || (attn_drop->p >= 0.f && attn_drop->p < 1.f), "gat_bwd: need 0 <= attn_drop->p < 1");
+    set_attn_drop(a, attn_drop, g->rev.eid);
+    if (!a.deid && launch_gat_bwd_hpl(a, s)) return check_launch("k_gat_bwd_hpl");
+    if (!a.deid && launch_gat_bwd_h1(a, g->rev.bucket_rows[1], g->rev.n_rows, false, s))
+        return check_launch("k_gat_bwd_h1");
     const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_loc) && aligned16(D_all) &&
                       aligned16(dT_loc);
     const int VEC = vec4 ? 4 : 1;
@@ -647,7 +667,8 @@ seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float*
 }
 
 seastar_status seastar_gat_der(seastar_graph g, const float* T_all, const float* el_all, const float* D_loc, int32_t H,
-                               int32_t F, int64_t ldt, float slope, float* der_loc, seastar_stream stream) {
+                               int32_t F, int64_t ldt, float slope, float* der_loc,
+                               const seastar_dropout_spec* attn_drop, seastar_stream stream) {
     SS_ARG(g && T_all && el_all && D_loc && der_loc, "gat_der: NULL argument");
     SS_ARG(ldt < (int64_t(1) << 31), "gat_der: ldt must be < 2^31");
     SS_ARG(H >= 1 && F >= 1 && ldt >= (int64_t)H * F, "gat_der: bad sizes");
@@ -660,8 +681,11 @@ seastar_status seastar_gat_der(seastar_graph g, const float* T_all, const float*
     a.H = H; a.F = F; a.ldt = ldt; a.ldd = seastar_gat_record_ld(H, F); a.slope = slope;
     a.der = der_loc;
     a.row_begin = 0; a.row_end = g->fwd.n_rows;
-    if (launch_gat_der_hpl(a, s)) return check_launch("k_gat_der_hpl");
-    if (launch_gat_bwd_h1(a, g->fwd.bucket_rows[1], g->fwd.n_rows, true, s)) return check_launch("k_gat_der_h1");
+    SS_ARG(!attn_drop || (attn_drop->p >= 0.f && attn_drop->p < 1.f), "gat_der: need 0 <= attn_drop->p < 1");
+    set_attn_drop(a, attn_drop, g->fwd.eid);
+    if (!a.deid && launch_gat_der_hpl(a, s)) return check_launch("k_gat_der_hpl");
+    if (!a.deid && launch_gat_bwd_h1(a, g->fwd.bucket_rows[1], g->fwd.n_rows, true, s))
+        return check_launch("k_gat_der_h1");
     const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_all) && aligned16(D_loc);
     const int VEC = vec4 ? 4 : 1;
     const int C = (H * F + VEC - 1) / VEC;

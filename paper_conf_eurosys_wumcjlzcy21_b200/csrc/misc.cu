@@ -199,14 +199,7 @@ __global__ void __launch_bounds__(256) k_adam(float* __restrict__ p, const float
 
 __global__ void k_step_inc(int32_t* c) { *c += 1; }
 
-// NEXT-3 dropout (reading #27): splitmix64 output function, counter = global element index
-__device__ __forceinline__ uint64_t sm64(uint64_t z) {
-    z += 0x9E3779B97F4A7C15ull;
-    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
-    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
-    return z ^ (z >> 31);
-}
-
+// NEXT-3 dropout (reading #27): counter = global element index (sm64: common.cuh)
 __global__ void __launch_bounds__(256) k_dropout(const float* X, int64_t M, uint32_t F, int64_t ldx, int64_t row0,
                                                  uint32_t thr, float scale, uint64_t seed, uint32_t site,
                                                  const int32_t* __restrict__ step, float* Y, int64_t ldy) {
@@ -287,8 +280,8 @@ seastar_status seastar_dropout(const float* X, int64_t M, int64_t F, int64_t ldx
     SS_ARG(X != Y || ldx == ldy, "dropout: in place needs ldx == ldy");
     SS_TRY(check_device());
     if (M == 0) return SEASTAR_OK;
-    const uint32_t thr = (uint32_t)llround((double)p * 16777216.0);
-    const float scale = (float)(1.0 / (1.0 - (double)p));
+    const uint32_t thr = drop_threshold(p);
+    const float scale = drop_scale(p);
     const int64_t n = M * F;
     int64_t blocks = (n + 255) / 256;
     const int64_t cap = 16 * (int64_t)num_sms();

@@ -249,7 +249,7 @@ class GAT2:
 
     def __init__(self, g: Graph, X_loc: torch.Tensor, labels_loc: torch.Tensor, params: dict, heads: int,
                  hidden: int, lr=0.005, slope=0.2, comm: Comm | None = None, n_pad_rows: int | None = None,
-                 save_der_factors: bool = True, dropout: float = 0.0, seed: int = 0):
+                 save_der_factors: bool = True, dropout: float = 0.0, seed: int = 0, attn_dropout: float = 0.0):
         self.g, self.X, self.lab, self.lr, self.slope = g, X_loc, labels_loc, lr, slope
         self.drop_p, self.drop_seed = float(dropout), int(seed)     # NEXT-3: feat_drop on both layer inputs
         self.save_B = save_der_factors
@@ -264,6 +264,9 @@ class GAT2:
         shapes = {"W1": (self.Fin, self.W1w), "al1": (heads, hidden), "ar1": (heads, hidden), "b1": (self.W1w,),
                   "W2": (self.W1w, self.C), "al2": (1, self.C), "ar2": (1, self.C), "b2": (self.C,)}
         self.P = _Params(shapes, params, dev)
+        # NEXT-3 attn_drop (sites 3 / 4, by user edge id and head; the generic chunked GAT kernels run)
+        self.ad = {"1": L.dropout_spec(attn_dropout, 3, seed, self.P.step),
+                   "2": L.dropout_spec(attn_dropout, 4, seed, self.P.step)}
         n, W1w, C = _local_rows(self), self.W1w, self.C
         self.ld1, self.ld2 = _ld(W1w), _ld(C)
         e = lambda r, c: torch.zeros((r, c), device=dev)
@@ -315,7 +318,7 @@ class GAT2:
         self._gathered1 = (T1_all, el1_all)
         self._t("gat_fwd1")
         L.seastar_gat_fwd(g.handle, T1_all, el1_all, self.er1, H, F, self.ld1, self.slope, p.p("b1"), "elu", self.A1,
-                          self.Y1, self.lse1, self.B1, self.bs1)
+                          self.Y1, self.lse1, self.B1, self.bs1, attn_drop=self.ad["1"])
         self._t("gat_fwd1_end")
         if self.drop_p > 0:
             L.seastar_dropout(self.Y1, n, W, self.ld1, g.row_begin, self.drop_p, self.drop_seed, 2, p.step, self.Y1d,
@@ -327,7 +330,7 @@ class GAT2:
         self._gathered2 = (T2_all, el2_all)
         self._t("gat_fwd2")
         L.seastar_gat_fwd(g.handle, T2_all, el2_all, self.er2, 1, C, self.ld2, self.slope, p.p("b2"), "none", self.A2,
-                          self.Y2, self.lse2, self.B2, self.bs2)
+                          self.Y2, self.lse2, self.B2, self.bs2, attn_drop=self.ad["2"])
         self._t("gat_fwd2_end")
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
         L.seastar_softmax_xent(self.Y2, n, self.g.N, C, self.ld2, self.lab, self.loss, self.dY2, self.ld2, ws,
@@ -343,11 +346,12 @@ class GAT2:
         L.seastar_colsum(D, n, H * F, ldd, db, ws, ws.numel())       # db = sum_v dA[v] (dA = first H*F columns)
         D_all = self.comm.all_gather(D_all_buf, D)
         self._t(f"gat_bwd{tag}")
-        L.seastar_gat_bwd(g.handle, T, el, D_all, H, F, T_loc_ld, self.slope, dT, del_)
+        L.seastar_gat_bwd(g.handle, T, el, D_all, H, F, T_loc_ld, self.slope, dT, del_, attn_drop=self.ad[tag])
         self._t(f"gat_bwd{tag}_end")
         if B is None:
             self._t(f"gat_der{tag}")
-            L.seastar_gat_der(g.handle, gathered[0], gathered[1], D, H, F, T_loc_ld, self.slope, der)
+            L.seastar_gat_der(g.handle, gathered[0], gathered[1], D, H, F, T_loc_ld, self.slope, der,
+                              attn_drop=self.ad[tag])
             self._t(f"gat_der{tag}_end")
         L.seastar_gat_attn_proj_bwd(T, n, H, F, T_loc_ld, al, ar, del_, der, dT, dal, dar, ws, ws.numel())
 

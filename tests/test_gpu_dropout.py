@@ -128,3 +128,49 @@ def test_gcn2_dropout_partitioned(env):
     assert abs(sum(r[0] for r in res) - rl) <= TOL * abs(rl)
     for k in rg:
         assert rel_err(res[0][1][k], rg[k].reshape(res[0][1][k].shape)) <= TOL, k
+
+
+@pytest.mark.parametrize("H,F", [(8, 8), (1, 41), (4, 16)])
+def test_gat_fwd_attn_dropout(env, H, F):
+    """NEXT-3 attention dropout in the fused forward: A = sum_e a_e m_e T_u with m_e keyed by (user edge id, head);
+    the softmax statistics (lse) are not masked."""
+    torch, L, Graph = env["torch"], env["L"], env["Graph"]
+    from helpers import hub_graph
+    ip, ix = hub_graph(N=2500, E_dir=20000, seed=64)
+    N, E = len(ip) - 1, len(ix)
+    g = Graph(ip, ix)
+    T = synth.uniform(1, (N, H, F))
+    el, er = synth.uniform(2, (N, H)), synth.uniform(3, (N, H))
+    ld = (H * F + 3) // 4 * 4
+    Tp = np.zeros((N, ld), np.float32)
+    Tp[:, :H * F] = T.reshape(N, H * F)
+    st = torch.tensor([4], dtype=torch.int32, device="cuda")
+    spec = L.dropout_spec(0.5, 3, 77, st)
+    d = lambda a: torch.from_numpy(np.ascontiguousarray(a, np.float32)).cuda()
+    A = torch.zeros((N, ld), device="cuda")
+    Y = torch.zeros((N, ld), device="cuda")
+    lse = torch.zeros((N, H), device="cuda")
+    L.seastar_gat_fwd(g.handle, d(Tp), d(el), d(er), H, F, ld, 0.2, None, "none", A, Y, lse, attn_drop=spec)
+    mask = oracle.dropout_mask(77, 3, 4, E, H, 0.5)
+    rA, rl, _ = oracle.gat_fwd(ip, ix, T, el, er, 0.2, mask=mask)
+    assert rel_err(A.cpu().numpy()[:, :H * F], rA.reshape(N, H * F)) <= TOL
+    lg = lse.cpu().numpy()
+    fin = np.isfinite(rl)
+    assert np.array_equal(np.isfinite(lg), fin) and rel_err(lg[fin], rl[fin]) <= TOL
+
+
+@pytest.mark.parametrize("save_B", [True, False])
+def test_gat2_attn_dropout(env, save_B):
+    """DGL's GAT defaults: feat_drop 0.6 on both layer inputs and attn_drop 0.6 on both layers' attention."""
+    torch, models, Graph = env["torch"], env["models"], env["Graph"]
+    ip, ix = synth.powerlaw_sym(1500, 12000, 0.6, 65)
+    N, Fin, heads, hid, C = 1500, 100, 8, 8, 41
+    X, lab = synth.uniform(11, (N, Fin)), synth.labels(12, N, C)
+    p = {"W1": synth.glorot(13, Fin, heads * hid), "al1": synth.uniform(14, (heads, hid), -0.5, 0.5),
+         "ar1": synth.uniform(15, (heads, hid), -0.5, 0.5), "b1": synth.uniform(16, (heads * hid,), -0.1, 0.1),
+         "W2": synth.glorot(17, heads * hid, C), "al2": synth.uniform(18, (1, C), -0.5, 0.5),
+         "ar2": synth.uniform(19, (1, C), -0.5, 0.5), "b2": synth.uniform(20, (C,), -0.1, 0.1)}
+    m = models.GAT2(Graph(ip, ix), torch.from_numpy(X).cuda(), torch.from_numpy(lab).cuda(), p, heads, hid,
+                    dropout=0.6, attn_dropout=0.6, seed=8, save_der_factors=save_B)
+    _check(m, *model_ref.gat2(ip, ix, X, lab, {k: v.astype(np.float64) for k, v in p.items()}, heads, hid,
+                              drop={"p": 0.6, "attn_p": 0.6, "seed": 8, "step": 0}))
