@@ -73,8 +73,8 @@ def _L():
             "orc_act_bwd": ([ctypes.c_int, _I, _P, _P, _P], None),
             "orc_linear_fwd": ([_I, _I, _I, _P, _P, _P, _P], None),
             "orc_linear_bwd": ([_I, _I, _I, _P, _P, _P, _P, _P, _P], None),
-            "orc_gcn_aggregate": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P], None),
-            "orc_gcn_aggregate_T": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P], None),
+            "orc_gcn_aggregate": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P, _P], None),
+            "orc_gcn_aggregate_T": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P, _P], None),
             "orc_gat_attn_proj": ([_I, _I, _I, _P, _P, _P, _P, _P], None),
             "orc_gat_fwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _I, _P, _P, _P, _P], None),
             "orc_gat_bwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _P, _I, _P, _P, _P, _P], None),
@@ -193,8 +193,8 @@ def linear_bwd(X, W, dY, need_dX=True, need_dW=True, need_db=True):
 # ------------------------------------------------------------------------------------------
 # GCN / APPNP
 # ------------------------------------------------------------------------------------------
-def gcn_aggregate(indptr, indices, H, src_norm=None, dst_norm=None, rows=None):
-    indptr, indices, H = _i64(indptr), _i64(indices), _f64(H)
+def gcn_aggregate(indptr, indices, H, src_norm=None, dst_norm=None, rows=None, edge_w=None):
+    indptr, indices, H, edge_w = _i64(indptr), _i64(indices), _f64(H), _f64(edge_w)
     N = indptr.size - 1
     F = H.shape[1]
     rows = _i64(rows)
@@ -202,12 +202,12 @@ def gcn_aggregate(indptr, indices, H, src_norm=None, dst_norm=None, rows=None):
     out = np.empty((nrows, F))
     sn, dn = _f64(src_norm), _f64(dst_norm)     # keep the converted arrays alive across the C call
     _L().orc_gcn_aggregate(N, int(indptr[-1]), _p(indptr), _p(indices), F, _p(H), _p(sn), _p(dn), _p(rows), nrows,
-                           _p(out))
+                           _p(out), _p(edge_w))
     return out
 
 
-def gcn_aggregate_T(indptr, indices, G, src_norm=None, dst_norm=None, rows=None):
-    indptr, indices, G = _i64(indptr), _i64(indices), _f64(G)
+def gcn_aggregate_T(indptr, indices, G, src_norm=None, dst_norm=None, rows=None, edge_w=None):
+    indptr, indices, G, edge_w = _i64(indptr), _i64(indices), _f64(G), _f64(edge_w)
     N = indptr.size - 1
     F = G.shape[1]
     rows = _i64(rows)
@@ -215,7 +215,7 @@ def gcn_aggregate_T(indptr, indices, G, src_norm=None, dst_norm=None, rows=None)
     out = np.empty((nrows, F))
     sn, dn = _f64(src_norm), _f64(dst_norm)     # keep the converted arrays alive across the C call
     _L().orc_gcn_aggregate_T(N, int(indptr[-1]), _p(indptr), _p(indices), F, _p(G), _p(sn), _p(dn), _p(rows),
-                             nrows, _p(out))
+                             nrows, _p(out), _p(edge_w))
     return out
 
 
@@ -245,28 +245,31 @@ def gcn_layer_bwd(indptr, indices, X, W, Zpre, act, src_norm, dst_norm, dY, need
     return dX, dW, db
 
 
-def appnp_fwd(indptr, indices, H0, K, alpha, norm=None):
+def appnp_fwd(indptr, indices, H0, K, alpha, norm=None, edge_masks=None):
     """APPNP propagation [38]: Z^0 = H0, Z^{k+1} = (1-a) * n * sum_in n_u Z^k_u + a * H0.
-    norm defaults to in-degree^-1/2 on both sides (DGL APPNPConv; reading in DESIGN.md)."""
+    norm defaults to in-degree^-1/2 on both sides (DGL APPNPConv; reading in DESIGN.md).
+    edge_masks: optional list of K [E] edge-dropout multipliers (by user edge id), one per step (NEXT-3)."""
     H0 = _f64(H0)
     if norm is None:
         norm, _ = degree_norms(indptr, indices)
     Z = H0.copy()
-    for _ in range(K):
-        Z = (1.0 - alpha) * gcn_aggregate(indptr, indices, Z, norm, norm) + alpha * H0
+    for k in range(K):
+        w = None if edge_masks is None else edge_masks[k]
+        Z = (1.0 - alpha) * gcn_aggregate(indptr, indices, Z, norm, norm, edge_w=w) + alpha * H0
     return Z
 
 
-def appnp_bwd(indptr, indices, dZ, K, alpha, norm=None):
-    """VJP of appnp_fwd w.r.t. H0 (reversing the recurrence)."""
+def appnp_bwd(indptr, indices, dZ, K, alpha, norm=None, edge_masks=None):
+    """VJP of appnp_fwd w.r.t. H0 (reversing the recurrence; step k's edge mask in reverse order)."""
     dZ = _f64(dZ)
     if norm is None:
         norm, _ = degree_norms(indptr, indices)
     G = dZ.copy()
     dH0 = np.zeros_like(dZ)
-    for _ in range(K):
+    for k in reversed(range(K)):
         dH0 += alpha * G
-        G = (1.0 - alpha) * gcn_aggregate_T(indptr, indices, G, norm, norm)
+        w = None if edge_masks is None else edge_masks[k]
+        G = (1.0 - alpha) * gcn_aggregate_T(indptr, indices, G, norm, norm, edge_w=w)
     return dH0 + G
 
 

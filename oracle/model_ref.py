@@ -93,13 +93,19 @@ def gat2(ip, ix, X, lab, p, heads, hidden, acts=None, drop=None):
     return loss, {"W1": dW1, "al1": dal1, "ar1": dar1, "b1": db1, "W2": dW2, "al2": dal2, "ar2": dar2, "b2": db2}
 
 
-def appnp(ip, ix, X, lab, p, K, alpha, acts=None):
+def appnp(ip, ix, X, lab, p, K, alpha, acts=None, drop=None):
+    """drop: dict(edge_p=..., seed=..., step=...): DGL APPNPConv's edge_drop, a fresh [E] mask per propagation
+    step k (site 16 + k, by user edge id)."""
     Z1 = oracle.linear_fwd(X, p["W1"], p["b1"])
     Hh = oracle.act_fwd("relu", Z1)
     H0 = oracle.linear_fwd(Hh, p["W2"], p["b2"])
-    Z = oracle.appnp_fwd(ip, ix, H0, K, alpha)
+    masks = None
+    if drop and drop.get("edge_p"):
+        E = int(ip[-1])
+        masks = [oracle.dropout_mask(drop["seed"], 16 + k, drop["step"], E, 1, drop["edge_p"])[:, 0] for k in range(K)]
+    Z = oracle.appnp_fwd(ip, ix, H0, K, alpha, edge_masks=masks)
     loss, dZ = oracle.softmax_xent(Z, lab)
-    dH0 = oracle.appnp_bwd(ip, ix, dZ, K, alpha)
+    dH0 = oracle.appnp_bwd(ip, ix, dZ, K, alpha, edge_masks=masks)
     dHh, dW2, db2 = oracle.linear_bwd(Hh, p["W2"], dH0)
     dZ1 = oracle.act_bwd("relu", Z1, dHh)
     _, dW1, db1 = oracle.linear_bwd(X, p["W1"], dZ1, need_dX=False)

@@ -286,9 +286,10 @@ void orc_linear_bwd(int64_t M, int64_t K, int64_t Nout, const double* X, const d
 /* ------------------------------------------------------------------------------------------ */
 
 /* out[r,:] = dst_norm[v] * sum_{e in in(v)} src_norm[src(e)] * H[src(e),:],  v = rows[r] */
+/* edge_w (optional, NEXT-3 edge dropout, reading #27): [E] multiplier of each edge's message by user edge id */
 void orc_gcn_aggregate(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices, int64_t F,
                        const double* H, const double* src_norm, const double* dst_norm,
-                       const int64_t* rows, int64_t nrows, double* out) {
+                       const int64_t* rows, int64_t nrows, double* out, const double* edge_w) {
     (void)E;
     if (!rows) nrows = N;
     #pragma omp parallel for schedule(dynamic, 64)
@@ -299,6 +300,7 @@ void orc_gcn_aggregate(int64_t N, int64_t E, const int64_t* indptr, const int64_
         for (int64_t e = indptr[v]; e < indptr[v + 1]; ++e) {
             int64_t u = indices[e];
             double w = src_norm ? src_norm[u] : 1.0;
+            if (edge_w) w *= edge_w[e];
             for (int64_t f = 0; f < F; ++f) o[f] += w * H[u * F + f];
         }
         double d = dst_norm ? dst_norm[v] : 1.0;
@@ -310,7 +312,7 @@ void orc_gcn_aggregate(int64_t N, int64_t E, const int64_t* indptr, const int64_
  * out[r,:] = src_norm[u] * sum_{e in out(u)} dst_norm[dst(e)] * G[dst(e),:],  u = rows[r] */
 void orc_gcn_aggregate_T(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices, int64_t F,
                          const double* G, const double* src_norm, const double* dst_norm,
-                         const int64_t* rows, int64_t nrows, double* out) {
+                         const int64_t* rows, int64_t nrows, double* out, const double* edge_w) {
     int64_t* dst = dst_of_edges(N, E, indptr);
     int64_t *optr, *oeid;
     out_adjacency(N, E, indices, &optr, &oeid);
@@ -323,6 +325,7 @@ void orc_gcn_aggregate_T(int64_t N, int64_t E, const int64_t* indptr, const int6
         for (int64_t p = optr[u]; p < optr[u + 1]; ++p) {
             int64_t v = dst[oeid[p]];
             double w = dst_norm ? dst_norm[v] : 1.0;
+            if (edge_w) w *= edge_w[oeid[p]];
             for (int64_t f = 0; f < F; ++f) o[f] += w * G[v * F + f];
         }
         double s = src_norm ? src_norm[u] : 1.0;

@@ -112,3 +112,28 @@ def test_gat_attention_mask_layer():
     # del / der are the gradients w.r.t. el (source side) and er (destination side)
     assert rel_err(dl, fd_grad(f, el)) < 1e-8
     assert rel_err(dr, fd_grad(f, er)) < 1e-8
+
+
+def test_appnp_edge_dropout_fd():
+    """APPNP with a fresh edge-dropout mask per propagation step: the model's gradients vs central differences,
+    and all-ones masks reduce to the plain propagation."""
+    import synth
+    from oracle import model_ref
+    from conftest import rel_err
+    from test_oracle_layers import fd_grad, small_graph
+    ip, ix = small_graph(23, N=10, E=44)
+    N, Fin, Hd, C, K = 10, 4, 5, 3, 3
+    X = synth.uniform(1, (N, Fin)).astype(np.float64)
+    lab = synth.labels(2, N, C)
+    p = {"W1": synth.uniform(3, (Fin, Hd)).astype(np.float64), "b1": synth.uniform(4, (Hd,)).astype(np.float64) * .1,
+         "W2": synth.uniform(5, (Hd, C)).astype(np.float64), "b2": synth.uniform(6, (C,)).astype(np.float64) * .1}
+    H0 = synth.uniform(7, (N, C)).astype(np.float64)
+    np.testing.assert_array_equal(oracle.appnp_fwd(ip, ix, H0, K, 0.1),
+                                  oracle.appnp_fwd(ip, ix, H0, K, 0.1, edge_masks=[np.ones(44)] * K))
+    drop = {"edge_p": 0.5, "seed": 3, "step": 1}
+    acts = {}
+    _, g = model_ref.appnp(ip, ix, X, lab, p, K, 0.1, acts, drop)
+    assert np.abs(acts["Z1"]).min() > 1e-4
+    for k in p:
+        fd = fd_grad(lambda: model_ref.appnp(ip, ix, X, lab, p, K, 0.1, None, drop)[0], p[k])
+        assert rel_err(g[k], fd) < 1e-7, k
