@@ -198,7 +198,10 @@ size_t seastar_linear_bwd_weight_workspace(int64_t M, int64_t K, int64_t Nout);
  */
 seastar_status seastar_gcn_fwd(seastar_graph g, const float* T_all, int64_t F, int64_t ld, const float* dst_norm,
                                const float* bias, seastar_act act, float alpha, const float* H0_loc,
-                               float* Y_loc, const float* out_scale, float* Ys_loc, seastar_stream stream);
+                               float* Y_loc, const float* out_scale, float* Ys_loc,
+                               const seastar_dropout_spec* edge_drop, seastar_stream stream);
+/* (edge_drop: NULL, or NEXT-3 edge dropout (DGL APPNPConv edge_drop): edge e's message is multiplied by
+ *  keep(eid) / (1 - p), eid = user edge id; the backward takes the same spec) */
 /*
  * Adjoint over the reverse CSR, for every owned vertex u:
  *   g       = scale * src_norm[u] * sum_{e in out(u)} dP_all[dst(e),:]
@@ -210,7 +213,8 @@ seastar_status seastar_gcn_fwd(seastar_graph g, const float* T_all, int64_t F, i
  */
 seastar_status seastar_gcn_bwd(seastar_graph g, const float* dP_all, int64_t F, int64_t ld, const float* src_norm,
                                float scale, const float* Yact_loc, seastar_act act, const float* post_scale,
-                               float* dA_loc, float* dP_loc, seastar_stream stream);
+                               float* dA_loc, float* dP_loc, const seastar_dropout_spec* edge_drop,
+                               seastar_stream stream);
 
 /* ------------------------------------------------------------------------------------------ */
 /* a6 / a9: GAT (Fig. 2 L95-L123, Fig. 3, FSM units L391-L393)                   */

@@ -64,8 +64,8 @@ _SIGS = {
     "seastar_linear_bwd_data": ([_P, _I64, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
     "seastar_linear_bwd_weight": ([_P, _I64, _I64, _I64, _P, _I64, _I64, _P, _P, _P, _SZ, _P], _ST),
     "seastar_linear_bwd_weight_workspace": ([_I64, _I64, _I64], _SZ),
-    "seastar_gcn_fwd": ([_P, _P, _I64, _I64, _P, _P, _I32, _F, _P, _P, _P, _P, _P], _ST),
-    "seastar_gcn_bwd": ([_P, _P, _I64, _I64, _P, _F, _P, _I32, _P, _P, _P, _P], _ST),
+    "seastar_gcn_fwd": ([_P, _P, _I64, _I64, _P, _P, _I32, _F, _P, _P, _P, _P, _P, _P], _ST),
+    "seastar_gcn_bwd": ([_P, _P, _I64, _I64, _P, _F, _P, _I32, _P, _P, _P, _P, _P], _ST),
     "seastar_gat_attn_proj": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P], _ST),
     "seastar_gat_fwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _I32, _P, _P, _P, _P, _P, _P, _P], _ST),
     "seastar_gat_record_ld": ([_I32, _I32], _I64),
@@ -231,17 +231,17 @@ def seastar_linear_bwd_weight(X, M, K, ldx, dY, Nout, ldy, dW, db, workspace, ws
 
 # ----------------------------------------------------------------------------------- GCN / APPNP
 def seastar_gcn_fwd(g, T_all, F, ld, dst_norm, bias, act, alpha, H0_loc, Y_loc, out_scale=None, Ys_loc=None,
-                    stream=None) -> None:
+                    stream=None, edge_drop=None) -> None:
     _call("seastar_gcn_fwd", g, _dptr(T_all, "T_all"), F, ld, _dptr(dst_norm, "dst_norm"), _dptr(bias, "bias"),
           _act(act), float(alpha), _dptr(H0_loc, "H0"), _dptr(Y_loc, "Y"), _dptr(out_scale, "out_scale"),
-          _dptr(Ys_loc, "Ys"), _stream(stream))
+          _dptr(Ys_loc, "Ys"), _spec(edge_drop), _stream(stream))
 
 
 def seastar_gcn_bwd(g, dP_all, F, ld, src_norm, scale, Yact_loc, act, post_scale, dA_loc, dP_loc,
-                    stream=None) -> None:
+                    stream=None, edge_drop=None) -> None:
     _call("seastar_gcn_bwd", g, _dptr(dP_all, "dP_all"), F, ld, _dptr(src_norm, "src_norm"), float(scale),
           _dptr(Yact_loc, "Yact"), _act(act), _dptr(post_scale, "post_scale"), _dptr(dA_loc, "dA"),
-          _dptr(dP_loc, "dP"), _stream(stream))
+          _dptr(dP_loc, "dP"), _spec(edge_drop), _stream(stream))
 
 
 # ----------------------------------------------------------------------------------- GAT

@@ -168,6 +168,14 @@ __device__ __forceinline__ float drop_mult(uint64_t key, uint64_t i, uint32_t th
 }
 inline uint32_t drop_threshold(float p) { return (uint32_t)llround((double)p * 16777216.0); }
 inline float drop_scale(float p) { return (float)(1.0 / (1.0 - (double)p)); }
+// dropout fields (deid, dseed, dstep, dsite, dthr, dscale) of a kernel argument block from the ABI spec
+// (NULL or p == 0: off, deid = nullptr); eid = the index set's user edge ids (the mask's counter)
+template <typename Args>
+inline void set_drop(Args& a, const seastar_dropout_spec* d, const int32_t* eid) {
+    if (!d || d->p <= 0.f) { a.deid = nullptr; return; }
+    a.deid = eid; a.dseed = d->seed; a.dstep = d->step; a.dsite = d->site;
+    a.dthr = drop_threshold(d->p); a.dscale = drop_scale(d->p);
+}
 
 // ----------------------------------------------------------------------------------------------
 // L2 residency of the gathered table.  Every edge of a graph kernel gathers a row of one table

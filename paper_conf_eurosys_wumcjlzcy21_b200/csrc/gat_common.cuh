@@ -55,13 +55,6 @@ struct GatBwdArgs {
     const int32_t* deid; uint64_t dseed; const int32_t* dstep; uint32_t dsite, dthr; float dscale;   // as GatFwdArgs
 };
 
-// attention-dropout fields of the argument blocks from the ABI spec (NULL or p == 0: off)
-template <typename Args>
-inline void set_attn_drop(Args& a, const seastar_dropout_spec* d, const int32_t* eid) {
-    if (!d || d->p <= 0.f) { a.deid = nullptr; return; }
-    a.deid = eid; a.dseed = d->seed; a.dstep = d->step; a.dsite = d->site;
-    a.dthr = drop_threshold(d->p); a.dscale = drop_scale(d->p);
-}
 
 // packed backward record D[v] = [dA (H*F, zero-padded to a multiple of 4) | per head (er, lse, c, nl2)]
 // with nl2 = -lse * log2(e), so a_e = ex2(LReLU(s_e) log2 e + nl2) is one FFMA + one SFU op

@@ -35,9 +35,11 @@ struct AggArgs {
     const float* H0; float alpha; const float* bias; int act; float* Y; const float* out_scale; float* Ys;
     // backward
     const float* Yact; float* dA; const float* post_scale; float* dP;
+    // NEXT-3 edge dropout (deid == nullptr: off): edge k's message is scaled by drop_mult(key, eid[k])
+    const int32_t* deid; uint64_t dseed; const int32_t* dstep; uint32_t dsite, dthr; float dscale;
 };
 
-template <int VEC, int L, int RL, int NB>
+template <int VEC, int L, int RL, int NB, bool DROP = false>
 __global__ void __launch_bounds__(256) k_aggregate(const AggArgs a) {
     constexpr int S = RL / L;                    // edge slots per row group
 #ifdef GCN_UB_FIXED
@@ -57,6 +59,7 @@ __global__ void __launch_bounds__(256) k_aggregate(const AggArgs a) {
     const int end = valid ? __ldg(a.off + row + 1) : 0;
     const int64_t v = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;
     const int C = (a.F + VEC - 1) / VEC;
+    const uint64_t dkey = DROP ? drop_key(a.dseed, a.dsite, a.dstep) : 0ull;
 
     for (int cb = 0; cb < C; cb += L) {
         const int chunk = cb + c;
@@ -93,6 +96,12 @@ __global__ void __launch_bounds__(256) k_aggregate(const AggArgs a) {
                         const int u = __shfl_sync(gmask, my[h], k & (RL - 1), RL);
                         if (k < n[h] && active) {
                             load_vec<VEC>(a.table + (int64_t)u * a.ld + col, val[h][jj]);
+                            if (DROP) {
+                                const float w = drop_mult(dkey, (uint64_t)__ldg(a.deid + base + h * RL + k), a.dthr,
+                                                          a.dscale);
+#pragma unroll
+                                for (int i = 0; i < VEC; ++i) val[h][jj][i] *= w;
+                            }
                         } else {
 #pragma unroll
                             for (int i = 0; i < VEC; ++i) val[h][jj][i] = 0.f;
@@ -176,12 +185,14 @@ static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s) {
         // narrow rows (L < 4 chunk lanes, F <= 8) take 4/L index chunks per iteration so every lane still has
         // 4 gathers in flight: F = 8 0.75 -> 0.50 ms, F = 1..4 0.54 -> 0.46 ms on Reddit (tools/ab_gcn.sh)
         constexpr int NBW = L >= 4 ? 1 : 4 / L;
-        launch_k(k_aggregate<VEC, L, 32, NBW>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        if (a.deid) launch_k(k_aggregate<VEC, L, 32, NBW, true>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        else launch_k(k_aggregate<VEC, L, 32, NBW>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
     } else {
         constexpr int RL = L < 4 ? 4 : L;   // at least 4 lanes per row group keeps index loads useful
         const int64_t per_block = threads / RL;
         const int64_t blocks = (rows + per_block - 1) / per_block;
-        launch_k(k_aggregate<VEC, L, RL, 1>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        if (a.deid) launch_k(k_aggregate<VEC, L, RL, 1, true>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        else launch_k(k_aggregate<VEC, L, RL, 1>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
     }
 }
 
@@ -228,7 +239,8 @@ extern "C" {
 
 seastar_status seastar_gcn_fwd(seastar_graph g, const float* T_all, int64_t F, int64_t ld, const float* dst_norm,
                                const float* bias, seastar_act act, float alpha, const float* H0_loc, float* Y_loc,
-                               const float* out_scale, float* Ys_loc, seastar_stream stream) {
+                               const float* out_scale, float* Ys_loc, const seastar_dropout_spec* edge_drop,
+                               seastar_stream stream) {
     SS_ARG(g != nullptr, "gcn_fwd: graph is NULL");
     SS_ARG(F >= 1 && ld >= F, "gcn_fwd: need 1 <= F <= ld (F=%lld, ld=%lld)", (long long)F, (long long)ld);
     SS_ARG(T_all != nullptr && Y_loc != nullptr, "gcn_fwd: T_all and Y_loc are required");
@@ -241,6 +253,8 @@ seastar_status seastar_gcn_fwd(seastar_graph g, const float* T_all, int64_t F, i
     a.table = T_all; a.ld = ld; a.F = (int)F; a.bwd = 0;
     a.rscale = dst_norm; a.gscale = 1.f;
     a.H0 = H0_loc; a.alpha = alpha; a.bias = bias; a.act = act; a.Y = Y_loc; a.out_scale = out_scale; a.Ys = Ys_loc;
+    SS_ARG(!edge_drop || (edge_drop->p >= 0.f && edge_drop->p < 1.f), "gcn_fwd: need 0 <= edge_drop->p < 1");
+    set_drop(a, edge_drop, g->fwd.eid);
     bool vec4 = (ld % 4 == 0) && aligned16(T_all) && aligned16(Y_loc) && (!H0_loc || aligned16(H0_loc)) &&
                 (!Ys_loc || aligned16(Ys_loc));
     return launch_aggregate(g->fwd, a, vec4, to_stream(stream));
@@ -248,7 +262,8 @@ seastar_status seastar_gcn_fwd(seastar_graph g, const float* T_all, int64_t F, i
 
 seastar_status seastar_gcn_bwd(seastar_graph g, const float* dP_all, int64_t F, int64_t ld, const float* src_norm,
                                float scale, const float* Yact_loc, seastar_act act, const float* post_scale,
-                               float* dA_loc, float* dP_loc, seastar_stream stream) {
+                               float* dA_loc, float* dP_loc, const seastar_dropout_spec* edge_drop,
+                               seastar_stream stream) {
     SS_ARG(g != nullptr, "gcn_bwd: graph is NULL");
     SS_ARG(F >= 1 && ld >= F, "gcn_bwd: need 1 <= F <= ld");
     SS_ARG(dP_all != nullptr, "gcn_bwd: dP_all is NULL");
@@ -261,6 +276,8 @@ seastar_status seastar_gcn_bwd(seastar_graph g, const float* dP_all, int64_t F, 
     a.table = dP_all; a.ld = ld; a.F = (int)F; a.bwd = 1;
     a.rscale = src_norm; a.gscale = scale;
     a.Yact = Yact_loc; a.act = act; a.dA = dA_loc; a.post_scale = post_scale; a.dP = dP_loc;
+    SS_ARG(!edge_drop || (edge_drop->p >= 0.f && edge_drop->p < 1.f), "gcn_bwd: need 0 <= edge_drop->p < 1");
+    set_drop(a, edge_drop, g->rev.eid);
     bool vec4 = (ld % 4 == 0) && aligned16(dP_all) && (!dA_loc || aligned16(dA_loc)) && (!dP_loc || aligned16(dP_loc)) &&
                 (!Yact_loc || aligned16(Yact_loc));
     return launch_aggregate(g->rev, a, vec4, to_stream(stream));

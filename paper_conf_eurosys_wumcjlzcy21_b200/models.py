@@ -388,7 +388,7 @@ class APPNPNet:
     Each propagation step is one fused gcn_fwd (APPNP epilogue, writes Z and n*Z for the next step)."""
 
     def __init__(self, g: Graph, X_loc, labels_loc, params: dict, K=10, alpha=0.1, lr=0.01, comm: Comm | None = None,
-                 n_pad_rows: int | None = None):
+                 n_pad_rows: int | None = None, edge_dropout: float = 0.0, seed: int = 0):
         self.g, self.X, self.lab, self.K, self.alpha, self.lr = g, X_loc, labels_loc, K, alpha, lr
         self.comm = comm or Comm()
         dev = X_loc.device
@@ -414,6 +414,8 @@ class APPNPNet:
         self.dHh = e(n, Hd)
         self.loss = torch.zeros(1, device=dev)
         self.ws = _Ws(dev)
+        # NEXT-3 edge_drop (DGL APPNPConv): a fresh mask per propagation step k (site 16 + k, by user edge id)
+        self.ed = [L.dropout_spec(edge_dropout, 16 + k, seed, self.P.step) for k in range(K)]
         P = self.comm.world
         self.Zs_all = e(self.rows_all, self.ldc) if P > 1 else None
         self.Gs_all = e(self.rows_all, self.ldc) if P > 1 else None
@@ -433,7 +435,7 @@ class APPNPNet:
             Zs_all = self.comm.all_gather(self.Zs_all, self.Zs[k])
             self._t("appnp_fwd") if k == 0 else None
             L.seastar_gcn_fwd(g.handle, Zs_all, C, ld, self.nrm, None, "none", self.alpha, self.H0, self.Z[k + 1],
-                              self.nrm, self.Zs[k + 1])
+                              self.nrm, self.Zs[k + 1], edge_drop=self.ed[k])
             self._t("appnp_fwd_end") if k == 0 else None
         out = self.Z[self.K] if self.K > 0 else self.H0
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
@@ -453,7 +455,8 @@ class APPNPNet:
             Gs_all = self.comm.all_gather(self.Gs_all, self.Gs[cur])
             nxt = self.Gtmp if G is self.G else self.G
             self._t("appnp_bwd") if k == 0 else None
-            L.seastar_gcn_bwd(g.handle, Gs_all, C, ld, self.nrm, 1.0 - a, None, "none", self.nrm, nxt, self.Gs[1 - cur])
+            L.seastar_gcn_bwd(g.handle, Gs_all, C, ld, self.nrm, 1.0 - a, None, "none", self.nrm, nxt, self.Gs[1 - cur],
+                              edge_drop=self.ed[self.K - 1 - k])
             self._t("appnp_bwd_end") if k == 0 else None
             G = nxt
             cur = 1 - cur

@@ -174,3 +174,41 @@ def test_gat2_attn_dropout(env, save_B):
                     dropout=0.6, attn_dropout=0.6, seed=8, save_der_factors=save_B)
     _check(m, *model_ref.gat2(ip, ix, X, lab, {k: v.astype(np.float64) for k, v in p.items()}, heads, hid,
                               drop={"p": 0.6, "attn_p": 0.6, "seed": 8, "step": 0}))
+
+
+def test_appnp_edge_dropout(env):
+    """DGL APPNPConv's edge_drop: a fresh edge mask per propagation step, fused into the aggregation kernels."""
+    torch, models, Graph = env["torch"], env["models"], env["Graph"]
+    ip, ix = synth.powerlaw_sym(1800, 15000, 0.5, 66)
+    N, Fin, Hd, C, K = 1800, 150, 64, 5, 10
+    X, lab = synth.uniform(21, (N, Fin)), synth.labels(22, N, C)
+    p = {"W1": synth.glorot(23, Fin, Hd), "b1": synth.uniform(24, (Hd,), -0.1, 0.1),
+         "W2": synth.glorot(25, Hd, C), "b2": synth.uniform(26, (C,), -0.1, 0.1)}
+    m = models.APPNPNet(Graph(ip, ix), torch.from_numpy(X).cuda(), torch.from_numpy(lab).cuda(), p, K=K, alpha=0.1,
+                        edge_dropout=0.5, seed=12)
+    _check(m, *model_ref.appnp(ip, ix, X, lab, {k: v.astype(np.float64) for k, v in p.items()}, K, 0.1,
+                               drop={"edge_p": 0.5, "seed": 12, "step": 0}))
+
+
+@pytest.mark.parametrize("F", [16, 5, 64])
+def test_gcn_edge_dropout_kernels(env, F):
+    """seastar_gcn_fwd / _bwd with edge dropout vs the weighted oracle aggregation (both degree buckets)."""
+    torch, L, Graph = env["torch"], env["L"], env["Graph"]
+    from helpers import hub_graph
+    ip, ix = hub_graph(N=2500, E_dir=20000, seed=67)
+    N, E = len(ip) - 1, len(ix)
+    g = Graph(ip, ix)
+    ld = (F + 3) // 4 * 4
+    T = synth.uniform(1, (N, F))
+    Tp = np.zeros((N, ld), np.float32)
+    Tp[:, :F] = T
+    st = torch.tensor([2], dtype=torch.int32, device="cuda")
+    spec = L.dropout_spec(0.3, 16, 5, st)
+    w = oracle.dropout_mask(5, 16, 2, E, 1, 0.3)[:, 0]
+    Y = torch.zeros((N, ld), device="cuda")
+    L.seastar_gcn_fwd(g.handle, torch.from_numpy(Tp).cuda(), F, ld, None, None, "none", 0.0, None, Y, edge_drop=spec)
+    assert rel_err(Y.cpu().numpy()[:, :F], oracle.gcn_aggregate(ip, ix, T, edge_w=w)) <= TOL
+    dA = torch.zeros((N, ld), device="cuda")
+    L.seastar_gcn_bwd(g.handle, torch.from_numpy(Tp).cuda(), F, ld, None, 1.0, None, "none", None, dA, None,
+                      edge_drop=spec)
+    assert rel_err(dA.cpu().numpy()[:, :F], oracle.gcn_aggregate_T(ip, ix, T, edge_w=w)) <= TOL
