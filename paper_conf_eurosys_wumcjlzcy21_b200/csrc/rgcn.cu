@@ -29,10 +29,17 @@ struct RgcnRowArgs {
     const float* Yact;                  // dX only: fused activation backward, out *= act'(Yact)
 };
 
-// stage W (or W^T) as [R][Fg][Fop] with Fop = round4(Fo), zero padded
+// stage W (or W^T) as [R][Fg][Fop] with Fop = round4(Fo), zero padded, consecutive types kStagePad floats apart
+// beyond their Fg*Fop block: the 32/RL row groups of a warp flush runs of different types at the same in-block
+// offset, and without the pad every W_r block starts on the same bank (Fg*Fop is a multiple of 32 for the
+// 16-wide layers), an up-to-8-way shared-memory bank conflict on every flush load
+constexpr int kStagePad = 4;
+__host__ __device__ inline int64_t w_stride(int Fg, int Fop) { return (int64_t)Fg * Fop + kStagePad; }
+
 __device__ void stage_w(const RgcnRowArgs& a, float* Ws) {
     const int Fop = (a.Fo + 3) & ~3;
     const int64_t n = (int64_t)a.R * a.Fg * Fop;
+    const int64_t ws = w_stride(a.Fg, Fop);
     for (int64_t idx = threadIdx.x; idx < n; idx += blockDim.x) {
         const int j = (int)(idx % Fop);
         const int64_t ri = idx / Fop;
@@ -45,13 +52,10 @@ __device__ void stage_w(const RgcnRowArgs& a, float* Ws) {
             w = a.transpose ? __ldg(a.W + ((int64_t)r * a.Fo + j) * a.Fg + i)
                             : __ldg(a.W + ((int64_t)r * a.Fg + i) * a.Fo + j);
         }
-        Ws[idx] = w;
+        Ws[r * ws + (int64_t)i * Fop + j] = w;
     }
 }
 
-// WPR = 1: RL lanes per row (rows of degree < 1024).  WPR > 1 (hub rows, degree >= 1024): one CTA of WPR
-// warps per row, warp w owns the contiguous edge slice w/WPR of the row (a type run cut at a slice border is
-// flushed through W_r by both warps -- linear, so exact), per-warp outputs merged in warp order.
 template <int L, int RL, int WPR, int BS = 512>
 __global__ void __launch_bounds__(BS) k_rgcn_rows(const RgcnRowArgs a) {
     extern __shared__ float4 smem4[];
@@ -87,7 +91,7 @@ __global__ void __launch_bounds__(BS) k_rgcn_rows(const RgcnRowArgs a) {
         float g[4] = {0.f, 0.f, 0.f, 0.f};
         int cur = -1;
         auto flush = [&](int r) {
-            const float* wr = Ws + (int64_t)r * a.Fg * Fop;
+            const float* wr = Ws + (int64_t)r * w_stride(a.Fg, Fop);
 #pragma unroll
             for (int cl = 0; cl < L; ++cl) {
                 if (cl >= Cg) break;
@@ -429,13 +433,14 @@ static seastar_status launch_rows(const RgcnRowArgs& a, size_t smem, cudaStream_
 
 template <int L>
 static seastar_status launch_buckets(const IndexSet& x, RgcnRowArgs a, size_t smem, cudaStream_t s) {
-    const int64_t hub = x.bucket_rows[0];     // degree >= 1024: a 16-warp CTA per row
+    const int64_t hub = x.bucket_rows[0];     // degree >= 1024: a 16- or 32-warp CTA per row
     const int64_t split = x.bucket_rows[1];   // rows with degree >= 32 get a warp with 32/L slots
     RgcnRowArgs hb = a, hi = a, lo = a;
     hb.row_begin = 0; hb.row_end = hub;
     hi.row_begin = hub; hi.row_end = split;
     lo.row_begin = split; lo.row_end = x.n_rows;
-    SS_TRY((launch_rows<L, 32, 16>(hb, smem, s)));
+    constexpr int WH = L <= 4 ? 32 : 16;     // hub rows: one CTA of WH warps (registers allow 1024 threads at L <= 4)
+    SS_TRY((launch_rows<L, 32, WH, 32 * WH>(hb, smem, s)));
     SS_TRY((launch_rows<L, 32>(hi, smem, s)));
     constexpr int RLo = L < 4 ? 4 : L;
     return launch_rows<L, RLo>(lo, smem, s);
@@ -443,7 +448,7 @@ static seastar_status launch_buckets(const IndexSet& x, RgcnRowArgs a, size_t sm
 
 static seastar_status launch_rows_L(const IndexSet& x, const RgcnRowArgs& a, cudaStream_t s) {
     const int Cm = ((a.Fg > a.Fo ? a.Fg : a.Fo) + 3) / 4;
-    const size_t smem = (size_t)a.R * a.Fg * ((a.Fo + 3) & ~3) * sizeof(float);
+    const size_t smem = (size_t)a.R * w_stride(a.Fg, (a.Fo + 3) & ~3) * sizeof(float);
     switch (pow2_ceil(Cm)) {
         case 1: return launch_buckets<1>(x, a, smem, s);
         case 2: return launch_buckets<2>(x, a, smem, s);
