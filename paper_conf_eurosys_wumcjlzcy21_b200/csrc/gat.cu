@@ -460,6 +460,67 @@ __global__ void __launch_bounds__(256) k_gat_bwd_prep(int64_t M, int H, int F, i
     }
 }
 
+// vectorised row pass for the common geometry (W = H*F <= 128, float4-aligned rows, H == 1 or F/4 a power of
+// two): LR = pow2(ceil(W/4)) lanes per row, one float4 chunk per lane, 32/LR rows per warp; per-head fp64 sums
+// by a segmented xor tree over the lanes of the head (deterministic).  Same outputs as k_gat_bwd_prep.
+template <int LR>
+__global__ void __launch_bounds__(256) k_gat_bwd_prep4(int64_t M, int H, int F, int64_t ldt,
+                                                       const float* __restrict__ dY, const float* __restrict__ Y,
+                                                       int act, const float* __restrict__ A,
+                                                       const float* __restrict__ er, const float* __restrict__ lse,
+                                                       float* __restrict__ D, int64_t ldd, const float* __restrict__ B,
+                                                       const float* __restrict__ bsum, float* __restrict__ der) {
+    const int lane = threadIdx.x & 31;
+    const int c = lane % LR;
+    const int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / LR;
+    const bool valid = v < M;
+    const int W = H * F, C4 = (W + 3) / 4;
+    const int lph = H == 1 ? LR : F / 4;                   // lanes per head (a power of two)
+    const int h = H == 1 ? 0 : c / lph;
+    double pc = 0.0, pb = 0.0;
+    if (valid && c < C4) {
+        const int64_t o = v * ldt + 4 * c;
+        float d[4], y[4], a[4], b[4];
+        const float4 dy = ldg4(dY + o);
+        d[0] = dy.x; d[1] = dy.y; d[2] = dy.z; d[3] = dy.w;
+        if (act != SEASTAR_ACT_NONE) {
+            const float4 y4 = ldg4(Y + o);
+            y[0] = y4.x; y[1] = y4.y; y[2] = y4.z; y[3] = y4.w;
+#pragma unroll
+            for (int i = 0; i < 4; ++i) d[i] *= act_grad_from_y(act, y[i]);
+        }
+        const float4 a4 = ldg4(A + o);
+        a[0] = a4.x; a[1] = a4.y; a[2] = a4.z; a[3] = a4.w;
+        if (B) {
+            const float4 b4 = ldg4(B + o);
+            b[0] = b4.x; b[1] = b4.y; b[2] = b4.z; b[3] = b4.w;
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            if (4 * c + i >= W) {                          // row padding (may hold NaN): zero in the record,
+                d[i] = 0.f;                                // never in the sums
+                continue;
+            }
+            pc += (double)d[i] * (double)a[i];
+            if (B) pb += (double)d[i] * (double)b[i];
+        }
+        *reinterpret_cast<float4*>(D + v * ldd + 4 * c) = make_float4(d[0], d[1], d[2], d[3]);
+    }
+    for (int off = lph >> 1; off; off >>= 1) {
+        pc += __shfl_xor_sync(0xffffffffu, pc, off, LR);
+        pb += __shfl_xor_sync(0xffffffffu, pb, off, LR);
+    }
+    if (!valid || (c % lph) != 0 || h >= H) return;
+    const int64_t i = v * H + h;
+    if (B) der[i] = (float)(pb - pc * (double)__ldg(bsum + i));
+    float* aux = D + v * ldd + rec_aux_offset(W) + 4 * h;
+    aux[0] = __ldg(er + i);
+    const float l = __ldg(lse + i);
+    aux[1] = l;
+    aux[2] = (float)pc;
+    aux[3] = -l * kLog2e;
+}
+
 // stage 1 of attn_proj_bwd: dT += del a_l + der a_r (in place) and per-block partial da_l, da_r
 __global__ void __launch_bounds__(256) k_gat_attn_proj_bwd1(const float* __restrict__ T, int64_t M, int H, int F,
                                                             int64_t ldt, const float* __restrict__ a_l,
@@ -628,6 +689,28 @@ seastar_status seastar_gat_bwd_prep(seastar_graph g, const float* dY_loc, const 
     SS_TRY(check_device());
     const int64_t M = g->n_loc();
     if (M == 0) return SEASTAR_OK;
+    const int W = H * F, C4 = (W + 3) / 4;
+    const bool geo4 = W <= 128 && ldt % 4 == 0 && aligned16(dY_loc) && aligned16(A_loc) && aligned16(D_loc) &&
+                      (!Y_loc || aligned16(Y_loc)) && (!B_loc || aligned16(B_loc)) &&
+                      (H == 1 || (F % 4 == 0 && ((F / 4) & (F / 4 - 1)) == 0 && F / 4 <= 32));
+    if (geo4) {
+        const int LR = pow2_ceil(C4);
+        const unsigned grid = (unsigned)((M * LR + 255) / 256);
+        const int64_t ldd = seastar_gat_record_ld(H, F);
+        cudaStream_t s = to_stream(stream);
+#define PREP4(LRV) k_gat_bwd_prep4<LRV><<<grid, 256, 0, s>>>(M, H, F, ldt, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, \
+                                                             D_loc, ldd, B_loc, b_loc, der_loc)
+        switch (LR) {
+            case 1: PREP4(1); break;
+            case 2: PREP4(2); break;
+            case 4: PREP4(4); break;
+            case 8: PREP4(8); break;
+            case 16: PREP4(16); break;
+            default: PREP4(32); break;
+        }
+#undef PREP4
+        return check_launch("k_gat_bwd_prep4");
+    }
     SS_ARG(H <= 8 || (32 % F == 0 && H <= 32), "gat_bwd_prep: H > 8 needs F dividing 32 (and H <= 32)");
     k_gat_bwd_prep<<<(unsigned)((M + 7) / 8), 256, 0, to_stream(stream)>>>(
         M, H, F, ldt, dY_loc, Y_loc, act, A_loc, er_loc, lse_loc, D_loc, seastar_gat_record_ld(H, F), B_loc, b_loc,
