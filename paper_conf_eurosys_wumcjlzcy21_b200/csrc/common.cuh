@@ -198,7 +198,8 @@ struct ScopedL2Window {
 
 size_t l2_persist_bytes();
 // out[(i / nc) * ldo + i % nc] = sum_b part[b * stride + i] for i < n: deterministic fp64 reduction of
-// split partials (fixed order: 8 warp-strided lanes of splits, then the 8 lanes in order); one block of
+// split partials (fixed order: 8 (or, for few outputs and many splits, 32) warp-strided lanes of splits, then
+// the lanes in order); one block of
 // 256 threads per 32 consecutive outputs, so the split count does not serialise the reduction
 void reduce_splits(const float* part, int64_t nsplit, int64_t stride, int64_t n, int64_t nc, int64_t ldo, float* out,
                    cudaStream_t s);   // device set-aside for persisting lines (configured on first use), 0 if none

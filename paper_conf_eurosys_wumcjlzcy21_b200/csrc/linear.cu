@@ -110,8 +110,79 @@ __global__ void __launch_bounds__(256) k_gemm(const GemmArgs g) {
     }
 }
 
+// Skinny products (K <= 64, N <= 64: the class-width layers, e.g. logits = P2 W2 and dY1 = dT2 W2^T on Reddit):
+// B is staged once per persistent CTA in shared memory (zero padded to 64 x 64), a warp owns 4 rows at a time,
+// lane n (and n + 32) owns output columns, A's row values are broadcast by shuffles.  Each output is the same
+// fp32 FMA chain over k = 0..K-1 as k_gemm's, so the result does not depend on the kernel choice.  HBM-bound:
+// A and C are streamed once (k_gemm's 128 x 64 tiles were ~8x off that bound at M = 233 k).
+template <int KC, int NC>
+__global__ void __launch_bounds__(256) k_gemm_skinny(const GemmArgs g) {
+    __shared__ float Bs[64][64];
+    for (int idx = threadIdx.x; idx < 64 * 64; idx += 256) {
+        const int k = idx / 64, n = idx % 64;
+        Bs[k][n] = (k < g.K && n < g.N) ? __ldg(g.B + (int64_t)k * g.ldb_k + (int64_t)n * g.ldb_n) : 0.f;
+    }
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t step = (int64_t)gridDim.x * 8 * 4;
+    for (int64_t m0 = ((int64_t)blockIdx.x * 8 + warp) * 4; m0 < g.M; m0 += step) {
+        float a[4][KC], acc[4][NC];
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+#pragma unroll
+            for (int c = 0; c < KC; ++c) {
+                const int k = lane + 32 * c;
+                a[r][c] = (m0 + r < g.M && k < g.K) ? __ldg(g.A + (m0 + r) * g.lda + k) : 0.f;
+            }
+#pragma unroll
+            for (int c = 0; c < NC; ++c) acc[r][c] = 0.f;
+        }
+#pragma unroll
+        for (int c = 0; c < KC; ++c) {
+            const int kend = (int)(g.K - 32 * c < 32 ? g.K - 32 * c : 32);
+            for (int kk = 0; kk < kend; ++kk) {
+                float b[NC];
+#pragma unroll
+                for (int j = 0; j < NC; ++j) b[j] = Bs[32 * c + kk][lane + 32 * j];
+#pragma unroll
+                for (int r = 0; r < 4; ++r) {
+                    const float av = __shfl_sync(0xffffffffu, a[r][c], kk);
+#pragma unroll
+                    for (int j = 0; j < NC; ++j) acc[r][j] = fmaf(av, b[j], acc[r][j]);
+                }
+            }
+        }
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            const int64_t gm = m0 + r;
+            if (gm >= g.M) break;
+            const float rs = g.row_scale ? __ldg(g.row_scale + gm) : 1.f;
+#pragma unroll
+            for (int j = 0; j < NC; ++j) {
+                const int64_t gn = lane + 32 * j;
+                if (gn >= g.N) continue;
+                float z = acc[r][j] + (g.bias ? __ldg(g.bias + gn) : 0.f);
+                z = rs * act_apply(g.act, z);
+                if (g.Yact) z *= act_grad_from_y(g.dact, __ldg(g.Yact + gm * g.ldc + gn));
+                g.C[gm * g.ldc + gn] = z;
+            }
+        }
+    }
+}
+
 static seastar_status launch_gemm(const GemmArgs& g, cudaStream_t s) {
     if (g.M == 0 || g.N == 0) return SEASTAR_OK;
+    if (g.K <= 64 && g.N <= 64) {
+        int64_t blocks = (g.M + 31) / 32;
+        const int64_t cap = 8 * (int64_t)num_sms();
+        if (blocks > cap) blocks = cap;
+        const int kc = g.K <= 32 ? 1 : 2, nc = g.N <= 32 ? 1 : 2;
+        if (kc == 1 && nc == 1) k_gemm_skinny<1, 1><<<(unsigned)blocks, 256, 0, s>>>(g);
+        else if (kc == 1) k_gemm_skinny<1, 2><<<(unsigned)blocks, 256, 0, s>>>(g);
+        else if (nc == 1) k_gemm_skinny<2, 1><<<(unsigned)blocks, 256, 0, s>>>(g);
+        else k_gemm_skinny<2, 2><<<(unsigned)blocks, 256, 0, s>>>(g);
+        return check_launch("k_gemm_skinny");
+    }
     if (g.N <= 16) {
         dim3 grid((unsigned)((g.M + 255) / 256), 1);
         k_gemm<256, 16, 4, 4><<<grid, 256, 0, s>>>(g);

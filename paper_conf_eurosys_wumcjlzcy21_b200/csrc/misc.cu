@@ -38,35 +38,43 @@ __global__ void __launch_bounds__(256) k_colsum1(const float* __restrict__ X, in
     }
 }
 
-__global__ void __launch_bounds__(256) k_reduce_splits(const float* __restrict__ part, int64_t nsplit, int64_t stride,
-                                                       int64_t n, int64_t nc, int64_t ldo, float* __restrict__ out) {
-    __shared__ double red[8][32];
+template <int WARPS>
+__global__ void __launch_bounds__(32 * WARPS) k_reduce_splits(const float* __restrict__ part, int64_t nsplit,
+                                                              int64_t stride, int64_t n, int64_t nc, int64_t ldo,
+                                                              float* __restrict__ out) {
+    __shared__ double red[WARPS][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t i = (int64_t)blockIdx.x * 32 + lane;
     double x = 0.0;
     if (i < n) {
         int64_t b = w;
-        for (; b + 24 < nsplit; b += 32) {      // 4 independent loads in flight per lane
-            const float a0 = __ldg(part + b * stride + i), a1 = __ldg(part + (b + 8) * stride + i);
-            const float a2 = __ldg(part + (b + 16) * stride + i), a3 = __ldg(part + (b + 24) * stride + i);
+        for (; b + 3 * WARPS < nsplit; b += 4 * WARPS) {      // 4 independent loads in flight per lane
+            const float a0 = __ldg(part + b * stride + i), a1 = __ldg(part + (b + WARPS) * stride + i);
+            const float a2 = __ldg(part + (b + 2 * WARPS) * stride + i), a3 = __ldg(part + (b + 3 * WARPS) * stride + i);
             x += (double)a0; x += (double)a1; x += (double)a2; x += (double)a3;
         }
-        for (; b < nsplit; b += 8) x += (double)__ldg(part + b * stride + i);
+        for (; b < nsplit; b += WARPS) x += (double)__ldg(part + b * stride + i);
     }
     red[w][lane] = x;
     __syncthreads();
     if (w == 0 && i < n) {
         double y = 0.0;
 #pragma unroll
-        for (int k = 0; k < 8; ++k) y += red[k][lane];
+        for (int k = 0; k < WARPS; ++k) y += red[k][lane];
         out[(i / nc) * ldo + (i % nc)] = (float)y;
     }
 }
 
+// few outputs (fewer 32-column blocks than SMs) and many splits: 32 split lanes per column instead of 8, so the
+// per-lane chains are 4x shorter (the attention-projection and bias reductions: 2 blocks x 1,184 splits)
 void reduce_splits(const float* part, int64_t nsplit, int64_t stride, int64_t n, int64_t nc, int64_t ldo, float* out,
                    cudaStream_t s) {
     if (n <= 0) return;
-    k_reduce_splits<<<(unsigned)((n + 31) / 32), 256, 0, s>>>(part, nsplit, stride, n, nc, ldo, out);
+    const int64_t blocks = (n + 31) / 32;
+    if (blocks < num_sms() && nsplit > 64)
+        k_reduce_splits<32><<<(unsigned)blocks, 1024, 0, s>>>(part, nsplit, stride, n, nc, ldo, out);
+    else
+        k_reduce_splits<8><<<(unsigned)blocks, 256, 0, s>>>(part, nsplit, stride, n, nc, ldo, out);
 }
 
 seastar_status colsum_impl(const float* X, int64_t M, int64_t F, int64_t ld, float* out, void* ws, size_t ws_bytes,
