@@ -39,8 +39,19 @@ struct AggArgs {
     const int32_t* deid; uint64_t dseed; const int32_t* dstep; uint32_t dsite, dthr; float dscale;
 };
 
+// minimum resident blocks (0: compiler's choice, 48 registers at F = 16).  Measured on Reddit: forcing 6 blocks
+// (40 registers) speeds the plain-sum sweep at F = 32 / 64 (1.12 / 2.00 -> 1.01 / 1.88 ms) but slows the GCN
+// training aggregation with its fused epilogue (0.68 -> 0.73 ms), so the default leaves it to the compiler
+#ifndef AGG_MB
+#define AGG_MB 0
+#endif
+#if AGG_MB > 0
+#define AGG_BOUNDS __launch_bounds__(256, AGG_MB)
+#else
+#define AGG_BOUNDS __launch_bounds__(256)
+#endif
 template <int VEC, int L, int RL, int NB, bool DROP = false>
-__global__ void __launch_bounds__(256) k_aggregate(const AggArgs a) {
+__global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
     constexpr int S = RL / L;                    // edge slots per row group
 #ifdef GCN_UB_FIXED
     constexpr int UB = GCN_UB_FIXED < 32 / L ? GCN_UB_FIXED : 32 / L;
