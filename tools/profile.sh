@@ -10,7 +10,7 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
 python tools/launch_summary.py gpurun_out/prof_launches_$TAG.csv > gpurun_out/prof_launches_$TAG.txt 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on \
     -k regex:"k_gat_bwd_hpl|k_gat_fwd_hpl|k_gat_bwd_h1|k_gat_fwd_h1|k_aggregate|k_gemm_tc|k_rgcn" -c 12 \
-    -o /tmp/prof_$TAG python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline "$@" > gpurun_out/prof_full_$TAG.log 2>&1
+    -o /tmp/prof_$TAG python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --cuda-graph off "$@" > gpurun_out/prof_full_$TAG.log 2>&1
 python tools/ncu_summary.py /tmp/prof_$TAG.ncu-rep > gpurun_out/prof_summary_$TAG.txt 2>&1
 ncu -i /tmp/prof_$TAG.ncu-rep --page raw --csv > gpurun_out/prof_raw_$TAG.csv 2>/dev/null
 gzip -f gpurun_out/prof_raw_$TAG.csv
