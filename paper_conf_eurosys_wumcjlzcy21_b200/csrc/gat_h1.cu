@@ -167,10 +167,17 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
 
 // DER = false: source-major dT/del over REV (own = T_u, gathered = records D[v]);
 // DER = true: destination-major der over FWD (own = dA_v from D[v], gathered = T_u)
+#ifndef GAT_MB_BWD_H1
+#define GAT_MB_BWD_H1 GAT_MB_BWD
+#endif
+#ifndef GAT_H1_BWD_UBMAX
+#define GAT_H1_BWD_UBMAX 4
+#endif
 template <int VPL, int L, int RL, bool DER>
-__global__ void __launch_bounds__(256, GAT_MB_BWD) k_gat_bwd_h1(const GatBwdArgs a) {
+__global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdArgs a) {
     constexpr int NV = 4 * VPL, S = RL / L;
-    constexpr int UE = h1_ub<VPL>() < L ? h1_ub<VPL>() : L;
+    constexpr int UB0 = h1_ub<VPL>() < GAT_H1_BWD_UBMAX ? h1_ub<VPL>() : GAT_H1_BWD_UBMAX;
+    constexpr int UE = UB0 < L ? UB0 : L;
     constexpr int NB = L / UE;
     const int lane = threadIdx.x & 31;
     const int gl = lane % RL, slot = gl / L, c = gl % L;
