@@ -149,6 +149,60 @@ __global__ void __launch_bounds__(256) k_softmax_xent(const float* __restrict__ 
     }
 }
 
+// C <= 64 (every config's class count): a warp takes 4 rows, all 8 loads issued before any reduction, so
+// one memory round trip serves 4 rows (the one-row-per-warp kernel is latency-bound: 66 us at M = 233 k)
+__global__ void __launch_bounds__(256) k_softmax_xent4(const float* __restrict__ Z, int64_t M, int64_t n_total, int C,
+                                                       int64_t ldz, const int64_t* __restrict__ labels,
+                                                       float* __restrict__ dZ, int64_t lddz, float* __restrict__ part) {
+    constexpr int RPW = 4;
+    __shared__ float wl[8];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t r0 = ((int64_t)blockIdx.x * 8 + w) * RPW;
+    const float inv = 1.f / (float)n_total;
+    float zv[RPW][2];
+    int64_t lab[RPW];
+#pragma unroll
+    for (int i = 0; i < RPW; ++i) {
+        const int64_t r = r0 + i;
+        const bool ok = r < M;
+        lab[i] = ok ? labels[r] : -1;
+#pragma unroll
+        for (int k = 0; k < 2; ++k)
+            zv[i][k] = (ok && lane + 32 * k < C) ? __ldg(Z + r * ldz + lane + 32 * k) : -INFINITY;
+    }
+    float loss = 0.f;
+#pragma unroll
+    for (int i = 0; i < RPW; ++i) {
+        const int64_t r = r0 + i;
+        if (r >= M) break;                        // warp-uniform
+        float m = fmaxf(zv[i][0], zv[i][1]);
+        for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        float sum = 0.f;
+#pragma unroll
+        for (int k = 0; k < 2; ++k) sum += (lane + 32 * k < C) ? expf(zv[i][k] - m) : 0.f;
+        for (int o = 16; o; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+        const float lse = m + logf(sum);
+        float zl = 0.f;
+#pragma unroll
+        for (int k = 0; k < 2; ++k) {
+            const int c = lane + 32 * k;
+            if (c < C) {
+                if (dZ) dZ[r * lddz + c] = (expf(zv[i][k] - lse) - (c == lab[i] ? 1.f : 0.f)) * inv;
+                if (c == lab[i]) zl = zv[i][k];
+            }
+        }
+        for (int o = 16; o; o >>= 1) zl += __shfl_xor_sync(0xffffffffu, zl, o);
+        loss += lse - zl;
+    }
+    if (lane == 0) wl[w] = loss;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        float x = 0.f;
+        for (int k = 0; k < 8; ++k) x += wl[k];
+        part[blockIdx.x] = x;
+    }
+}
+
 __global__ void k_loss_final(const float* __restrict__ part, int64_t n, int64_t n_total, float* __restrict__ loss) {
     __shared__ double red[256];
     double x = 0.0;
@@ -251,9 +305,15 @@ seastar_status seastar_softmax_xent(const float* Z, int64_t M, int64_t n_total, 
     SS_ARG(ws_bytes >= seastar_softmax_xent_workspace(M), "softmax_xent: workspace too small");
     SS_TRY(check_device());
     cudaStream_t s = to_stream(stream);
-    const int64_t nblk = (M + 7) / 8;
     float* part = static_cast<float*>(workspace);
-    k_softmax_xent<<<(unsigned)nblk, 256, 0, s>>>(Z, M, n_total, C, ldz, labels, dZ, lddz, part);
+    int64_t nblk;
+    if (C <= 64) {
+        nblk = (M + 31) / 32;
+        k_softmax_xent4<<<(unsigned)nblk, 256, 0, s>>>(Z, M, n_total, C, ldz, labels, dZ, lddz, part);
+    } else {
+        nblk = (M + 7) / 8;
+        k_softmax_xent<<<(unsigned)nblk, 256, 0, s>>>(Z, M, n_total, C, ldz, labels, dZ, lddz, part);
+    }
     k_loss_final<<<1, 256, 0, s>>>(part, nblk, n_total, loss);
     return check_launch("k_softmax_xent");
 }
