@@ -264,7 +264,10 @@ __global__ void __launch_bounds__(256) k_gemm_tn(const float* __restrict__ X, in
 
 static void tn_geometry(int64_t M, int64_t K, int64_t& ktiles, int64_t& nsplit, int64_t& rows_per_split) {
     ktiles = (K + 63) / 64;
-    int64_t want = (2 * num_sms() + ktiles - 1) / ktiles;   // ~2 waves of blocks
+#ifndef TN_WAVES
+#define TN_WAVES 2
+#endif
+    int64_t want = (TN_WAVES * num_sms() + ktiles - 1) / ktiles;   // ~TN_WAVES waves of blocks
     int64_t max_split = (M + 255) / 256;                    // >= 256 rows per split
     nsplit = want < max_split ? want : max_split;
     if (nsplit < 1) nsplit = 1;
