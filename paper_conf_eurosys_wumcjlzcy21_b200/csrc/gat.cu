@@ -562,6 +562,71 @@ __global__ void __launch_bounds__(256) k_gat_attn_proj_bwd1(const float* __restr
     }
 }
 
+// vectorised stage 1 for float4-aligned rows with W = H*F <= 128 (H == 1 or F % 4 == 0): LR = pow2(ceil(W/4)) lanes
+// per row, 32/LR rows per warp instruction, two row groups in flight per warp; per-lane float4 partials of
+// da_l / da_r merged in a fixed (warp, row-slot) order through shared memory.  Same outputs as stage 1 above.
+template <int LR>
+__global__ void __launch_bounds__(256) k_gat_attn_proj_bwd4(const float* __restrict__ T, int64_t M, int H, int F,
+                                                            int64_t ldt, const float* __restrict__ a_l,
+                                                            const float* __restrict__ a_r,
+                                                            const float* __restrict__ del,
+                                                            const float* __restrict__ der, float* __restrict__ dT,
+                                                            int64_t rows_per_block, float* __restrict__ part) {
+    constexpr int RPW = 32 / LR;
+    __shared__ __align__(16) float red[8][RPW][2][4 * LR];
+    const int W = H * F, C4 = (W + 3) / 4;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int c = lane % LR, sub = lane / LR;
+    const bool act = c < C4;
+    const int nv = act ? min(4, W - 4 * c) : 0;          // valid columns of this chunk (row padding past W)
+    const int h = act ? (H == 1 ? 0 : (4 * c) / F) : 0;
+    const int64_t r0 = blockIdx.x * rows_per_block;
+    const int64_t r1 = min(M, r0 + rows_per_block);
+    float4 al4 = make_float4(0.f, 0.f, 0.f, 0.f), ar4 = al4, sl = al4, sr = al4;
+    if (act) {
+        float* pa = &al4.x;
+        float* pr = &ar4.x;
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            if (q < nv) { pa[q] = __ldg(a_l + 4 * c + q); pr[q] = __ldg(a_r + 4 * c + q); }
+    }
+    const int64_t stride = 8 * RPW;
+    for (int64_t rb = r0 + w * RPW + sub; rb < r1; rb += 2 * stride) {
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+            const int64_t r = rb + u * stride;
+            if (!act || r >= r1) continue;
+            const float dl = del ? __ldg(del + r * H + h) : 0.f;
+            const float dr = der ? __ldg(der + r * H + h) : 0.f;
+            float4 t = ldg4(T + r * ldt + 4 * c);
+            if (nv < 4) {                                    // padding columns: out of the sums, dT unchanged
+                t.w = 0.f;
+                if (nv < 3) t.z = 0.f;
+                if (nv < 2) t.y = 0.f;
+            }
+            float4* pd = reinterpret_cast<float4*>(dT + r * ldt + 4 * c);
+            float4 d = *pd;
+            d.x += dl * al4.x + dr * ar4.x; d.y += dl * al4.y + dr * ar4.y;
+            d.z += dl * al4.z + dr * ar4.z; d.w += dl * al4.w + dr * ar4.w;
+            *pd = d;
+            sl.x = fmaf(dl, t.x, sl.x); sl.y = fmaf(dl, t.y, sl.y); sl.z = fmaf(dl, t.z, sl.z); sl.w = fmaf(dl, t.w, sl.w);
+            sr.x = fmaf(dr, t.x, sr.x); sr.y = fmaf(dr, t.y, sr.y); sr.z = fmaf(dr, t.z, sr.z); sr.w = fmaf(dr, t.w, sr.w);
+        }
+    }
+    reinterpret_cast<float4*>(red[w][sub][0])[c] = sl;
+    reinterpret_cast<float4*>(red[w][sub][1])[c] = sr;
+    __syncthreads();
+    float* pl = part + (int64_t)blockIdx.x * 2 * W;
+    for (int i = threadIdx.x; i < 2 * W; i += blockDim.x) {
+        const int which = i / W, j = i % W;
+        float x = 0.f;
+        for (int ww = 0; ww < 8; ++ww)
+#pragma unroll
+            for (int q = 0; q < RPW; ++q) x += red[ww][q][which][j];
+        pl[which * W + j] = x;
+    }
+}
+
 static int64_t proj_bwd_blocks(int64_t M) {
     int64_t b = 8 * num_sms();
     if (M < b * 64) b = (M + 63) / 64;
@@ -795,7 +860,24 @@ seastar_status seastar_gat_attn_proj_bwd(const float* T, int64_t M, int32_t H, i
     const int64_t nblk = proj_bwd_blocks(M);
     const int64_t rpb = (M + nblk - 1) / nblk;
     float* part = static_cast<float*>(workspace);
-    k_gat_attn_proj_bwd1<<<(unsigned)nblk, 256, 0, s>>>(T, M, H, F, ldt, a_l, a_r, del, der, dT, rpb > 0 ? rpb : 1, part);
+    const bool vec = W <= 128 && (H == 1 || F % 4 == 0) && ldt % 4 == 0 && aligned16(T) && aligned16(dT);
+    if (vec) {
+        const int LR = pow2_ceil((W + 3) / 4);
+#define PROJ4(LRV) k_gat_attn_proj_bwd4<LRV><<<(unsigned)nblk, 256, 0, s>>>(T, M, H, F, ldt, a_l, a_r, del, der, dT, \
+                                                                         rpb > 0 ? rpb : 1, part)
+        switch (LR) {
+            case 1: PROJ4(1); break;
+            case 2: PROJ4(2); break;
+            case 4: PROJ4(4); break;
+            case 8: PROJ4(8); break;
+            case 16: PROJ4(16); break;
+            default: PROJ4(32); break;
+        }
+#undef PROJ4
+    } else {
+        k_gat_attn_proj_bwd1<<<(unsigned)nblk, 256, 0, s>>>(T, M, H, F, ldt, a_l, a_r, del, der, dT, rpb > 0 ? rpb : 1,
+                                                            part);
+    }
     reduce_splits(part, nblk, 2 * (int64_t)W, W, W, W, da_l, s);
     reduce_splits(part + W, nblk, 2 * (int64_t)W, W, W, W, da_r, s);
     return check_launch("k_gat_attn_proj_bwd");
