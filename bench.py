@@ -304,8 +304,12 @@ def kernel_bytes(cfg, g):
             "gat_der1": bytes_gat_der(E_f, n, heads, hid), "gat_der2": bytes_gat_der(E_f, n, 1, C)}
 
 
-# our kernels launched per training epoch (counted from the ncu launch list, profiles/r1/launches_*.csv)
-LAUNCHES_PER_EPOCH = {"gcn": 20, "gat": 31, "appnp": 47, "rgcn": 12, "rgcnb": 19}
+# our kernels launched per step of each workload, counted from ncu launch lists of this code
+# (tools/count_launches.sh: kernels between two consecutive epochs' Adam step counters; the count depends on
+# the graph -- degree buckets present -- and the dense shapes).  Reddit: GCN 20 + GAT 31.
+LAUNCHES_PER_STEP = {"reddit": 51, "cora_gcn": 24, "corafull_gat": 35, "physics_appnp": 71, "am_rgcn": 21,
+                     "aifb_rgcnb": 25, "mutag_rgcnb": 28, "bgs_rgcnb": 28}
+LAUNCHES_PER_EPOCH_REDDIT = {"gcn": 20, "gat": 31}
 
 
 def main():
@@ -530,7 +534,9 @@ def main():
                "seconds": t}
 
     if rank == 0:
-        gpu_launches = args.steps * sum(LAUNCHES_PER_EPOCH[k] for k in models)
+        per_step = (sum(LAUNCHES_PER_EPOCH_REDDIT[k] for k in models) if args.workload == "reddit"
+                    else LAUNCHES_PER_STEP[args.workload])
+        gpu_launches = args.steps * per_step
         line = {
             "metric": "GAT/GCN train epoch ms and edges/s at 1/2/4/8 B200; achieved HBM GB/s",
             "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
