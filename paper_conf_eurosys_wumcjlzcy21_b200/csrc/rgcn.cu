@@ -29,30 +29,32 @@ struct RgcnRowArgs {
     const float* Yact;                  // dX only: fused activation backward, out *= act'(Yact)
 };
 
-// stage W (or W^T) as [R][Fg][Fop] with Fop = round4(Fo), zero padded, consecutive types kStagePad floats apart
-// beyond their Fg*Fop block: the 32/RL row groups of a warp flush runs of different types at the same in-block
-// offset, and without the pad every W_r block starts on the same bank (Fg*Fop is a multiple of 32 for the
-// 16-wide layers), an up-to-8-way shared-memory bank conflict on every flush load
-constexpr int kStagePad = 4;
-__host__ __device__ inline int64_t w_stride(int Fg, int Fop) { return (int64_t)Fg * Fop + kStagePad; }
+// stage W (or W^T) as [R][Fg][Fop] with Fop = round4(Fo), zero padded; consecutive W_r blocks start at a stride
+// of 16 mod 32 floats: the 32/RL row groups of a warp flush runs of different types at the same in-block offset, and a
+// 128-bit shared load is served 8 lanes (two 4-lane groups) per wavefront, so two groups whose types differ in parity
+// never share a bank, and equal types broadcast (with a 4-float pad, measured on the AM shape: 37 % of the flush
+// wavefronts were bank conflicts)
+__host__ __device__ inline int64_t w_stride(int Fg, int Fop) { return (((int64_t)Fg * Fop + 31) & ~(int64_t)31) + 16; }
 
 __device__ void stage_w(const RgcnRowArgs& a, float* Ws) {
+    // 32-bit index math: the staged table fits in shared memory, and 64-bit div/mod made the staging of the 136 KB
+    // AM table cost tens of microseconds per CTA
     const int Fop = (a.Fo + 3) & ~3;
-    const int64_t n = (int64_t)a.R * a.Fg * Fop;
-    const int64_t ws = w_stride(a.Fg, Fop);
-    for (int64_t idx = threadIdx.x; idx < n; idx += blockDim.x) {
-        const int j = (int)(idx % Fop);
-        const int64_t ri = idx / Fop;
-        const int i = (int)(ri % a.Fg);
-        const int r = (int)(ri / a.Fg);
+    const int n = a.R * a.Fg * Fop;
+    const int ws = (int)w_stride(a.Fg, Fop);
+    for (int idx = threadIdx.x; idx < n; idx += blockDim.x) {
+        const int j = idx % Fop;
+        const int ri = idx / Fop;
+        const int i = ri % a.Fg;
+        const int r = ri / a.Fg;
         float w = 0.f;
         if (j < a.Fo) {
             // forward: Ws[r][i][j] = W[r][i][j] (i in F_in, j in F_out)
             // dX     : Ws[r][j'][i'] = W[r][i'][j'] with gathered index = j' (F_out), output = i' (F_in)
-            w = a.transpose ? __ldg(a.W + ((int64_t)r * a.Fo + j) * a.Fg + i)
-                            : __ldg(a.W + ((int64_t)r * a.Fg + i) * a.Fo + j);
+            w = a.transpose ? __ldg(a.W + (r * a.Fo + j) * a.Fg + i)
+                            : __ldg(a.W + ri * a.Fo + j);
         }
-        Ws[r * ws + (int64_t)i * Fop + j] = w;
+        Ws[r * ws + i * Fop + j] = w;
     }
 }
 
@@ -442,7 +444,10 @@ static seastar_status launch_buckets(const IndexSet& x, RgcnRowArgs a, size_t sm
     constexpr int WH = L <= 4 ? 32 : 16;     // hub rows: one CTA of WH warps (registers allow 1024 threads at L <= 4)
     SS_TRY((launch_rows<L, 32, WH, 32 * WH>(hb, smem, s)));
     SS_TRY((launch_rows<L, 32>(hi, smem, s)));
-    constexpr int RLo = L < 4 ? 4 : L;
+#ifndef RGCN_RLO
+#define RGCN_RLO 4   // lanes per low-degree row (>= L): A/B knob for tools/build_variant.sh
+#endif
+    constexpr int RLo = L < RGCN_RLO ? RGCN_RLO : L;
     return launch_rows<L, RLo>(lo, smem, s);
 }
 
