@@ -1,4 +1,5 @@
 # A/B of the low-degree R-GCN row mapping (lanes per row) on the AM shape: bench timers + R-GCN parity per variant
+# (needs variants/ on the box: drop the variants/ line from .gpurunignore for that call)
 LIB=paper_conf_eurosys_wumcjlzcy21_b200/libseastar.so
 mkdir -p gpurun_out
 cp $LIB /tmp/libseastar_orig.so
