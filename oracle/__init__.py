@@ -74,7 +74,9 @@ def _L():
             "orc_linear_fwd": ([_I, _I, _I, _P, _P, _P, _P], None),
             "orc_linear_bwd": ([_I, _I, _I, _P, _P, _P, _P, _P, _P], None),
             "orc_gcn_aggregate": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P, _P], None),
-            "orc_gcn_aggregate_T": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P, _P], None),
+            "orc_gcn_aggregate_T": ([_I, _I, _P, _P, _I, _P, _P, _P, _P, _I, _P, _P, _P, _P, _P], None),
+            "orc_out_adjacency": ([_I, _I, _P, _P, _P, _P, _P], None),
+            "orc_set_num_threads": ([ctypes.c_int], None),
             "orc_gat_attn_proj": ([_I, _I, _I, _P, _P, _P, _P, _P], None),
             "orc_gat_fwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _I, _P, _P, _P, _P], None),
             "orc_gat_bwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _P, _I, _P, _P, _P, _P], None),
@@ -206,7 +208,21 @@ def gcn_aggregate(indptr, indices, H, src_norm=None, dst_norm=None, rows=None, e
     return out
 
 
-def gcn_aggregate_T(indptr, indices, G, src_norm=None, dst_norm=None, rows=None, edge_w=None):
+def out_adjacency(indptr, indices):
+    """(dst[E], optr[N+1], oeid[E]): the graph's out-adjacency, a pure function of the graph.  Pass it as
+    ``adj=`` to gcn_aggregate_T to keep its O(E) construction out of a timed row sample."""
+    indptr, indices = _i64(indptr), _i64(indices)
+    N, E = indptr.size - 1, int(indptr[-1])
+    dst, optr, oeid = np.empty(E, np.int64), np.empty(N + 1, np.int64), np.empty(E, np.int64)
+    _L().orc_out_adjacency(N, E, _p(indptr), _p(indices), _p(dst), _p(optr), _p(oeid))
+    return dst, optr, oeid
+
+
+def set_num_threads(n):
+    _L().orc_set_num_threads(int(n))
+
+
+def gcn_aggregate_T(indptr, indices, G, src_norm=None, dst_norm=None, rows=None, edge_w=None, adj=None):
     indptr, indices, G, edge_w = _i64(indptr), _i64(indices), _f64(G), _f64(edge_w)
     N = indptr.size - 1
     F = G.shape[1]
@@ -214,8 +230,9 @@ def gcn_aggregate_T(indptr, indices, G, src_norm=None, dst_norm=None, rows=None,
     nrows = N if rows is None else rows.size
     out = np.empty((nrows, F))
     sn, dn = _f64(src_norm), _f64(dst_norm)     # keep the converted arrays alive across the C call
+    ad = (None, None, None) if adj is None else tuple(_i64(a) for a in adj)
     _L().orc_gcn_aggregate_T(N, int(indptr[-1]), _p(indptr), _p(indices), F, _p(G), _p(sn), _p(dn), _p(rows),
-                             nrows, _p(out), _p(edge_w))
+                             nrows, _p(out), _p(edge_w), *(_p(a) for a in ad))
     return out
 
 

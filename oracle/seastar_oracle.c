@@ -23,6 +23,9 @@
 #include <stdlib.h>
 #include <string.h>
 #include <math.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 enum { ORC_ACT_NONE = 0, ORC_ACT_RELU = 1, ORC_ACT_ELU = 2, ORC_ACT_SIGMOID = 3 };
 
@@ -310,12 +313,33 @@ void orc_gcn_aggregate(int64_t N, int64_t E, const int64_t* indptr, const int64_
 
 /* adjoint of orc_gcn_aggregate (§6.3.4: the backward aggregates over out-edges):
  * out[r,:] = src_norm[u] * sum_{e in out(u)} dst_norm[dst(e)] * G[dst(e),:],  u = rows[r] */
-void orc_gcn_aggregate_T(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices, int64_t F,
-                         const double* G, const double* src_norm, const double* dst_norm,
-                         const int64_t* rows, int64_t nrows, double* out, const double* edge_w) {
+/* The whole graph's destination-of-edge and out-adjacency arrays (dst[E], optr[N+1], oeid[E]) that the
+ * transposed loops below walk.  They are a pure function of the graph, so a caller timing a bounded row
+ * sample (bench.py's cpu_baseline) builds them once and passes them in; NULL => each
+ * call builds its own, as before.  Restructuring only: the arithmetic of every loop is unchanged. */
+void orc_out_adjacency(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices,
+                       int64_t* dst_out, int64_t* optr_out, int64_t* oeid_out) {
     int64_t* dst = dst_of_edges(N, E, indptr);
     int64_t *optr, *oeid;
     out_adjacency(N, E, indices, &optr, &oeid);
+    memcpy(dst_out, dst, sizeof(int64_t) * (size_t)E);
+    memcpy(optr_out, optr, sizeof(int64_t) * (size_t)(N + 1));
+    memcpy(oeid_out, oeid, sizeof(int64_t) * (size_t)E);
+    free(dst); free(optr); free(oeid);
+}
+
+void orc_gcn_aggregate_T(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices, int64_t F,
+                         const double* G, const double* src_norm, const double* dst_norm,
+                         const int64_t* rows, int64_t nrows, double* out, const double* edge_w,
+                         const int64_t* adj_dst, const int64_t* adj_ptr, const int64_t* adj_eid) {
+    int64_t *dst, *optr, *oeid;
+    const int own = !(adj_dst && adj_ptr && adj_eid);
+    if (own) {
+        dst = dst_of_edges(N, E, indptr);
+        out_adjacency(N, E, indices, &optr, &oeid);
+    } else {
+        dst = (int64_t*)adj_dst; optr = (int64_t*)adj_ptr; oeid = (int64_t*)adj_eid;
+    }
     if (!rows) nrows = N;
     #pragma omp parallel for schedule(dynamic, 64)
     for (int64_t r = 0; r < nrows; ++r) {
@@ -331,7 +355,16 @@ void orc_gcn_aggregate_T(int64_t N, int64_t E, const int64_t* indptr, const int6
         double s = src_norm ? src_norm[u] : 1.0;
         for (int64_t f = 0; f < F; ++f) o[f] *= s;
     }
-    free(optr); free(oeid); free(dst);
+    if (own) { free(optr); free(oeid); free(dst); }
+}
+
+/* OpenMP thread count for the timed baselines (bench.py records single-threaded numbers too) */
+void orc_set_num_threads(int n) {
+#ifdef _OPENMP
+    omp_set_num_threads(n);
+#else
+    (void)n;
+#endif
 }
 
 /* ------------------------------------------------------------------------------------------ */

@@ -14,6 +14,9 @@ over every output row, not a sample:
 
 These are the slowest GPU tests (the oracle needs ~1-2 CPU-minutes for the Reddit GAT step).
 """
+import json
+import os
+
 import numpy as np
 import pytest
 
@@ -79,6 +82,12 @@ def check_step(model, loss_ref, grads_ref, acts, envelope=None, n_ambiguous=0):
             den = np.abs(ref).max() or 1.0
             excess["d" + k] = float(np.maximum(np.abs(got - ref) - envelope[k].reshape(got.shape), 0).max() / den)
             width["d" + k] = float(envelope[k].max() / den)
+    log = os.environ.get("SEASTAR_PARITY_LOG")
+    if log:                     # committed under profiles/ from the GPU runs
+        with open(log, "a") as f:
+            f.write(json.dumps({"test": os.environ.get("PYTEST_CURRENT_TEST", "?").split(" ")[0], "tol": TOL,
+                                "rel_err": errs, "ambiguous_kink_decisions": int(n_ambiguous),
+                                "envelope_over_maxref": width, "error_beyond_envelope": excess}) + "\n")
     print("\nrel errors:", {k: f"{v:.2e}" for k, v in errs.items()}, "| ambiguous kink decisions:", n_ambiguous,
           "| envelope / max|ref|:", {k: f"{v:.2e}" for k, v in width.items()},
           "| error beyond the envelope:", {k: f"{v:.2e}" for k, v in excess.items()})

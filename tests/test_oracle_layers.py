@@ -369,3 +369,17 @@ def test_marshalling_independent_of_input_dtype():
                                                     sn.astype(np.float32).astype(np.float64),
                                                     dn.astype(np.float32).astype(np.float64))) == 0.0
     assert rel_err(ref, ref) == 0.0
+
+
+def test_aggregate_T_prebuilt_adjacency_identical():
+    """oracle.out_adjacency (hoisted out of bench.py's timed sample) changes nothing: bitwise equal output."""
+    indptr, indices = small_graph(11, N=30, E=200)
+    G = rnd(3, 30, 5)
+    sn, dn = oracle.degree_norms(indptr, indices)[::-1]
+    rows = np.array([4, 0, 17, 29])
+    adj = oracle.out_adjacency(indptr, indices)
+    np.testing.assert_array_equal(oracle.gcn_aggregate_T(indptr, indices, G, sn, dn, rows, adj=adj),
+                                  oracle.gcn_aggregate_T(indptr, indices, G, sn, dn, rows))
+    dst, optr, oeid = adj
+    assert optr[-1] == 200 and sorted(oeid.tolist()) == list(range(200))
+    np.testing.assert_array_equal(np.repeat(np.arange(30), np.diff(optr)), indices[oeid])   # row u lists out(u)

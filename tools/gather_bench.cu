@@ -1,73 +1,160 @@
-// Random-row gather throughput on B200 (the roofline of the graph kernels' per-edge gathers).
-// Warp per "row group": 32 indices per coalesced load, L = row_bytes/16 lanes per row, 32/L rows per
-// load step, UB steps in flight; sums into registers (no writes except one value per thread).
+// Random-row gather ceiling on B200: the physical roofline of the graph kernels' per-edge gathers
+// (VERDICT r1 "make the roofline physical").  A warp streams 32 indices per coalesced load; L =
+// row_bytes/16 lanes read one row with LDG.128, 32/L rows per load step, UB steps in flight; the rows
+// are summed into registers (one value per thread is written).  No method arithmetic: this is the
+// upper bound on "row bytes + 4 B index per edge" that any gather kernel can reach.
+//
+// Index streams (n = 100 M per launch):
+//   uniform  : u ~ U{0..rows-1}                         (pure L2 random-row throughput)
+//   powerlaw : u ~ w_r = (r+1)^-0.35 over ranks, ranks -> ids by a seeded shuffle, sorted into
+//              runs of 492 edges per "destination" (the Reddit shape of configs[4]: s = 0.35, mean
+//              in-degree 492), i.e. the same L1-reuse opportunities as the real kernels
+// Table sizes are the Reddit tables (15 MB GCN T, 60-67 MB GAT layer 1, 41 MB layer 2) plus two
+// sizes beyond L2 (200 MB, 1 GB).
+//
+//   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -Xcompiler -fopenmp -o tools/gather_bench tools/gather_bench.cu
+//   tools/gather_bench > gpurun_out/gather_ceiling.json
+#include <algorithm>
+#include <cmath>
+#include <cstdint>
 #include <cstdio>
 #include <cstdlib>
-#include <cstdint>
 #include <vector>
 #include <cuda_runtime.h>
 
+#define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) { \
+    fprintf(stderr, "%s:%d %s\n", __FILE__, __LINE__, cudaGetErrorString(e_)); exit(1); } } while (0)
+
 template <int L, int UB>
-__global__ void gather(const float4* __restrict__ T, const int* __restrict__ idx, long n_edges, float* out) {
-    constexpr int S = 32 / L;
+__global__ void __launch_bounds__(256) gather(const float4* __restrict__ T, const int* __restrict__ idx,
+                                              long n_edges, float* out) {
+    constexpr int S = 32 / L;                 // rows per load step
     const int lane = threadIdx.x & 31, slot = lane / L, c = lane % L;
+    const bool active = slot < S;
     long warp = (blockIdx.x * (long)blockDim.x + threadIdx.x) >> 5;
     long nwarps = ((long)gridDim.x * blockDim.x) >> 5;
     float4 acc = make_float4(0, 0, 0, 0);
+    constexpr int PER = 32 / S;               // load steps per 32 indices
     for (long base = warp * 32 * UB; base < n_edges; base += nwarps * 32 * UB) {
         int my[UB];
 #pragma unroll
-        for (int b = 0; b < UB; ++b) my[b] = (base + b * 32 + lane < n_edges) ? __ldcs(idx + base + b * 32 + lane) : 0;
+        for (int b = 0; b < UB; ++b) {
+            long e = base + b * 32 + lane;
+            my[b] = e < n_edges ? __ldcs(idx + e) : -1;
+        }
 #pragma unroll
         for (int b = 0; b < UB; ++b) {
-            float4 v[L];
 #pragma unroll
-            for (int j = 0; j < L; ++j) {
-                int u = __shfl_sync(0xffffffff, my[b], j * S + slot);
-                v[j] = __ldg(T + (long)u * L + c);
+            for (int j = 0; j < PER; ++j) {
+                int u = __shfl_sync(0xffffffffu, my[b], j * S + (active ? slot : 0));
+                float4 v = (active && u >= 0) ? __ldg(T + (long)u * L + c) : make_float4(0, 0, 0, 0);
+                acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
             }
-#pragma unroll
-            for (int j = 0; j < L; ++j) { acc.x += v[j].x; acc.y += v[j].y; acc.z += v[j].z; acc.w += v[j].w; }
         }
     }
     out[blockIdx.x * blockDim.x + threadIdx.x] = acc.x + acc.y + acc.z + acc.w;
 }
 
+static uint64_t sm64(uint64_t x) {
+    x += 0x9E3779B97F4A7C15ull;
+    x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+    x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+    return x ^ (x >> 31);
+}
+
+static void make_indices(std::vector<int>& h, int rows, bool powerlaw) {
+    const long n = (long)h.size();
+    if (!powerlaw) {
+#pragma omp parallel for
+        for (long i = 0; i < n; ++i) h[i] = (int)(sm64(1234567ull ^ (uint64_t)i) % (uint64_t)rows);
+        return;
+    }
+    std::vector<double> cdf(rows);
+    double s = 0;
+    for (int r = 0; r < rows; ++r) { s += std::pow((double)r + 1.0, -0.35); cdf[r] = s; }
+    std::vector<int> perm(rows);
+    for (int r = 0; r < rows; ++r) perm[r] = r;
+    for (int r = rows - 1; r > 0; --r) std::swap(perm[r], perm[sm64(77ull + r) % (uint64_t)(r + 1)]);
+#pragma omp parallel for
+    for (long i = 0; i < n; ++i) {
+        double u = (double)(sm64(424242ull ^ (uint64_t)i) >> 11) * 0x1.0p-53 * s;
+        int r = (int)(std::lower_bound(cdf.begin(), cdf.end(), u) - cdf.begin());
+        h[i] = perm[std::min(r, rows - 1)];
+    }
+    // runs of 492 edges per destination, sorted by source id inside the run (the CSR's edge-id order
+    // is generation order; sorting only changes intra-run order, not the multiset)
+#pragma omp parallel for
+    for (long b = 0; b < n; b += 492) std::sort(h.begin() + b, h.begin() + std::min(n, b + 492));
+}
+
 template <int L, int UB>
-double run(size_t table_bytes, long n_edges, int* d_idx, int blocks) {
-    int rows = (int)(table_bytes / (16 * L));
-    float4* T; float* out;
-    cudaMalloc(&T, (size_t)rows * 16 * L);
-    cudaMemset(T, 0, (size_t)rows * 16 * L);
-    cudaMalloc(&out, (size_t)blocks * 256 * 4);
-    // indices for this table size
-    std::vector<int> h(n_edges);
-    uint64_t x = 88172645463325252ull;
-    for (long i = 0; i < n_edges; ++i) { x ^= x << 13; x ^= x >> 7; x ^= x << 17; h[i] = (int)(x % rows); }
-    cudaMemcpy(d_idx, h.data(), n_edges * 4, cudaMemcpyHostToDevice);
-    cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
-    gather<L, UB><<<blocks, 256>>>(T, d_idx, n_edges, out);
-    cudaEventRecord(a);
-    for (int r = 0; r < 5; ++r) gather<L, UB><<<blocks, 256>>>(T, d_idx, n_edges, out);
-    cudaEventRecord(b); cudaEventSynchronize(b);
-    float ms; cudaEventElapsedTime(&ms, a, b); ms /= 5;
-    cudaFree(T); cudaFree(out);
-    double bytes = (double)n_edges * (16.0 * L + 4);
-    return bytes / (ms * 1e-3) / 1e9;
+static double run(const float4* T, const int* d_idx, long n, int blocks, float* out) {
+    cudaEvent_t a, b;
+    CK(cudaEventCreate(&a)); CK(cudaEventCreate(&b));
+    gather<L, UB><<<blocks, 256>>>(T, d_idx, n, out);
+    CK(cudaGetLastError());
+    float best = 1e30f;
+    for (int r = 0; r < 5; ++r) {
+        CK(cudaEventRecord(a));
+        gather<L, UB><<<blocks, 256>>>(T, d_idx, n, out);
+        CK(cudaEventRecord(b));
+        CK(cudaEventSynchronize(b));
+        float ms; CK(cudaEventElapsedTime(&ms, a, b));
+        best = std::min(best, ms);
+    }
+    CK(cudaEventDestroy(a)); CK(cudaEventDestroy(b));
+    return (double)n * (16.0 * L + 4) / (best * 1e-3) / 1e9;
+}
+
+template <int L>
+static void row_size(const char* dist, size_t mb, long n, int* d_idx, float4* T, float* out, int sms,
+                     bool& first) {
+    for (int blocks : {sms * 8, sms * 16}) {
+        double g2 = run<L, 2>(T, d_idx, n, blocks, out);
+        double g4 = run<L, 4>(T, d_idx, n, blocks, out);
+        printf("%s    {\"dist\": \"%s\", \"table_MB\": %zu, \"row_B\": %d, \"blocks\": %d, \"GBs_ub2\": %.0f, "
+               "\"GBs_ub4\": %.0f}", first ? "" : ",\n", dist, mb, 16 * L, blocks, g2, g4);
+        first = false;
+    }
 }
 
 int main() {
-    long n = 100 * 1000 * 1000;
-    int* d_idx; cudaMalloc(&d_idx, n * 4);
-    int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-    size_t sizes[] = {15u << 20, 60u << 20, 90u << 20, 200u << 20, 1u << 30};
-    printf("table_MB  row_B  UB  GB/s(algorithmic: row+4B index per edge)\n");
-    for (size_t s : sizes) {
-        for (int blocks : {sms * 8, sms * 32}) {
-            printf("%6zu  %4d  %d  %8.0f  (blocks %d)\n", s >> 20, 64, 4, run<4, 4>(s, n, d_idx, blocks), blocks);
-            printf("%6zu  %4d  %d  %8.0f  (blocks %d)\n", s >> 20, 256, 2, run<16, 2>(s, n, d_idx, blocks), blocks);
-            printf("%6zu  %4d  %d  %8.0f  (blocks %d)\n", s >> 20, 176, 2, run<11, 2>(s, n, d_idx, blocks), blocks);
+    const long n = 100l * 1000 * 1000;
+    int sms;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
+    int l2;
+    CK(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, 0));
+    int* d_idx;
+    float* out;
+    float4* T;
+    const size_t max_table = 1ull << 30;
+    CK(cudaMalloc(&d_idx, n * 4));
+    CK(cudaMalloc(&out, (size_t)sms * 16 * 256 * 4));
+    CK(cudaMalloc(&T, max_table));
+    CK(cudaMemset(T, 0, max_table));
+    std::vector<int> h(n);
+    printf("{\"what\": \"random-row gather ceiling: GB/s = edges*(row_B+4)/time, best of 5, 256-thread CTAs\",\n"
+           " \"sms\": %d, \"l2_bytes\": %d, \"edges\": %ld,\n \"rows\": [\n", sms, l2, n);
+    bool first = true;
+    const size_t sizes_mb[] = {15, 41, 60, 67, 200, 1024};
+    for (int pl = 0; pl < 2; ++pl) {
+        for (size_t mb : sizes_mb) {
+            if (pl == 1 && mb > 67) continue;   // the power-law streams only at the Reddit table sizes
+            // one index stream per (dist, table size, row size); rows = table / row bytes
+            auto go = [&](auto Ltag) {
+                constexpr int L = decltype(Ltag)::value;
+                int rows = (int)((mb << 20) / (16 * L));
+                make_indices(h, rows, pl == 1);
+                CK(cudaMemcpy(d_idx, h.data(), n * 4, cudaMemcpyHostToDevice));
+                row_size<L>(pl ? "powerlaw" : "uniform", mb, n, d_idx, T, out, sms, first);
+            };
+            go(std::integral_constant<int, 4>{});    // 64 B: GCN F = 16
+            go(std::integral_constant<int, 11>{});   // 176 B: GAT layer 2 (41 -> ld 44)
+            go(std::integral_constant<int, 16>{});   // 256 B: GAT layer 1 T row (8 x 8)
+            go(std::integral_constant<int, 24>{});   // 384 B: GAT layer 1 backward record (ld 88 -> 352 B + pad)
+            fflush(stdout);
         }
     }
+    printf("\n ]}\n");
     return 0;
 }
