@@ -16,6 +16,8 @@ is fixed as N grows ("strong" scaling); the step time is the max over ranks.
 from __future__ import annotations
 
 import argparse
+import glob
+import hashlib
 import json
 import os
 import statistics
@@ -43,7 +45,9 @@ def parse():
     ap.add_argument("--cuda-graph", default="auto", choices=["auto", "on", "off"],
                     help="replay each model epoch from a CUDA graph (auto: on one GPU)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-sample-edges", type=int, default=10_000_000)
+    ap.add_argument("--cpu-sample-frac", type=float, default=1.0,
+                    help="fraction of the Reddit in-edges the cpu_baseline oracle sample covers (--impl reference: /8 "
+                         "per step)")
     ap.add_argument("--workload", default="reddit", choices=list(synth.CONFIGS),
                     help="BASELINE config to train (default: configs[4], the Reddit-shaped GCN+GAT headline)")
     return ap.parse_args()
@@ -94,6 +98,92 @@ def bytes_gat_der(E, n, H, F):
     W = H * F
     ldd = (W + 3) // 4 * 4 + 4 * H
     return E * (4 + 4 * H + 4 * W) + n * (8 + 4 * ldd + 4 * H)
+
+
+# ------------------------------------------------------------------------------------------
+# provenance: source hash, input hash, host description
+# ------------------------------------------------------------------------------------------
+def lib_src_sha() -> str:
+    """SHA-256 over libseastar.so's sources (csrc/* and include/seastar.h): identifies the kernels a
+    committed ncu traffic capture belongs to."""
+    h = hashlib.sha256()
+    files = sorted(glob.glob(os.path.join(ROOT, "paper_conf_eurosys_wumcjlzcy21_b200", "csrc", "*")))
+    for f in files + [os.path.join(ROOT, "include", "seastar.h")]:
+        h.update(os.path.basename(f).encode())
+        with open(f, "rb") as fh:
+            h.update(fh.read())
+    return h.hexdigest()
+
+
+def inputs_sha(w) -> str:
+    """SHA-256 of the step's seeded inputs (graph, features, labels, initial parameters), in a fixed order."""
+    h = hashlib.sha256()
+    for k in ("indptr", "indices", "etypes", "X", "labels"):
+        a = w.get(k)
+        if a is not None:
+            h.update(k.encode())
+            h.update(memoryview(np.ascontiguousarray(a)).cast("B"))
+    for m in ("gcn", "gat", "appnp", "rgcn", "rgcnb"):
+        for k, a in sorted((w.get(m) or {}).items()):
+            h.update(f"{m}.{k}".encode())
+            h.update(memoryview(np.ascontiguousarray(a)).cast("B"))
+    return h.hexdigest()
+
+
+def host_info() -> dict:
+    info = {"nproc": os.cpu_count()}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            if k.strip() in ("Model name", "Socket(s)", "Core(s) per socket", "Thread(s) per core"):
+                info[k.strip()] = v.strip()
+    except Exception:
+        pass
+    return info
+
+
+# ------------------------------------------------------------------------------------------
+# physical ceilings: the measured L2 random-row gather ceiling and the per-kernel ncu traffic at HEAD
+# ------------------------------------------------------------------------------------------
+GATHER_CEILING = os.path.join(ROOT, "profiles", "r2", "gather_ceiling.json")
+
+
+def traffic_path(workload: str) -> str:
+    return os.path.join(ROOT, "profiles", "r2", f"ncu_traffic_{workload}.json")
+
+
+def l2_ceiling(row_b: int):
+    """Best measured gather GB/s (row_B + 4 B index per edge, power-law index stream, N = 232,965-row table) at
+    the measured row size nearest to row_b (tools/gather_bench.cu on B200), or None."""
+    try:
+        rows = [r for r in json.load(open(GATHER_CEILING))["rows"] if r.get("reddit_rows") and r["dist"] == "powerlaw"]
+    except Exception:
+        return None
+    if not rows:
+        return None
+    r = min(rows, key=lambda r: abs(r["row_B"] - row_b))
+    return {"GB/s": float(r["GBs_best"]), "row_B": r["row_B"], "table_MB": r["table_MB"]}
+
+
+def gathered_row_bytes(cfg) -> dict:
+    """Bytes of the row each bench kernel gathers per edge (the gather-ceiling lookup key)."""
+    ld = lambda f: (f + 3) // 4 * 4
+    if cfg.model == "appnp":
+        return {"appnp_fwd": 4 * ld(cfg.classes), "appnp_bwd": 4 * ld(cfg.classes)}
+    if cfg.model == "rgcn":
+        return {"rgcn_fwd1": 4 * ld(cfg.F_in)}
+    if cfg.model == "rgcnb":
+        B = cfg.extra["bases"]
+        return {"rgcnb_fwd1": 4 * B * cfg.hidden, "rgcnb_bwd1": 4 * B * cfg.hidden}
+    heads, hid, C = cfg.heads, cfg.extra.get("gat_hidden", cfg.hidden), cfg.classes
+    rec = lambda H, F: 4 * (ld(H * F) + 4 * H)
+    # GAT forward / der: the T row (the el scalars come from a second, 8x smaller table: one extra sector per edge,
+    # counted in the kernel's algorithmic bytes but not in the ceiling's row size)
+    return {"gcn_fwd1": 4 * ld(cfg.hidden), "gcn_bwd2": 4 * ld(cfg.hidden),
+            "gat_fwd1": 4 * ld(heads * hid), "gat_bwd1": rec(heads, hid),
+            "gat_fwd2": 4 * ld(C), "gat_bwd2": rec(1, C),
+            "gat_der1": 4 * ld(heads * hid), "gat_der2": 4 * ld(C)}
 
 
 # ------------------------------------------------------------------------------------------
@@ -153,36 +243,48 @@ class Clocks:
 # ------------------------------------------------------------------------------------------
 # CPU oracle baseline (bounded sample of the same workload) -- the only use of oracle/ here
 # ------------------------------------------------------------------------------------------
-def oracle_sample(ip, ix, X, sample_edges, seed=0):
-    """Oracle fwd+bwd aggregations of both GCN layers (F=16) and the GAT forward layers (8x8, 1x41)
-    over the first vertices (by id; ids are shuffled) covering ~sample_edges edges.  Returns
-    (edges processed, seconds, description)."""
+_ADJ = {}
+
+
+def oracle_sample(ip, ix, X, frac=1.0, gat_bwd=True):
+    """The graph passes of one GCN epoch and one GAT epoch on the oracle (plain fp64 edge loops, OpenMP over rows):
+    GCN forward and transposed aggregations of both layers (F = 16) and GAT forward (+ backward when gat_bwd; the
+    oracle's GAT backward always visits the whole graph: its dst-major der pass is over all N) of both layers
+    (8 x 8 and 1 x 41), for the first vertex ids (ids are shuffled) covering `frac` of the in-edges (1.0 = the
+    whole graph).  Dense transforms, loss and Adam are not timed.  Returns (edges, seconds, description) with
+    edges = 2 * (sampled in-edges): the same "E per model epoch" count as the GPU arm's value."""
     import oracle
     N = len(ip) - 1
     deg_in = np.diff(ip)
-    k = int(np.searchsorted(np.cumsum(deg_in), sample_edges)) + 1
-    k = min(k, N)
-    rows = np.arange(k, dtype=np.int64)
-    outdeg = np.bincount(ix, minlength=N)
-    e_in, e_out = int(deg_in[:k].sum()), int(outdeg[:k].sum())
+    E = int(ip[-1])
+    k = N if frac >= 1.0 else min(N, int(np.searchsorted(np.cumsum(deg_in), frac * E)) + 1)
+    rows = None if k == N else np.arange(k, dtype=np.int64)
+    e_in = int(deg_in[:k].sum())
     in_n, out_n = oracle.degree_norms(ip, ix)
     H16 = X[:, :16].astype(np.float64)
     T64 = X[:, :64].reshape(N, 8, 8).astype(np.float64)
     T41 = X[:, 64:105].reshape(N, 1, 41).astype(np.float64)
     el8, er8 = X[:, 105:113].astype(np.float64), X[:, 113:121].astype(np.float64)
     el1, er1 = X[:, 121:122].astype(np.float64), X[:, 122:123].astype(np.float64)
+    key = (id(ip), id(ix))                  # a function of the graph: built once, outside the timed sample
+    if _ADJ.get("key") != key:
+        _ADJ.update(key=key, adj=oracle.out_adjacency(ip, ix))
+    adj = _ADJ["adj"]
     t0 = time.perf_counter()
     for _ in range(2):     # GCN layers 1 and 2: forward aggregation, backward (transposed) aggregation
         oracle.gcn_aggregate(ip, ix, H16, out_n, in_n, rows)
-        oracle.gcn_aggregate_T(ip, ix, H16, out_n, in_n, rows)
-    oracle.gat_fwd(ip, ix, T64, el8, er8, 0.2, rows)
-    oracle.gat_fwd(ip, ix, T41, el1, er1, 0.2, rows)
+        oracle.gcn_aggregate_T(ip, ix, H16, out_n, in_n, rows, adj=adj)
+    for T, el, er in ((T64, el8, er8), (T41, el1, er1)):     # GAT layers: forward, backward (the dA = T stand-in)
+        oracle.gat_fwd(ip, ix, T, el, er, 0.2, rows)
+        if gat_bwd:
+            oracle.gat_bwd(ip, ix, T, el, er, T, 0.2, rows, adj=adj)
     dt = time.perf_counter() - t0
-    edges = 2 * (e_in + e_out) + 2 * e_in
-    desc = (f"oracle fwd+bwd GCN aggregations (F=16, 2 layers) and GAT forward layers (8x8, 1x41) for the "
-            f"first {k} vertex ids ({e_in} in-edges, {e_out} out-edges) of the Reddit-shaped graph; "
-            f"edges/s = aggregated edge visits / wall time")
-    return edges, dt, desc
+    desc = (f"oracle graph passes of one GCN epoch (fwd + transposed aggregations, F=16, 2 layers) and one GAT epoch "
+            f"({'fwd + bwd' if gat_bwd else 'fwd only'}, 8x8 and 1x41) over {'all' if rows is None else f'the first {k}'} vertex ids ({e_in} of {E} "
+            f"in-edges) of the Reddit-shaped graph; dense transforms, loss and Adam not timed; the graph's "
+            f"out-adjacency built once outside the timed region (like the GPU's graph_create); edges/s = 2 x sampled "
+            f"in-edges / wall time")
+    return 2 * e_in, dt, desc
 
 
 def oracle_step(w, names):
@@ -219,7 +321,7 @@ def omp_threads():
 def run_reference(args, rank, world):
     """--impl reference: the CPU oracle, as written, on the box's host cores (rank 0 only), on the same
     workload, metric and unit as the GPU arm; each step is a bounded sample of that workload (Reddit:
-    the first vertex ids covering ~cpu_sample_edges/4 in-edges; configs[0..3]: one whole step)."""
+    the first vertex ids covering 1/8 of the in-edges; configs[0..3]: one whole step)."""
     if rank != 0:
         return
     w = synth.workload(args.workload)
@@ -228,7 +330,8 @@ def run_reference(args, rank, world):
 
     def one():
         if args.workload == "reddit":
-            return oracle_sample(w["indptr"], w["indices"], w["X"], max(200_000, args.cpu_sample_edges // 4))
+            # bounded per step (K + W steps within minutes): 1/8 of the rows, GAT backward left out (it is whole-graph)
+            return oracle_sample(w["indptr"], w["indices"], w["X"], args.cpu_sample_frac / 8, gat_bwd=False)
         return oracle_step(w, names)
     for _ in range(args.warmup):
         one()
@@ -344,6 +447,9 @@ def main():
         if backend == "gloo":
             dist.init_process_group("gloo")
         else:
+            # NCCL's init lines (rank count, transports, NVLS) go to stderr so the driver can check them
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
             dist.init_process_group("nccl", device_id=dev)
     from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
     from paper_conf_eurosys_wumcjlzcy21_b200.graph import Graph
@@ -351,6 +457,7 @@ def main():
     from paper_conf_eurosys_wumcjlzcy21_b200.models import Comm
     L.seastar_device_check()
 
+    free0 = torch.cuda.mem_get_info(dev)[0]
     t_setup = time.perf_counter()
     w = synth.workload(args.workload)
     cfg = w["cfg"]
@@ -371,6 +478,7 @@ def main():
     models = build_models(args.workload, w, g, X_loc, lab_loc, comm, rows_all, args.model)
     torch.cuda.synchronize()
     setup_s = time.perf_counter() - t_setup
+    min_free = torch.cuda.mem_get_info(dev)[0]
 
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # > 126 MB L2
@@ -378,7 +486,14 @@ def main():
     # per-kernel event timers on the launching stream
     kt = {}
 
+    nvtx = os.environ.get("SEASTAR_NVTX") == "1"     # tools/capture_traffic.sh: ncu renames kernels by range
+
     def timer(name):
+        if nvtx:
+            if name.endswith("_end"):
+                torch.cuda.nvtx.range_pop()
+            else:
+                torch.cuda.nvtx.range_push(name)
         ev = torch.cuda.Event(enable_timing=True)
         ev.record(stream)
         kt.setdefault(name, []).append(ev)
@@ -392,15 +507,29 @@ def main():
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
-    # one CUDA graph per model epoch (single GPU; the partitioned path stays eager around its NCCL calls)
-    use_graph = args.cuda_graph == "on" or (args.cuda_graph == "auto" and world == 1)
+    # one CUDA graph per model epoch; partitioned over NCCL the collectives are captured with the kernels
+    # (a staged gloo process group cannot be captured: it stays eager)
+    use_graph = args.cuda_graph == "on" or (args.cuda_graph == "auto" and (world == 1 or backend == "nccl"))
     runners = models
+    launch_mode = "eager"
+    kernel_names = None
     if use_graph:
         from paper_conf_eurosys_wumcjlzcy21_b200.models import CapturedEpoch
-        runners = {k: CapturedEpoch(m) for k, m in models.items()}
-        for r in runners.values():          # replays stay in the warm-up: the graph path is exercised untimed
-            r.epoch()
-        torch.cuda.synchronize()
+        try:
+            runners = {k: CapturedEpoch(m) for k, m in models.items()}
+            for r in runners.values():          # replays stay in the warm-up: the graph path is exercised untimed
+                r.epoch()
+            torch.cuda.synchronize()
+            launch_mode = "cuda-graph replay per model epoch" + (" (NCCL collectives captured)" if world > 1 else "")
+        except Exception as ex:             # keep the run: eager epochs, and say so in the JSON line
+            runners = models
+            launch_mode = f"eager (capture failed: {type(ex).__name__}: {str(ex)[:120]})"
+            torch.cuda.synchronize()
+        if runners is not models:
+            try:
+                kernel_names = {k: r.kernel_names() for k, r in runners.items()}
+            except Exception as ex:
+                kernel_names = {"error": f"{type(ex).__name__}: {str(ex)[:120]}"}
 
     if world > 1:
         torch.distributed.barrier()
@@ -427,14 +556,19 @@ def main():
     if world > 1:
         torch.distributed.barrier()
     ck = clocks.stop()
+    min_free = min(min_free, torch.cuda.mem_get_info(dev)[0])
 
     # per-kernel durations: eager steps with CUDA events around the hot graph kernels, on the launching stream
     for m in models.values():
         m.timer = timer if hasattr(m, "timer") else None
+    if nvtx:
+        torch.cuda.nvtx.range_push("seastar_timed")
     for _ in range(min(args.steps, 10)):
         flush.zero_()
         step()
     torch.cuda.synchronize()
+    if nvtx:
+        torch.cuda.nvtx.range_pop()
     for m in models.values():
         m.timer = None
 
@@ -464,22 +598,59 @@ def main():
     except Exception:
         pass
     hbm = peaks.get("hbm_gbs", 6650.0)
+    hbm_src = "MEASURED_PEAKS.json hbm_gbs (of measured)" if peaks else "B200_PROFILING.md fallback 6650 GB/s (of fallback)"
+    # ncu DRAM traffic per bench kernel, captured by tools/capture_traffic.sh; used only if captured at these sources
+    src_sha = lib_src_sha()
+    traffic, traffic_src = {}, "none captured for this workload"
+    try:
+        tj = json.load(open(traffic_path(args.workload)))
+        if tj.get("src_sha256") == src_sha:
+            traffic = tj["kernels"]
+            traffic_src = f"{os.path.relpath(traffic_path(args.workload), ROOT)} (captured at this source, sha {src_sha[:12]})"
+        else:
+            traffic_src = f"stale: {os.path.relpath(traffic_path(args.workload), ROOT)} is from other sources; not used"
+    except Exception:
+        pass
+    rowb = gathered_row_bytes(cfg)
+    per_kernel = {}
+    for k, ms in kernels.items():
+        if k not in alg:
+            per_kernel[k] = {"ms": ms}
+            continue
+        a = alg[k] / (ms / 1e3) / 1e9
+        d = {"ms": ms, "algorithmic_bytes": alg[k], "alg_GB/s": a, "alg_over_hbm": a / hbm}
+        ceil = l2_ceiling(rowb[k]) if args.workload == "reddit" and k in rowb else None
+        if ceil:
+            d.update({"l2_gather_peak": ceil["GB/s"], "l2_frac": a / ceil["GB/s"], "gathered_row_B": rowb[k],
+                      "ceiling_row_B": ceil["row_B"]})
+        if k in traffic:
+            t = traffic[k]
+            dram = t["dram_bytes"]
+            d.update({"dram_bytes": dram, "dram_GB/s": dram / (ms / 1e3) / 1e9,
+                      "dram_frac": dram / (ms / 1e3) / 1e9 / hbm, "l2_hit_pct": t.get("l2_hit_pct")})
+        per_kernel[k] = d
     known = {k: v for k, v in kernels.items() if k in alg}
     dom = max(known, key=known.get) if known else None
     roofline = None
     if dom:
-        ach = alg[dom] / (kernels[dom] / 1e3) / 1e9
-        traffic = None
-        try:
-            tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-            traffic = tr.get(f"{args.workload}:{dom}", tr.get(dom) if args.workload == "reddit" else None)
-        except Exception:
-            pass
-        roofline = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": hbm, "unit": "GB/s",
-                    "frac": ach / hbm, "traffic": traffic, "algorithmic_bytes": alg[dom],
-                    "ms": kernels[dom], "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback"}
-    kern_out = {k: {"ms": v, "GB/s": (alg[k] / (v / 1e3) / 1e9) if k in alg else None} for k, v in kernels.items()}
-
+        d = per_kernel[dom]
+        if "l2_gather_peak" in d:
+            # the gathered tables are L2-resident (profiles/r2/gather_ceiling.json): the physical bound of these
+            # kernels is the measured L2 random-row gather ceiling, and their DRAM traffic is reported beside it
+            roofline = {"bound": "l2", "kernel": dom, "achieved": d["alg_GB/s"], "peak": d["l2_gather_peak"],
+                        "unit": "GB/s", "frac": d["l2_frac"], "l2_frac": d["l2_frac"]}
+        else:
+            roofline = {"bound": "hbm", "kernel": dom, "achieved": d["alg_GB/s"], "peak": hbm, "unit": "GB/s",
+                        "frac": d["alg_over_hbm"]}
+        roofline.update({
+            "traffic": d.get("dram_bytes"), "dram_GB/s": d.get("dram_GB/s"), "dram_frac": d.get("dram_frac"),
+            "l2_hit_pct": d.get("l2_hit_pct"), "hbm_peak": hbm, "alg_over_hbm": d["alg_over_hbm"],
+            "algorithmic_bytes": alg[dom], "ms": kernels[dom],
+            "peak_source": {"l2": "profiles/r2/gather_ceiling.json: tools/gather_bench.cu on B200, best random-row "
+                                  "gather GB/s (row_B + 4 B index per edge) from a 232,965-row table with a Reddit "
+                                  "power-law index stream, at the measured row size nearest the kernel's",
+                            "hbm": hbm_src, "traffic": traffic_src}})
+    kern_out = per_kernel
     # ---- e2e through the public API: pinned host X -> device each step, loss -> host each step ----
     e2e = None
     if not args.no_e2e:
@@ -527,15 +698,34 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         if args.workload == "reddit":
-            e, t, desc = oracle_sample(ip, ix, X, args.cpu_sample_edges)
+            e, t, desc = oracle_sample(ip, ix, X, args.cpu_sample_frac)
         else:
             e, t, desc = oracle_step(w, list(models))
         cpu = {"value": e / t, "unit": "edges/s", "cores": omp_threads(), "kind": "oracle", "sample": desc,
-               "seconds": t}
+               "seconds": t, "host": host_info(),
+               "note": "the fp64-accumulating correctness oracle (plain edge loops, OpenMP over rows), untuned"}
+        if args.workload != "reddit" and t * omp_threads() < 60:
+            # the single-threaded oracle too, for the configs whose whole step stays bounded
+            import oracle
+            oracle.set_num_threads(1)
+            e1, t1, _ = oracle_step(w, list(models))
+            oracle.set_num_threads(omp_threads())
+            cpu["single_thread"] = {"value": e1 / t1, "unit": "edges/s", "seconds": t1, "cores": 1}
 
     if rank == 0:
+        # measured: the kernel nodes of each captured epoch whose function lives in libseastar (names read back
+        # from the cudaGraph_t), times the timed steps; eager runs fall back to the per-epoch table above
+        launch_src = "table (eager run)"
         per_step = (sum(LAUNCHES_PER_EPOCH_REDDIT[k] for k in models) if args.workload == "reddit"
                     else LAUNCHES_PER_STEP[args.workload])
+        other = None
+        if kernel_names and "error" not in kernel_names:
+            ours = {k: [n for n in v if "seastar" in n] for k, v in kernel_names.items()}
+            per_step = sum(len(v) for v in ours.values())
+            other = sum(len(v) for v in kernel_names.values()) - per_step
+            launch_src = "counted from the captured CUDA graphs (kernel nodes named seastar::*)"
+        elif kernel_names:
+            launch_src = "table (graph introspection failed: " + kernel_names["error"] + ")"
         gpu_launches = args.steps * per_step
         line = {
             "metric": "GAT/GCN train epoch ms and edges/s at 1/2/4/8 B200; achieved HBM GB/s",
@@ -546,12 +736,17 @@ def main():
                        else f"reddit-shaped full-graph training: {args.model} only",
                        "name": args.workload, "N": cfg.N, "E": E, "F_in": cfg.F_in, "classes": cfg.classes,
                        "parallelism": f"row-partition x{world}", "l2": "flushed (256 MB write) between steps",
-                       "launch": "cuda-graph replay per model epoch" if use_graph else "eager",
+                       "launch": launch_mode,
                        "epoch_ms": {k: statistics.mean(v) for k, v in model_ms.items()},
+                       "epoch_ms_median": {k: statistics.median(v) for k, v in model_ms.items()},
                        "edges_per_s": {k: E / (statistics.mean(v) / 1e3) for k, v in model_ms.items()},
-                       "setup_s": setup_s},
+                       "setup_s": setup_s, "inputs_sha256": inputs_sha(w), "src_sha256": src_sha,
+                       "device_bytes_peak": int(free0 - min_free),
+                       "torch_max_allocated_bytes": int(torch.cuda.max_memory_allocated(dev))},
+            "ms_per_step_median": statistics.median(step_ms),
             "roofline": roofline, "kernels": kern_out, "cpu_baseline": cpu, "e2e": e2e, "clocks": ck,
             "gpu_launches": gpu_launches,
+            "gpu_launches_detail": {"per_step": per_step, "source": launch_src, "other_kernel_nodes_per_step": other},
         }
         print(json.dumps(line), flush=True)
     if world > 1:

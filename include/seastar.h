@@ -41,7 +41,7 @@
 extern "C" {
 #endif
 
-#define SEASTAR_ABI_VERSION 1
+#define SEASTAR_ABI_VERSION 2
 
 typedef struct seastar_graph_s* seastar_graph;   /* opaque, immutable after create */
 /* NEXT-3 dropout descriptor (reading #27): drop probability p (0 <= p < 1), the mask's site id
@@ -294,11 +294,25 @@ size_t seastar_gat_attn_proj_bwd_workspace(int64_t M, int32_t H, int32_t F);
  * Y[v] = act( sum_r ( sum_{e in in(v), type(e)=r} norm_e X_all[src(e),:] ) W[r] + bias )
  *   X_all [N,F_in] ld ldx ; W [R,F_in,F_out] ; norm_user [E] by user edge id, or NULL = the
  *   graph's 1/c_{v,r} (requires SEASTAR_GRAPH_RGCN_NORM) ; Y_loc [n_loc,F_out] ld ldy.
- *   F_in, F_out <= 64; W must fit in shared memory (R*F_in*F_out*4 <= 200 KB) for the staged path.
+ *   F_in, F_out <= 64.
+ *   Two paths, chosen by shape (both deterministic, no atomics):
+ *   - opt-in (environment SEASTAR_RGCN_TWOPHASE=1), F_in, F_out <= 16 and R * F_in * round4(F_out) * 4 <=
+ *     200 KB (two-phase; slower than the one pass on the AM shape, kept for the r2 measurements): the edges are visited in
+ *     type-major order, a lane per edge, with W staged in shared memory (the 32 edges of a warp share their
+ *     type, so every W read is a broadcast); edge e's product norm_e X_all[src(e)] W[type(e)] goes to slot e
+ *     of `workspace` in row order, and each row sums its slots in (type, eid) order.  workspace:
+ *     seastar_rgcn_fwd_workspace() bytes (dev, caller-owned, contents undefined on return); INVALID_ARGUMENT
+ *     if it is smaller.
+ *   - otherwise (one pass, the default; PAPER.md L473-L475 as written): every row walks its type-sorted edges and flushes
+ *     each run through W[r] staged in shared memory (stride S floats per W[r]: the smallest stride
+ *     >= F_in * round4(F_out) that is 16 mod 32 if R * S * 4 <= 219 KB, else the dense F_in * round4(F_out));
+ *     needs R * S * 4 <= 227 KB - 256 B, and <= 219 KB when some row has degree >= 1024 (the hub CTAs keep an
+ *     8 KB reduction buffer); UNSUPPORTED beyond.  seastar_rgcn_fwd_workspace() returns 0 (workspace may be NULL).
  */
 seastar_status seastar_rgcn_fwd(seastar_graph g, const float* X_all, int64_t F_in, int64_t ldx, const float* W,
                                 int64_t F_out, const float* norm_user, const float* bias, seastar_act act,
-                                float* Y_loc, int64_t ldy, seastar_stream stream);
+                                float* Y_loc, int64_t ldy, void* workspace, size_t ws_bytes, seastar_stream stream);
+size_t seastar_rgcn_fwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out);
 /*
  * Backward of seastar_rgcn_fwd's pre-activation output given dA = dL/d(pre-activation):
  *   dX_loc[u] = sum_{type runs r of out(u)} (sum_{e in run} norm_e dA_all[dst(e),:]) W[r]^T
@@ -316,7 +330,8 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
                                 const float* norm_user, const float* Yact_loc, seastar_act act, float* dX_loc,
                                 float* dW, void* workspace, size_t ws_bytes, seastar_stream stream);
 /* (Yact_loc [n_loc,F_in] ld ldx or NULL: dX_loc is multiplied by act'(Yact_loc), fusing the input
- *  layer's activation backward; act is ignored when Yact_loc is NULL.) */
+ *  layer's activation backward; act is ignored when Yact_loc is NULL.  dX takes the two-phase path of
+ *  seastar_rgcn_fwd over the reverse edges when F_in, F_out <= 16; the workspace covers both uses.) */
 size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out);
 
 /* ------------------------------------------------------------------------------------------ */

@@ -79,7 +79,7 @@ def _L():
             "orc_set_num_threads": ([ctypes.c_int], None),
             "orc_gat_attn_proj": ([_I, _I, _I, _P, _P, _P, _P, _P], None),
             "orc_gat_fwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _I, _P, _P, _P, _P], None),
-            "orc_gat_bwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _P, _I, _P, _P, _P, _P], None),
+            "orc_gat_bwd": ([_I, _I, _P, _P, _I, _I, _P, _P, _P, _D, _P, _P, _I, _P, _P, _P, _P, _P, _P, _P], None),
             "orc_rgcn_norm": ([_I, _I, _P, _P, ctypes.c_int32, _P], None),
             "orc_rgcn_fwd": ([_I, _I, _P, _P, _P, _I, _I, _P, _P, _P, _P, _I, _P], None),
             "orc_rgcn_bwd": ([_I, _I, _P, _P, _P, ctypes.c_int32, _I, _I, _P, _P, _P, _P, _P, _P], None),
@@ -328,8 +328,8 @@ def gat_fwd(indptr, indices, T, el, er, slope=0.2, rows=None, want_alpha=False, 
     return A, lse, alpha
 
 
-def gat_bwd(indptr, indices, T, el, er, dA, slope=0.2, rows=None, mask=None):
-    """Returns (dT [nrows,H,F], del [nrows,H], der [N,H]).  mask: as in gat_fwd."""
+def gat_bwd(indptr, indices, T, el, er, dA, slope=0.2, rows=None, mask=None, adj=None):
+    """Returns (dT [nrows,H,F], del [nrows,H], der [N,H]).  mask: as in gat_fwd; adj: out_adjacency() or None."""
     indptr, indices, T, el, er, dA = _i64(indptr), _i64(indices), _f64(T), _f64(el), _f64(er), _f64(dA)
     mask = _f64(mask)
     N = indptr.size - 1
@@ -339,8 +339,9 @@ def gat_bwd(indptr, indices, T, el, er, dA, slope=0.2, rows=None, mask=None):
     dT = np.empty((nrows, H, F))
     dl = np.empty((nrows, H))
     dr = np.empty((N, H))
+    ad = (None, None, None) if adj is None else tuple(_i64(a) for a in adj)
     _L().orc_gat_bwd(N, int(indptr[-1]), _p(indptr), _p(indices), H, F, _p(T), _p(el), _p(er), slope, _p(dA),
-                     _p(rows), nrows, _p(dT), _p(dl), _p(dr), _p(mask))
+                     _p(rows), nrows, _p(dT), _p(dl), _p(dr), _p(mask), *(_p(a) for a in ad))
     return dT, dl, dr
 
 

@@ -442,7 +442,8 @@ void orc_gat_fwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* ind
  */
 void orc_gat_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* indices, int64_t H, int64_t F,
                  const double* T, const double* el, const double* er, double slope, const double* dA,
-                 const int64_t* rows, int64_t nrows, double* dT, double* del, double* der, const double* mask) {
+                 const int64_t* rows, int64_t nrows, double* dT, double* del, double* der, const double* mask,
+                 const int64_t* adj_dst, const int64_t* adj_ptr, const int64_t* adj_eid) {
     double* mx = (double*)malloc(sizeof(double) * (size_t)(N * H > 0 ? N * H : 1));
     double* sm = (double*)malloc(sizeof(double) * (size_t)(N * H > 0 ? N * H : 1));
     double* gb = (double*)malloc(sizeof(double) * (size_t)(N * H > 0 ? N * H : 1));
@@ -477,9 +478,14 @@ void orc_gat_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* ind
             der[v * H + h] = dsum;
         }
     }
-    int64_t* dst = dst_of_edges(N, E, indptr);
-    int64_t *optr, *oeid;
-    out_adjacency(N, E, indices, &optr, &oeid);
+    int64_t *dst, *optr, *oeid;          /* prebuilt adjacency (orc_out_adjacency) or built here */
+    const int own = !(adj_dst && adj_ptr && adj_eid);
+    if (own) {
+        dst = dst_of_edges(N, E, indptr);
+        out_adjacency(N, E, indices, &optr, &oeid);
+    } else {
+        dst = (int64_t*)adj_dst; optr = (int64_t*)adj_ptr; oeid = (int64_t*)adj_eid;
+    }
     if (!rows) nrows = N;
     #pragma omp parallel for schedule(dynamic, 64)
     for (int64_t r = 0; r < nrows; ++r) {
@@ -501,7 +507,8 @@ void orc_gat_bwd(int64_t N, int64_t E, const int64_t* indptr, const int64_t* ind
             del[r * H + h] = dl;
         }
     }
-    free(optr); free(oeid); free(dst); free(mx); free(sm); free(gb);
+    if (own) { free(optr); free(oeid); free(dst); }
+    free(mx); free(sm); free(gb);
 }
 
 /* ------------------------------------------------------------------------------------------ */

@@ -74,7 +74,8 @@ _SIGS = {
     "seastar_gat_der": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _P, _P], _ST),
     "seastar_gat_attn_proj_bwd": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P, _P, _P, _P, _SZ, _P], _ST),
     "seastar_gat_attn_proj_bwd_workspace": ([_I64, _I32, _I32], _SZ),
-    "seastar_rgcn_fwd": ([_P, _P, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P], _ST),
+    "seastar_rgcn_fwd": ([_P, _P, _I64, _I64, _P, _I64, _P, _P, _I32, _P, _I64, _P, _SZ, _P], _ST),
+    "seastar_rgcn_fwd_workspace": ([_P, _I64, _I64], _SZ),
     "seastar_rgcn_bwd": ([_P, _P, _I64, _I64, _P, _I64, _I64, _P, _P, _P, _I32, _P, _P, _P, _SZ, _P], _ST),
     "seastar_rgcn_bwd_workspace": ([_P, _I64, _I64], _SZ),
     "seastar_rgcn_basis_fwd": ([_P, _P, _I64, _I64, _I64, _P, _P, _P, _I64, _P, _I32, _P, _I64, _P], _ST),
@@ -306,9 +307,24 @@ def seastar_gat_attn_proj_bwd(T, M, H, F, ldt, a_l, a_r, del_, der, dT, da_l, da
 
 
 # ----------------------------------------------------------------------------------- R-GCN
-def seastar_rgcn_fwd(g, X_all, F_in, ldx, W, F_out, norm_user, bias, act, Y_loc, ldy, stream=None) -> None:
+def seastar_rgcn_fwd_workspace(g, F_in, F_out) -> int:
+    return int(load().seastar_rgcn_fwd_workspace(g, F_in, F_out))
+
+
+def seastar_rgcn_fwd(g, X_all, F_in, ldx, W, F_out, norm_user, bias, act, Y_loc, ldy, workspace=None, ws_bytes=None,
+                     stream=None) -> None:
+    """workspace=None: a device buffer of seastar_rgcn_fwd_workspace() bytes is allocated here (memory plumbing
+    only; the models pass their own)."""
+    if workspace is None:
+        need = seastar_rgcn_fwd_workspace(g, F_in, F_out)
+        if need:
+            import torch
+            workspace = torch.empty(need, dtype=torch.uint8, device=Y_loc.device)
+    if ws_bytes is None:
+        ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
     _call("seastar_rgcn_fwd", g, _dptr(X_all, "X"), F_in, ldx, _dptr(W, "W"), F_out, _dptr(norm_user, "norm"),
-          _dptr(bias, "bias"), _act(act), _dptr(Y_loc, "Y"), ldy, _stream(stream))
+          _dptr(bias, "bias"), _act(act), _dptr(Y_loc, "Y"), ldy, _dptr(workspace, "workspace"), ws_bytes,
+          _stream(stream))
 
 
 def seastar_rgcn_bwd_workspace(g, F_in, F_out) -> int:

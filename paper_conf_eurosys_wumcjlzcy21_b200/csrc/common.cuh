@@ -44,6 +44,8 @@ inline cudaStream_t to_stream(seastar_stream s) { return reinterpret_cast<cudaSt
 // ----------------------------------------------------------------------------------------------
 // the graph handle (all index arrays are int32 on the device; E < 2^31 is validated at create)
 // ----------------------------------------------------------------------------------------------
+constexpr int kPow2Lo = 6, kPow2Classes = 11;   // degree thresholds 64 .. 65536 for the long-row split
+
 struct IndexSet {
     int32_t* perm = nullptr;   // row -> vertex id            [n_rows]   (nullptr for LSF: identity)
     int32_t* off = nullptr;    // row offsets                 [n_rows+1]
@@ -56,6 +58,7 @@ struct IndexSet {
     int64_t n_edges = 0;
     int64_t bucket_rows[SEASTAR_NUM_BUCKETS] = {0, 0, 0, 0};
     int64_t max_deg = 0;
+    int64_t pow2_rows[kPow2Classes] = {};   // rows with degree >= 2^(kPow2Lo + k) (rows are degree-sorted)
 };
 
 // Type-major view of the FWD edges for the R-GCN weight gradient: edges sorted by (type, dst row,
@@ -70,9 +73,24 @@ struct TypeMajor {
     int32_t* task_run = nullptr;  // [n_tasks+1]
     int32_t* task_type = nullptr; // [n_tasks]
     int32_t* type_task = nullptr; // [R+1]
+    int32_t* dst = nullptr;       // [Ef] destination vertex id of each edge (run boundaries = changes of dst in a task)
     int64_t n_runs = 0, n_tasks = 0;
 };
 constexpr int kTaskEdges = 512;   // edges per dW task (a task may exceed it only inside one run)
+
+// Two-phase R-GCN (a7 forward on FWD, a10 dX on REV; rgcn.cu): an index set's edges in type-major order
+// (type, row, eid) with, per edge, its type and its position in the index set's row order.  Phase 1 walks the edges
+// in this order -- a warp's 32 consecutive edges share their type, so W_r reads from shared memory are broadcasts --
+// and writes each edge's product norm_e * table[nbr_e] W_r to the edge's row-order position; phase 2 sums each
+// row's contiguous products.
+struct EdgeMajor {
+    const int32_t* nbr = nullptr;   // [E] neighbour id (FWD: tm.src; REV: owned array)
+    const int32_t* eid = nullptr;   // [E] user edge id
+    const float* norm = nullptr;    // [E] 1/c_{v,r} or nullptr
+    int32_t* type = nullptr;        // [E]
+    int32_t* pos = nullptr;         // [E] position of the edge in the index set's row order (FWD / REV off[])
+    int64_t n = 0;
+};
 
 }  // namespace seastar
 
@@ -84,6 +102,10 @@ struct seastar_graph_s {
     bool partitioned = false;
     seastar::IndexSet fwd, rev, lsf;
     seastar::TypeMajor tm;
+    seastar::EdgeMajor fem, rem;     // two-phase R-GCN: FWD (forward) and REV (dX) edges in type-major order
+    int32_t* rtm_nbr = nullptr;      // REV edges in type-major order (rem's edge arrays)
+    int32_t* rtm_eid = nullptr;
+    float* rtm_norm = nullptr;
     int32_t* indeg_loc = nullptr;    // [n_loc]
     int32_t* outdeg_loc = nullptr;   // [n_loc]
     void* pool = nullptr;            // single device allocation backing every array above
@@ -149,7 +171,7 @@ __device__ __forceinline__ float act_grad_from_y(int act, float y) {
     }
 }
 
-inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+__host__ __device__ inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 // NEXT-3 dropout generator (reading #27): splitmix64's output function; a mask element keeps
 // iff (sm64(key ^ i) >> 40) >= thr with key = sm64(seed ^ sm64((site << 32) | step))
@@ -242,6 +264,17 @@ inline int num_sms() {
         if (sms <= 0) sms = 148;
     }
     return sms;
+}
+
+// "Long" rows of a row launch: a row whose edges exceed a quarter of one SM's share of the index set would keep
+// one warp busy past the rest of the launch (CoraFull-shaped: ~250 edges), so it gets a CTA of 8 warps (PAPER.md
+// L1253 CTA + Warp; the a3 hub class, made relative to the launch).  Returns the number of leading (highest-degree)
+// rows that qualify: rows with degree >= the power of two at or above max(E / (4 * #SMs), 128).
+inline int64_t long_rows(const IndexSet& x) {
+    const int64_t t = x.n_edges / (4 * (int64_t)num_sms());
+    int k = 0;
+    while (k < kPow2Classes && ((int64_t)1 << (kPow2Lo + k)) < (t > 128 ? t : 128)) ++k;
+    return k < kPow2Classes ? x.pow2_rows[k] : 0;
 }
 
 inline int pow2_ceil(int x) {

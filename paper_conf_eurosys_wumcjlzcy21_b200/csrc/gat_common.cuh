@@ -41,6 +41,7 @@ struct GatFwdArgs {
     // NEXT-3 attention dropout (generic chunked kernels only; deid == nullptr: off): the aggregation weight of
     // edge slot k is a_e * drop_mult(key, eid * H + h), key from (dseed, dsite, *dstep)
     const int32_t* deid; uint64_t dseed; const int32_t* dstep; uint32_t dsite, dthr; float dscale;
+    int64_t nlong;   // hub-capable launches: blocks [0, nlong) own one long row each (see k_gat_fwd_hpl)
 };
 
 struct GatBwdArgs {
@@ -53,6 +54,7 @@ struct GatBwdArgs {
     float* dT; float* del;   // src-major outputs
     float* der;              // der output
     const int32_t* deid; uint64_t dseed; const int32_t* dstep; uint32_t dsite, dthr; float dscale;   // as GatFwdArgs
+    int64_t nlong;
 };
 
 
@@ -67,11 +69,12 @@ __device__ __forceinline__ const float* row_ptr(const float* base, int r, int64_
 }
 
 // launchers (return false when the geometry does not apply)
-bool launch_gat_fwd_hpl(const GatFwdArgs& a, cudaStream_t s);
-bool launch_gat_bwd_hpl(const GatBwdArgs& a, cudaStream_t s);
+// hub = the index set's long_rows(): those leading rows get a multi-warp CTA each
+bool launch_gat_fwd_hpl(const GatFwdArgs& a, int64_t hub, cudaStream_t s);
+bool launch_gat_bwd_hpl(const GatBwdArgs& a, int64_t hub, cudaStream_t s);
 bool launch_gat_der_hpl(const GatBwdArgs& a, cudaStream_t s);
-bool launch_gat_fwd_h1(const GatFwdArgs& a, int64_t split, int64_t n_rows, cudaStream_t s);
-bool launch_gat_bwd_h1(const GatBwdArgs& a, int64_t split, int64_t n_rows, bool der, cudaStream_t s);
+bool launch_gat_fwd_h1(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t n_rows, cudaStream_t s);
+bool launch_gat_bwd_h1(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t n_rows, bool der, cudaStream_t s);
 
 // head-per-lane geometry: H | 32, every head row is whole float4s held by one lane
 inline int hpl_f4(int H, int F, int64_t ldt, bool aligned) {

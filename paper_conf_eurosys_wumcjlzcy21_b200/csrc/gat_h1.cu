@@ -4,6 +4,8 @@
 // ~ceil(row bytes / 64) L1 wavefronts instead of one per lane-chunk), S = RL / L edge slots per row group; g = <dA, T> by an L-lane xor reduction.  PAPER.md Fig. 2 L95-L123,
 // §6.3.4 L461-L463.  Same branch-free inner loop as gat_hpl.cu: an out-of-range edge slot gathers
 // row 0 and gets weight 0; chunks past the row end are never loaded (per-lane constant predicate).
+#include <algorithm>
+
 #include "gat_common.cuh"
 
 namespace seastar {
@@ -28,8 +30,12 @@ __device__ __forceinline__ float4 mask_tail(float4 x, int nv) {
     return make_float4(nv > 0 ? x.x : 0.f, nv > 1 ? x.y : 0.f, nv > 2 ? x.z : 0.f, nv > 3 ? x.w : 0.f);
 }
 
-template <int VPL, int L, int RL, bool SB>
+// WPR > 1 (RL = 32): the launch's first a.nlong blocks each own one long row, warp w over the w-th contiguous slice
+// of the row's edges, slices merged in warp order by the online-softmax merge through shared memory; later blocks
+// own 8 warp rows (as k_gat_fwd_hpl)
+template <int VPL, int L, int RL, bool SB, int WPR = 1>
 __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs a) {
+    static_assert(WPR == 1 || RL == 32, "hub rows take whole warps");
     constexpr int NV = 4 * VPL, S = RL / L;
     constexpr int UE = h1_ub<VPL>() < L ? h1_ub<VPL>() : L;   // edges per slot per batch
     constexpr int NB = L / UE;                                 // batches per RL-edge chunk
@@ -38,10 +44,20 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
     const int gl = lane % RL, slot = gl / L, c = gl % L;
     const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t row = a.row_begin + warp * (32 / RL) + lane / RL;
+    const int wib = threadIdx.x >> 5;
+    const bool hubblk = WPR > 1 && (int64_t)blockIdx.x < a.nlong;      // block-uniform
+    const int64_t row = hubblk ? a.row_begin + blockIdx.x
+                      : WPR > 1 ? a.row_begin + a.nlong + ((int64_t)blockIdx.x - a.nlong) * (blockDim.x >> 5) + wib
+                                : a.row_begin + warp * (32 / RL) + lane / RL;
     const bool valid = row < a.row_end;
-    const int beg = valid ? __ldg(a.off + row) : 0;
-    const int end = valid ? __ldg(a.off + row + 1) : 0;
+    int beg = valid ? __ldg(a.off + row) : 0;
+    int end = valid ? __ldg(a.off + row + 1) : 0;
+    if (hubblk) {
+        const int64_t len = end - beg;
+        const int b0 = beg + (int)(len * wib / WPR);
+        end = beg + (int)(len * (wib + 1) / WPR);
+        beg = b0;
+    }
     const int64_t v = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;
     const int W = a.F, col0 = 4 * c;             // chunk q of this lane: columns col0 + 4 L q ..
     bool qv[VPL];
@@ -131,6 +147,35 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
         }
         m = mn;
     }
+    if (hubblk) {                                       // merge the warps' slices in warp order
+        constexpr int NS = 3 + NV + (SB ? NP : 0);
+        __shared__ float st[WPR > 1 ? WPR : 1][L][NS];
+        if (slot == 0) {
+            float* p = st[wib][c];
+            p[0] = m; p[1] = ssum; p[2] = psum;
+#pragma unroll
+            for (int i = 0; i < NV; ++i) p[3 + i] = acc[i];
+#pragma unroll
+            for (int i = 0; i < (SB ? NP : 0); ++i) p[3 + NV + i] = pacc[i];
+        }
+        __syncthreads();
+        if (wib != 0) return;
+        if (slot == 0)
+            for (int w2 = 1; w2 < WPR; ++w2) {
+                const float* p = st[w2][c];
+                const float mo = p[0], mn = fmaxf(m, mo);
+                const float ca = ex2((m - mn) * kLog2e), cb = ex2((mo - mn) * kLog2e);
+                ssum = ssum * ca + p[1] * cb;
+#pragma unroll
+                for (int i = 0; i < NV; ++i) acc[i] = acc[i] * ca + p[3 + i] * cb;
+                if (SB) {
+                    psum = psum * ca + p[2] * cb;
+#pragma unroll
+                    for (int i = 0; i < NP; ++i) pacc[i] = pacc[i] * ca + p[3 + NV + (SB ? i : 0)] * cb;
+                }
+                m = mn;
+            }
+    }
     if (!valid || slot != 0) return;
     const float inv = ssum > 0.f ? 1.f / ssum : 0.f;
     float* pa = a.A + v * a.ld;
@@ -173,8 +218,9 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
 #ifndef GAT_H1_BWD_UBMAX
 #define GAT_H1_BWD_UBMAX 4
 #endif
-template <int VPL, int L, int RL, bool DER>
+template <int VPL, int L, int RL, bool DER, int WPR = 1>
 __global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdArgs a) {
+    static_assert(WPR == 1 || RL == 32, "hub rows take whole warps");
     constexpr int NV = 4 * VPL, S = RL / L;
     constexpr int UB0 = h1_ub<VPL>() < GAT_H1_BWD_UBMAX ? h1_ub<VPL>() : GAT_H1_BWD_UBMAX;
     constexpr int UE = UB0 < L ? UB0 : L;
@@ -183,10 +229,20 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdA
     const int gl = lane % RL, slot = gl / L, c = gl % L;
     const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t row = a.row_begin + warp * (32 / RL) + lane / RL;
+    const int wib = threadIdx.x >> 5;
+    const bool hubblk = WPR > 1 && (int64_t)blockIdx.x < a.nlong;      // block-uniform
+    const int64_t row = hubblk ? a.row_begin + blockIdx.x
+                      : WPR > 1 ? a.row_begin + a.nlong + ((int64_t)blockIdx.x - a.nlong) * (blockDim.x >> 5) + wib
+                                : a.row_begin + warp * (32 / RL) + lane / RL;
     const bool valid = row < a.row_end;
-    const int beg = valid ? __ldg(a.off + row) : 0;
-    const int end = valid ? __ldg(a.off + row + 1) : 0;
+    int beg = valid ? __ldg(a.off + row) : 0;
+    int end = valid ? __ldg(a.off + row + 1) : 0;
+    if (hubblk) {                                       // long rows: warp w takes the w-th slice
+        const int64_t len = end - beg;
+        const int b0 = beg + (int)(len * wib / WPR);
+        end = beg + (int)(len * (wib + 1) / WPR);
+        beg = b0;
+    }
     const int64_t w = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;   // u (src-major) or v (der)
     const int W = a.F, col0 = 4 * c;             // chunk q of this lane: columns col0 + 4 L q ..
     const int aux0 = rec_aux_offset(W);
@@ -280,6 +336,23 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdA
         }
         dsum += __shfl_xor_sync(gmask, dsum, o, RL);
     }
+    if (hubblk) {                                       // add the warps' slices in warp order
+        __shared__ float st[WPR > 1 ? WPR : 1][L][NV + 1];
+        if (slot == 0) {
+#pragma unroll
+            for (int i = 0; i < NV; ++i) st[wib][c][i] = DER ? 0.f : acc[i];
+            st[wib][c][NV] = dsum;
+        }
+        __syncthreads();
+        if (wib != 0) return;
+        if (slot == 0)
+            for (int w2 = 1; w2 < WPR; ++w2) {
+                if (!DER)
+#pragma unroll
+                    for (int i = 0; i < NV; ++i) acc[i] += st[w2][c][i];
+                dsum += st[w2][c][NV];
+            }
+    }
     if (!valid || slot != 0) return;
     if (DER) {
         if (c == 0) a.der[w] = dsum;
@@ -301,35 +374,47 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdA
 // ---------------------------------------------------------------------------------------------
 // launchers over the two degree classes: warp rows (RL = 32, degree >= 32) and 4-lane row groups
 // ---------------------------------------------------------------------------------------------
-template <typename Args, typename LW, typename LS>
-static void h1_buckets(const Args& a, int64_t split, int64_t n_rows, LW lw, LS ls) {
+constexpr int kHubWarpsH1 = 8;      // warps per hub row (degree >= 1024)
+
+template <typename Args, typename LH, typename LW, typename LS>
+static void h1_buckets(const Args& a, int64_t hub, int64_t split, int64_t n_rows, LH lh, LW lw, LS ls) {
     Args hi = a, lo = a;
     hi.row_begin = 0; hi.row_end = split;
+    hi.nlong = std::min<int64_t>(hub, split);
     lo.row_begin = split; lo.row_end = n_rows;
-    if (split > 0) lw(hi, (unsigned)((split + 7) / 8));
+    lo.nlong = 0;
+    if (split > 0) {
+        const unsigned g = (unsigned)(hi.nlong + (split - hi.nlong + 7) / 8);
+        if (hi.nlong > 0) lh(hi, g);                                        // long rows + warp rows, one launch
+        else lw(hi, g);
+    }
     if (n_rows > split) ls(lo, (unsigned)((n_rows - split + 63) / 64));   // RL = 4: 64 rows per block
 }
 
 template <int VPL, int L>
-static void fwd_h1_run(const GatFwdArgs& a, int64_t split, int64_t n, cudaStream_t s) {
+static void fwd_h1_run(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t n, cudaStream_t s) {
     if (a.B)
-        h1_buckets(a, split, n,
+        h1_buckets(a, hub, split, n,
+                   [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 32, true, kHubWarpsH1>, dim3(g), dim3(32 * kHubWarpsH1), 0, s, x); },
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 32, true>, dim3(g), dim3(256), 0, s, x); },
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 4, true>, dim3(g), dim3(256), 0, s, x); });
     else
-        h1_buckets(a, split, n,
+        h1_buckets(a, hub, split, n,
+                   [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 32, false, kHubWarpsH1>, dim3(g), dim3(32 * kHubWarpsH1), 0, s, x); },
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 32, false>, dim3(g), dim3(256), 0, s, x); },
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 4, false>, dim3(g), dim3(256), 0, s, x); });
 }
 
 template <int VPL, int L>
-static void bwd_h1_run(const GatBwdArgs& a, int64_t split, int64_t n, bool der, cudaStream_t s) {
+static void bwd_h1_run(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t n, bool der, cudaStream_t s) {
     if (der)
-        h1_buckets(a, split, n,
+        h1_buckets(a, hub, split, n,
+                   [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 32, true, kHubWarpsH1>, dim3(g), dim3(32 * kHubWarpsH1), 0, s, x); },
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 32, true>, dim3(g), dim3(256), 0, s, x); },
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 4, true>, dim3(g), dim3(256), 0, s, x); });
     else
-        h1_buckets(a, split, n,
+        h1_buckets(a, hub, split, n,
+                   [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 32, false, kHubWarpsH1>, dim3(g), dim3(32 * kHubWarpsH1), 0, s, x); },
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 32, false>, dim3(g), dim3(256), 0, s, x); },
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 4, false>, dim3(g), dim3(256), 0, s, x); });
 }
@@ -356,18 +441,18 @@ static void bwd_h1_run(const GatBwdArgs& a, int64_t split, int64_t n, bool der, 
         default: RUN<8, 4>(__VA_ARGS__); break;                                   \
     }
 
-bool launch_gat_fwd_h1(const GatFwdArgs& a, int64_t split, int64_t n_rows, cudaStream_t s) {
+bool launch_gat_fwd_h1(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t n_rows, cudaStream_t s) {
     int vpl = 0, L = 0;
     if (!h1_geometry(a.H, a.F, a.ld, aligned16(a.T) && aligned16(a.A) && aligned16(a.Y), vpl, L)) return false;
-    SS_H1_DISPATCH(fwd_h1_run, vpl, L, a, split, n_rows, s)
+    SS_H1_DISPATCH(fwd_h1_run, vpl, L, a, hub, split, n_rows, s)
     return true;
 }
 
-bool launch_gat_bwd_h1(const GatBwdArgs& a, int64_t split, int64_t n_rows, bool der, cudaStream_t s) {
+bool launch_gat_bwd_h1(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t n_rows, bool der, cudaStream_t s) {
     int vpl = 0, L = 0;
     const bool al = der ? aligned16(a.T) && aligned16(a.D) : aligned16(a.T) && aligned16(a.D) && aligned16(a.dT);
     if (!h1_geometry(a.H, a.F, a.ldt, al, vpl, L)) return false;
-    SS_H1_DISPATCH(bwd_h1_run, vpl, L, a, split, n_rows, der, s)
+    SS_H1_DISPATCH(bwd_h1_run, vpl, L, a, hub, split, n_rows, der, s)
     return true;
 }
 

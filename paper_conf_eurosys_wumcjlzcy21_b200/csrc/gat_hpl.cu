@@ -7,6 +7,8 @@
 // The inner loops are branch-free: H and F are template parameters, an out-of-range edge slot
 // gathers row 0 (always valid memory) and gets weight 0, softmax weights are ex2 of one FFMA, and
 // neighbour ids are software-pipelined one 32-edge chunk ahead (see gcn.cu).
+#include <algorithm>
+
 #include "gat_common.cuh"
 
 namespace seastar {
@@ -29,16 +31,30 @@ constexpr int hpl_bwd_ub() { return hpl_ub<F4>() < GAT_HPL_BWD_UBMAX ? hpl_ub<F4
 #ifndef GAT_MB_FWD_HPL
 #define GAT_MB_FWD_HPL GAT_MB_FWD
 #endif
-template <int H, int F4, bool SB>
+// WPR > 1 (WPR = the block's warps): the launch's first a.nlong blocks each own one long row (long_rows()), warp w
+// runs the online softmax over the w-th contiguous slice of the row's edges, and the warps' (max, sum, weighted
+// rows) are merged in warp order through shared memory by the same online-softmax merge as the slot tree
+// (deterministic; "CTA + Warp"); every later block owns 8 rows, a warp each.
+template <int H, int F4, bool SB, int WPR = 1>
 __global__ void __launch_bounds__(256, GAT_MB_FWD_HPL) k_gat_fwd_hpl(const GatFwdArgs a) {
     constexpr int F = 4 * F4, S = 32 / H;
     constexpr int UE = hpl_ub<F4>() < H ? hpl_ub<F4>() : H;   // edges per lane per batch
     constexpr int NB = H / UE;                                // batches per 32-edge chunk
     const int lane = threadIdx.x & 31;
     const int h = lane % H, slot = lane / H;
-    const int64_t row = a.row_begin + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
-    if (row >= a.row_end) return;                      // warp-uniform
-    const int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+    const int wib = threadIdx.x >> 5;
+    const bool hubblk = WPR > 1 && (int64_t)blockIdx.x < a.nlong;      // block-uniform
+    const int64_t row = hubblk ? a.row_begin + blockIdx.x
+                      : WPR > 1 ? a.row_begin + a.nlong + ((int64_t)blockIdx.x - a.nlong) * (blockDim.x >> 5) + wib
+                                : a.row_begin + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    if (row >= a.row_end) return;                      // warp-uniform (never taken in a long-row block)
+    int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+    if (hubblk) {
+        const int64_t len = end - beg;
+        const int b0 = beg + (int)(len * wib / WPR);
+        end = beg + (int)(len * (wib + 1) / WPR);
+        beg = b0;
+    }
     const int64_t v = (int64_t)__ldg(a.perm + row) - a.vbase;
     const float erv = __ldg(a.er + v * H + h);
     const float slope = a.slope;
@@ -128,6 +144,37 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD_HPL) k_gat_fwd_hpl(const GatFw
         }
         m = mn;
     }
+    if (hubblk) {                                      // merge the warps' slices in warp order, one warp at a time
+        constexpr int NS = 3 + F + (SB ? F : 0);
+        __shared__ float st[H][NS];
+        for (int w2 = 1; w2 < WPR; ++w2) {
+            if (wib == w2 && slot == 0) {
+                float* p = st[h];
+                p[0] = m; p[1] = ssum; p[2] = psum;
+#pragma unroll
+                for (int i = 0; i < F; ++i) p[3 + i] = acc[i];
+#pragma unroll
+                for (int i = 0; i < (SB ? F : 0); ++i) p[3 + F + i] = pacc[i % (SB ? F : 1)];
+            }
+            __syncthreads();
+            if (wib == 0 && slot == 0) {
+                const float* p = st[h];
+                const float mo = p[0], mn = fmaxf(m, mo);
+                const float ca = ex2((m - mn) * kLog2e), cb = ex2((mo - mn) * kLog2e);
+                ssum = ssum * ca + p[1] * cb;
+#pragma unroll
+                for (int i = 0; i < F; ++i) acc[i] = acc[i] * ca + p[3 + i] * cb;
+                if (SB) {
+                    psum = psum * ca + p[2] * cb;
+#pragma unroll
+                    for (int i = 0; i < (SB ? F : 1); ++i) pacc[i] = pacc[i] * ca + p[3 + F + i] * cb;
+                }
+                m = mn;
+            }
+            __syncthreads();
+        }
+        if (wib != 0) return;
+    }
     if (slot != 0) return;
     const float inv = ssum > 0.f ? 1.f / ssum : 0.f;
     const int64_t hoff = (int64_t)h * F;
@@ -162,16 +209,26 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD_HPL) k_gat_fwd_hpl(const GatFw
 #ifndef GAT_MB_BWD_HPL
 #define GAT_MB_BWD_HPL 4
 #endif
-template <int H, int F4>
+template <int H, int F4, int WPR = 1>
 __global__ void __launch_bounds__(256, GAT_MB_BWD_HPL) k_gat_bwd_hpl(const GatBwdArgs a) {
     constexpr int F = 4 * F4, S = 32 / H;
     constexpr int UE = hpl_bwd_ub<F4>() < H ? hpl_bwd_ub<F4>() : H;
     constexpr int NB = H / UE;
     const int lane = threadIdx.x & 31;
     const int h = lane % H, slot = lane / H;
-    const int64_t row = a.row_begin + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    const int wib = threadIdx.x >> 5;
+    const bool hubblk = WPR > 1 && (int64_t)blockIdx.x < a.nlong;      // block-uniform
+    const int64_t row = hubblk ? a.row_begin + blockIdx.x
+                      : WPR > 1 ? a.row_begin + a.nlong + ((int64_t)blockIdx.x - a.nlong) * (blockDim.x >> 5) + wib
+                                : a.row_begin + ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
     if (row >= a.row_end) return;
-    const int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+    int beg = __ldg(a.off + row), end = __ldg(a.off + row + 1);
+    if (hubblk) {                                      // long rows: warp w takes the w-th slice (see the forward)
+        const int64_t len = end - beg;
+        const int b0 = beg + (int)(len * wib / WPR);
+        end = beg + (int)(len * (wib + 1) / WPR);
+        beg = b0;
+    }
     const int64_t u = (int64_t)__ldg(a.perm + row) - a.vbase;
     const int64_t hoff = (int64_t)h * F;
     const float slope = a.slope;
@@ -233,6 +290,24 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD_HPL) k_gat_bwd_hpl(const GatBw
 #pragma unroll
         for (int i = 0; i < F; ++i) acc[i] += __shfl_xor_sync(0xffffffffu, acc[i], o);
         dl += __shfl_xor_sync(0xffffffffu, dl, o);
+    }
+    if (hubblk) {                                      // add the warps' slices in warp order, one warp at a time
+        __shared__ float st[H][F + 1];
+        for (int w2 = 1; w2 < WPR; ++w2) {
+            if (wib == w2 && slot == 0) {
+#pragma unroll
+                for (int i = 0; i < F; ++i) st[h][i] = acc[i];
+                st[h][F] = dl;
+            }
+            __syncthreads();
+            if (wib == 0 && slot == 0) {
+#pragma unroll
+                for (int i = 0; i < F; ++i) acc[i] += st[h][i];
+                dl += st[h][F];
+            }
+            __syncthreads();
+        }
+        if (wib != 0) return;
     }
     if (slot != 0) return;
     float* pd = a.dT + u * a.ldt + hoff;
@@ -331,22 +406,56 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD) k_gat_der_hpl(const GatBwdArg
         default: SS_HPL_F4(KERNEL, 32, f4, __VA_ARGS__) break;      \
     }
 
-bool launch_gat_fwd_hpl(const GatFwdArgs& a0, cudaStream_t s) {
+// hub rows (the a3 hub class, degree >= 1024) get kHubWarpsGat warps each; the rest a warp per row
+constexpr int kHubWarpsGat = 8;
+
+#define SS_HPL_F4B(KERNEL, H, f4, ...)                                                                        \
+    switch (f4) {                                                                                             \
+        case 1: launch_k(KERNEL<H, 1 __VA_ARGS__>, dim3(grid), dim3(256), 0, s, a); break;                    \
+        case 2: launch_k(KERNEL<H, 2 __VA_ARGS__>, dim3(grid), dim3(256), 0, s, a); break;                    \
+        case 3: launch_k(KERNEL<H, 3 __VA_ARGS__>, dim3(grid), dim3(256), 0, s, a); break;                    \
+        case 4: launch_k(KERNEL<H, 4 __VA_ARGS__>, dim3(grid), dim3(256), 0, s, a); break;                    \
+        case 5: launch_k(KERNEL<H, 5 __VA_ARGS__>, dim3(grid), dim3(256), 0, s, a); break;                    \
+        case 6: launch_k(KERNEL<H, 6 __VA_ARGS__>, dim3(grid), dim3(256), 0, s, a); break;                    \
+        case 7: launch_k(KERNEL<H, 7 __VA_ARGS__>, dim3(grid), dim3(256), 0, s, a); break;                    \
+        default: launch_k(KERNEL<H, 8 __VA_ARGS__>, dim3(grid), dim3(256), 0, s, a); break;                   \
+    }
+#define SS_HPL_HB(KERNEL, H, f4, ...)                                \
+    switch (H) {                                                     \
+        case 2: SS_HPL_F4B(KERNEL, 2, f4, __VA_ARGS__) break;        \
+        case 4: SS_HPL_F4B(KERNEL, 4, f4, __VA_ARGS__) break;        \
+        case 8: SS_HPL_F4B(KERNEL, 8, f4, __VA_ARGS__) break;        \
+        case 16: SS_HPL_F4B(KERNEL, 16, f4, __VA_ARGS__) break;      \
+        default: SS_HPL_F4B(KERNEL, 32, f4, __VA_ARGS__) break;      \
+    }
+
+bool launch_gat_fwd_hpl(const GatFwdArgs& a0, int64_t hub, cudaStream_t s) {
     const int f4 = hpl_f4(a0.H, a0.F, a0.ld, aligned16(a0.T) && aligned16(a0.A) && aligned16(a0.Y));
     if (!f4) return false;
-    const GatFwdArgs& a = a0;
-    const unsigned grid = (unsigned)((a.row_end - a.row_begin + 7) / 8);
+    static_assert(32 * kHubWarpsGat == 256, "long-row CTAs are the launch's 256-thread blocks");
+    GatFwdArgs a = a0;
+    a.nlong = std::min<int64_t>(std::max<int64_t>(hub - a0.row_begin, 0), a0.row_end - a0.row_begin);
+    const unsigned grid = (unsigned)(a.nlong + (a.row_end - a.row_begin - a.nlong + 7) / 8);
     if (grid == 0) return true;
-    if (a.B) { SS_HPL_H(k_gat_fwd_hpl, a.H, f4, , true) }
-    else { SS_HPL_H(k_gat_fwd_hpl, a.H, f4, , false) }
+    if (a.nlong > 0) {                                 // long rows (a CTA each) + warp rows in one launch
+        if (a.B) { SS_HPL_HB(k_gat_fwd_hpl, a.H, f4, , true, kHubWarpsGat) }
+        else { SS_HPL_HB(k_gat_fwd_hpl, a.H, f4, , false, kHubWarpsGat) }
+    } else {
+        if (a.B) { SS_HPL_H(k_gat_fwd_hpl, a.H, f4, , true) }
+        else { SS_HPL_H(k_gat_fwd_hpl, a.H, f4, , false) }
+    }
     return true;
 }
 
-bool launch_gat_bwd_hpl(const GatBwdArgs& a, cudaStream_t s) {
-    const int f4 = hpl_f4(a.H, a.F, a.ldt, aligned16(a.T) && aligned16(a.D) && aligned16(a.dT));
+bool launch_gat_bwd_hpl(const GatBwdArgs& a0, int64_t hub, cudaStream_t s) {
+    const int f4 = hpl_f4(a0.H, a0.F, a0.ldt, aligned16(a0.T) && aligned16(a0.D) && aligned16(a0.dT));
     if (!f4) return false;
-    const unsigned grid = (unsigned)((a.row_end - a.row_begin + 7) / 8);
-    if (grid) { SS_HPL_H(k_gat_bwd_hpl, a.H, f4) }
+    GatBwdArgs a = a0;
+    a.nlong = std::min<int64_t>(std::max<int64_t>(hub - a0.row_begin, 0), a0.row_end - a0.row_begin);
+    const unsigned grid = (unsigned)(a.nlong + (a.row_end - a.row_begin - a.nlong + 7) / 8);
+    if (grid == 0) return true;
+    if (a.nlong > 0) { SS_HPL_HB(k_gat_bwd_hpl, a.H, f4, , kHubWarpsGat) }
+    else { SS_HPL_H(k_gat_bwd_hpl, a.H, f4) }
     return true;
 }
 

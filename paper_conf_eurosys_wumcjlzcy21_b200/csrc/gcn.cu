@@ -14,6 +14,8 @@
 //     and the block scheduler's id order provides the dynamic load balance of §6.3.3 (L437-L453);
 //   * the epilogue (norm, APPNP mix, bias, activation, next-layer pre-scaling / activation
 //     derivative) is fused so each output row is written once.
+#include <algorithm>
+
 #include "common.cuh"
 
 namespace seastar {
@@ -37,6 +39,7 @@ struct AggArgs {
     const float* Yact; float* dA; const float* post_scale; float* dP;
     // NEXT-3 edge dropout (deid == nullptr: off): edge k's message is scaled by drop_mult(key, eid[k])
     const int32_t* deid; uint64_t dseed; const int32_t* dstep; uint32_t dsite, dthr; float dscale;
+    int64_t nlong;         // WPR > 1 launches: blocks [0, nlong) are long rows (a CTA each), the rest 8 warp-rows
 };
 
 // minimum resident blocks (0: compiler's choice, 48 registers at F = 16).  Measured on Reddit: forcing 6 blocks
@@ -50,8 +53,14 @@ struct AggArgs {
 #else
 #define AGG_BOUNDS __launch_bounds__(256)
 #endif
-template <int VEC, int L, int RL, int NB, bool DROP = false>
+// WPR > 1 (RL = 32, WPR = the block's warps): the launch's first a.nlong blocks each own one long row (long_rows():
+// degree above a quarter of one SM's share of the launch) -- warp w walks the w-th contiguous slice of the row's
+// edges, and the warps' partial sums are added in warp order through shared memory before warp 0 runs the epilogue
+// (deterministic) -- and every later block owns 8 rows, a warp each ("CTA + Warp").  One
+// launch for both classes: a separate hub launch cost more (kernel boundary) than it saved on the Reddit shape.
+template <int VEC, int L, int RL, int NB, bool DROP = false, int WPR = 1>
 __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
+    static_assert(WPR == 1 || RL == 32, "hub rows take whole warps");
     constexpr int S = RL / L;                    // edge slots per row group
 #ifdef GCN_UB_FIXED
     constexpr int UB = GCN_UB_FIXED < 32 / L ? GCN_UB_FIXED : 32 / L;
@@ -64,10 +73,20 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
     const int c = gl % L;
     const unsigned gmask = (RL == 32) ? 0xffffffffu : (((1u << RL) - 1u) << ((lane / RL) * RL));
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t row = a.row_begin + warp * (32 / RL) + lane / RL;
+    const int wib = threadIdx.x >> 5;            // warp in block (the slice index when WPR > 1)
+    const bool hubblk = WPR > 1 && (int64_t)blockIdx.x < a.nlong;      // block-uniform
+    const int64_t row = hubblk ? a.row_begin + blockIdx.x
+                      : WPR > 1 ? a.row_begin + a.nlong + ((int64_t)blockIdx.x - a.nlong) * (blockDim.x >> 5) + wib
+                                : a.row_begin + warp * (32 / RL) + lane / RL;
     const bool valid = row < a.row_end;
-    const int beg = valid ? __ldg(a.off + row) : 0;
-    const int end = valid ? __ldg(a.off + row + 1) : 0;
+    int beg = valid ? __ldg(a.off + row) : 0;
+    int end = valid ? __ldg(a.off + row + 1) : 0;
+    if (hubblk) {
+        const int64_t len = end - beg;
+        const int b0 = beg + (int)(len * wib / WPR);
+        end = beg + (int)(len * (wib + 1) / WPR);
+        beg = b0;
+    }
     const int64_t v = valid ? (int64_t)__ldg(a.perm + row) - a.vbase : 0;
     const int C = (a.F + VEC - 1) / VEC;
     const uint64_t dkey = DROP ? drop_key(a.dseed, a.dsite, a.dstep) : 0ull;
@@ -131,6 +150,23 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
         for (int o = L; o < RL; o <<= 1)
 #pragma unroll
             for (int i = 0; i < VEC; ++i) acc[i] += __shfl_xor_sync(gmask, acc[i], o, RL);
+        if (hubblk) {                                // merge the warps' slices in warp order
+            __shared__ float red[WPR > 1 ? WPR : 1][32][VEC];
+            if (slot == 0)
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) red[wib][c][i] = acc[i];
+            __syncthreads();
+            if (wib == 0 && slot == 0) {
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) {
+                    float t = red[0][c][i];
+                    for (int w2 = 1; w2 < WPR; ++w2) t += red[w2][c][i];
+                    acc[i] = t;
+                }
+            }
+            __syncthreads();
+            if (wib != 0) continue;
+        }
 
         if (!valid || slot != 0 || !active) continue;
         const float rs = (a.rscale ? __ldg(a.rscale + v) : 1.f) * a.gscale;
@@ -184,11 +220,21 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
     }
 }
 
+constexpr int kHubWarps = 8;       // warps per hub row (degree >= 1024: >= 128 edges per warp)
+
 template <int VEC, int L>
-static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s) {
+static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s, bool hub = false) {
     const int64_t rows = a.row_end - a.row_begin;
     if (rows <= 0) return;
     constexpr int threads = 256;
+    if (hub) {                                   // long rows (a CTA each) + warp rows in one launch
+        static_assert(32 * kHubWarps == threads, "hub CTAs are the launch's 256-thread blocks");
+        constexpr int NBW = L >= 4 ? 1 : 4 / L;
+        const unsigned grid = (unsigned)(a.nlong + (rows - a.nlong + kHubWarps - 1) / kHubWarps);
+        if (a.deid) launch_k(k_aggregate<VEC, L, 32, NBW, true, kHubWarps>, dim3(grid), dim3(threads), 0, s, a);
+        else launch_k(k_aggregate<VEC, L, 32, NBW, false, kHubWarps>, dim3(grid), dim3(threads), 0, s, a);
+        return;
+    }
     if (warp_rows) {
         const int64_t blocks = (rows + (threads / 32) - 1) / (threads / 32);
         // NB = 1: measured on Reddit F=16, NB=2 (66 regs) is 18% slower than NB=1 (48 regs): occupancy
@@ -208,14 +254,14 @@ static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s) {
 }
 
 template <int VEC>
-static void launch_vec(AggArgs a, int L, bool warp_rows, cudaStream_t s) {
+static void launch_vec(AggArgs a, int L, bool warp_rows, cudaStream_t s, bool hub = false) {
     switch (L) {
-        case 1: launch_rl<VEC, 1>(a, warp_rows, s); break;
-        case 2: launch_rl<VEC, 2>(a, warp_rows, s); break;
-        case 4: launch_rl<VEC, 4>(a, warp_rows, s); break;
-        case 8: launch_rl<VEC, 8>(a, warp_rows, s); break;
-        case 16: launch_rl<VEC, 16>(a, warp_rows, s); break;
-        default: launch_rl<VEC, 32>(a, warp_rows, s); break;
+        case 1: launch_rl<VEC, 1>(a, warp_rows, s, hub); break;
+        case 2: launch_rl<VEC, 2>(a, warp_rows, s, hub); break;
+        case 4: launch_rl<VEC, 4>(a, warp_rows, s, hub); break;
+        case 8: launch_rl<VEC, 8>(a, warp_rows, s, hub); break;
+        case 16: launch_rl<VEC, 16>(a, warp_rows, s, hub); break;
+        default: launch_rl<VEC, 32>(a, warp_rows, s, hub); break;
     }
 }
 
@@ -231,12 +277,14 @@ seastar_status launch_aggregate(const IndexSet& x, AggArgs a, bool vec4, cudaStr
     a.nbr = x.nbr;
     AggArgs hi = a, lo = a;
     hi.row_begin = 0; hi.row_end = split;
+    hi.nlong = std::min<int64_t>(long_rows(x), split);     // long rows lead the degree-sorted order
     lo.row_begin = split; lo.row_end = x.n_rows;
+    lo.nlong = 0;
     if (vec4) {
-        launch_vec<4>(hi, L, true, s);
+        launch_vec<4>(hi, L, true, s, hi.nlong > 0);
         launch_vec<4>(lo, L, L >= 32, s);
     } else {
-        launch_vec<1>(hi, L, true, s);
+        launch_vec<1>(hi, L, true, s, hi.nlong > 0);
         launch_vec<1>(lo, L, L >= 32, s);
     }
     return check_launch("k_aggregate");

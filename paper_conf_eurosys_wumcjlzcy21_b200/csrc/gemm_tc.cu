@@ -321,11 +321,8 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 template <int NP>
 static seastar_status launch_tc_np(const CUtensorMap& tm, const TcArgs& a, cudaStream_t s) {
     using C = TcCfg<NP>;
-    static bool attr = false;
-    if (!attr) {
-        SS_CUDA(cudaFuncSetAttribute(k_gemm_tc<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
-        attr = true;
-    }
+    // set per call: the attribute is per device, and setting it is a cheap host-side call
+    SS_CUDA(cudaFuncSetAttribute(k_gemm_tc<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
     const unsigned grid = (unsigned)((a.M + C::BM - 1) / C::BM);
     k_gemm_tc<NP><<<grid, 192, C::SMEM, s>>>(tm, a);
     return check_launch("k_gemm_tc");
@@ -579,11 +576,8 @@ template <int NP32>
 static seastar_status launch_tc_tn(const CUtensorMap& tx, const CUtensorMap& ty, const TcTnArgs& a, dim3 grid,
                                    cudaStream_t s) {
     using C = TcTnCfg<NP32>;
-    static bool attr = false;
-    if (!attr) {
-        SS_CUDA(cudaFuncSetAttribute(k_gemm_tc_tn<NP32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
-        attr = true;
-    }
+    // set per call: the attribute is per device, and setting it is a cheap host-side call
+    SS_CUDA(cudaFuncSetAttribute(k_gemm_tc_tn<NP32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
     k_gemm_tc_tn<NP32><<<grid, 192, C::SMEM, s>>>(tx, ty, a);
     return check_launch("k_gemm_tc_tn");
 }

@@ -248,6 +248,18 @@ __global__ void k_rgcn_runs(int64_t N, const int64_t* __restrict__ indptr, const
     }
 }
 
+// long-row classes over degree-sorted rows: out[k] = #rows with deg >= 2^(kPow2Lo + k)
+__global__ void k_pow2_rows(int64_t n, const int32_t* __restrict__ off, long long* __restrict__ out) {
+    int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    const int32_t d = off[k + 1] - off[k];
+    const int32_t dn = (k + 1 < n) ? off[k + 2] - off[k + 1] : -1;
+    for (int i = 0; i < kPow2Classes; ++i) {
+        const int32_t th = 1 << (kPow2Lo + i);
+        if (d >= th && dn < th) out[i] = k + 1;
+    }
+}
+
 // degree buckets over degree-sorted rows: out[i] = #rows with deg >= threshold[i]; out[4] = max degree
 __global__ void k_buckets(int64_t n, const int32_t* __restrict__ off, long long* __restrict__ out) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -285,13 +297,15 @@ __global__ void k_tm_keys(int64_t n, const int32_t* __restrict__ rowidx, const i
 }
 __global__ void k_tm_fill(int64_t n, const int32_t* __restrict__ pos, const int32_t* __restrict__ src,
                           const int32_t* __restrict__ eid, const float* __restrict__ norm, int32_t* __restrict__ tsrc,
-                          int32_t* __restrict__ teid, float* __restrict__ tnorm) {
+                          int32_t* __restrict__ teid, float* __restrict__ tnorm, const int32_t* __restrict__ rowidx = nullptr,
+                          const int32_t* __restrict__ perm = nullptr, int32_t* __restrict__ tdst = nullptr) {
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i >= n) return;
     const int32_t p = pos[i];
     tsrc[i] = src[p];
     teid[i] = eid[p];
     if (tnorm) tnorm[i] = norm[p];
+    if (tdst) tdst[i] = perm[rowidx[p]];
 }
 __global__ void k_tm_run_heads(int64_t n, const uint64_t* __restrict__ key, int32_t* __restrict__ head) {
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -341,6 +355,12 @@ __global__ void k_tm_tasks(int64_t bound, long long* __restrict__ meta, const in
         task_run[tid[r]] = (int32_t)nr;
         meta[1] = tid[r];
     }
+}
+
+// ---- two-phase R-GCN edge-major views: the type of every type-major edge (from its sort key)
+__global__ void k_em_type(int64_t n, const uint64_t* __restrict__ key, int rbits, int32_t* __restrict__ type) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < n) type[i] = (int32_t)(key[i] >> rbits);
 }
 
 // ----------------------------------------------------------------------------------------------
@@ -548,6 +568,15 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
         want(&g->tm.task_run, Ef + 1, tm_on);
         want(&g->tm.task_type, Ef, tm_on);
         want(&g->tm.type_task, R + 1, tm_on);
+        want(&g->tm.dst, Ef, tm_on);
+        const bool rtm_on = etypes != nullptr && Er > 0;
+        want(&g->fem.type, Ef, tm_on);
+        want(&g->fem.pos, Ef, tm_on);
+        want(&g->rtm_nbr, Er, rtm_on);
+        want(&g->rtm_eid, Er, rtm_on);
+        want(&g->rtm_norm, Er, rtm_on && want_norm);
+        want(&g->rem.type, Er, rtm_on);
+        want(&g->rem.pos, Er, rtm_on);
         size_t total = 0;
         for (auto& sl : slots) total += (sl.bytes + 255) & ~size_t(255);
         {
@@ -694,9 +723,11 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
         }
 
         // ---- type-major runs/tasks for the R-GCN weight gradient -----------------------------------
+        constexpr int kMeta = 2 * (SEASTAR_NUM_BUCKETS + 1) + 2 + 2 * kPow2Classes;
         long long* d_b;
-        if (t.alloc(&d_b, 2 * (SEASTAR_NUM_BUCKETS + 1) + 2)) return fail(cuda_status(cudaErrorMemoryAllocation, "temps"));
-        cudaMemsetAsync(d_b, 0, sizeof(long long) * (2 * (SEASTAR_NUM_BUCKETS + 1) + 2), s);
+        if (t.alloc(&d_b, kMeta)) return fail(cuda_status(cudaErrorMemoryAllocation, "temps"));
+        cudaMemsetAsync(d_b, 0, sizeof(long long) * kMeta, s);
+        long long* d_p2 = d_b + 2 * (SEASTAR_NUM_BUCKETS + 1) + 2;   // [FWD classes | REV classes]
         long long* d_tm = d_b + 2 * (SEASTAR_NUM_BUCKETS + 1);   // [n_runs, n_tasks]
         if (etypes && Ef > 0) {
             const int rbits = bit_width((uint64_t)n_loc);
@@ -717,7 +748,7 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
             CKS_LAUNCH("k_tm_keys");
             CKS(radix_sort_pairs<uint64_t>(t, k0, k1, iota, tm_pos, Ef, rbits + tbits));
             k_tm_fill<<<grid_for(Ef, 256), 256, 0, s>>>(Ef, tm_pos, g->fwd.nbr, g->fwd.eid, g->fwd.norm, g->tm.src,
-                                                        g->tm.eid, g->tm.norm);
+                                                        g->tm.eid, g->tm.norm, rowidx, g->fwd.perm, g->tm.dst);
             k_tm_run_heads<<<grid_for(Ef, 256), 256, 0, s>>>(Ef, k1, head);
             CKS_LAUNCH("k_tm_run_heads");
             CKS(inclusive_sum(t, head, rid, Ef));
@@ -731,15 +762,45 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
                                                          g->tm.task_type, cnt);
             CKS_LAUNCH("k_tm_tasks");
             CKS(exclusive_sum(t, cnt, g->tm.type_task, R + 1));
+            // two-phase forward: the same type-major order, with each edge's type and FWD position
+            g->fem.nbr = g->tm.src; g->fem.eid = g->tm.eid; g->fem.norm = g->tm.norm; g->fem.n = Ef;
+            k_em_type<<<grid_for(Ef, 256), 256, 0, s>>>(Ef, k1, rbits, g->fem.type);
+            CK(cudaMemcpyAsync(g->fem.pos, tm_pos, sizeof(int32_t) * Ef, cudaMemcpyDeviceToDevice, s));
+            CKS_LAUNCH("k_em_type");
+        }
+        if (etypes && Er > 0) {
+            // REV edges in type-major order (type, rev row, eid) and their segments (two-phase dX)
+            const int rbits = bit_width((uint64_t)n_loc);
+            int32_t *rowidx, *iota, *pos;
+            uint64_t *k0, *k1;
+            CK(t.alloc(&rowidx, Er));
+            CK(t.alloc(&iota, Er));
+            CK(t.alloc(&pos, Er));
+            CK(t.alloc(&k0, Er));
+            CK(t.alloc(&k1, Er));
+            k_row_index<<<8 * num_sms(), 256, 0, s>>>(n_loc, g->rev.off, rowidx);
+            k_tm_keys<<<grid_for(Er, 256), 256, 0, s>>>(Er, rowidx, g->rev.type, rbits, k0);
+            k_iota<<<grid_for(Er, 256), 256, 0, s>>>(Er, iota);
+            CKS_LAUNCH("k_tm_keys(rev)");
+            CKS(radix_sort_pairs<uint64_t>(t, k0, k1, iota, pos, Er, rbits + tbits));
+            k_tm_fill<<<grid_for(Er, 256), 256, 0, s>>>(Er, pos, g->rev.nbr, g->rev.eid, g->rev.norm, g->rtm_nbr,
+                                                        g->rtm_eid, g->rtm_norm);
+            CKS_LAUNCH("k_tm_fill(rev)");
+            g->rem.nbr = g->rtm_nbr; g->rem.eid = g->rtm_eid; g->rem.norm = g->rtm_norm; g->rem.n = Er;
+            k_em_type<<<grid_for(Er, 256), 256, 0, s>>>(Er, k1, rbits, g->rem.type);
+            CK(cudaMemcpyAsync(g->rem.pos, pos, sizeof(int32_t) * Er, cudaMemcpyDeviceToDevice, s));
+            CKS_LAUNCH("k_em_type(rev)");
         }
 
         // ---- a3: degree buckets (second and last sync) --------------------------------------------
         if (n_loc > 0) {
             k_buckets<<<grid_for(n_loc, 256), 256, 0, s>>>(n_loc, g->fwd.off, d_b);
             k_buckets<<<grid_for(n_loc, 256), 256, 0, s>>>(n_loc, g->rev.off, d_b + SEASTAR_NUM_BUCKETS + 1);
+            k_pow2_rows<<<grid_for(n_loc, 256), 256, 0, s>>>(n_loc, g->fwd.off, d_p2);
+            k_pow2_rows<<<grid_for(n_loc, 256), 256, 0, s>>>(n_loc, g->rev.off, d_p2 + kPow2Classes);
         }
         CKS_LAUNCH("k_buckets");
-        long long hb[2 * (SEASTAR_NUM_BUCKETS + 1) + 2];
+        long long hb[kMeta];
         cudaMemcpyAsync(hb, d_b, sizeof(hb), cudaMemcpyDeviceToHost, s);
         cudaError_t e = cudaStreamSynchronize(s);
         if (e != cudaSuccess) return fail(cuda_status(e, "graph_create(final)"));
@@ -751,6 +812,10 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
         }
         g->fwd.bucket_rows[SEASTAR_NUM_BUCKETS - 1] = n_loc;
         g->rev.bucket_rows[SEASTAR_NUM_BUCKETS - 1] = n_loc;
+        for (int i = 0; i < kPow2Classes; ++i) {
+            g->fwd.pow2_rows[i] = hb[2 * (SEASTAR_NUM_BUCKETS + 1) + 2 + i];
+            g->rev.pow2_rows[i] = hb[2 * (SEASTAR_NUM_BUCKETS + 1) + 2 + kPow2Classes + i];
+        }
         g->fwd.max_deg = hb[SEASTAR_NUM_BUCKETS];
         g->rev.max_deg = hb[2 * SEASTAR_NUM_BUCKETS + 1];
     }  // temporaries released (stream-ordered)

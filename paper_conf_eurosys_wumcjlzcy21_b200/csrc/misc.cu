@@ -9,30 +9,44 @@
 namespace seastar {
 
 static int64_t colsum_blocks(int64_t M) {
-    int64_t b = 2 * num_sms();
-    if (M < b * 32) b = (M + 31) / 32;
+    int64_t b = 32 * num_sms();
+    if (M < b * 64) b = (M + 63) / 64;
     return b < 1 ? 1 : b;
 }
 
 size_t colsum_ws(int64_t M, int64_t F) { return (size_t)colsum_blocks(M) * (size_t)F * sizeof(float) + 256; }
 
-// stage 1: block b sums rows [b*rpb, (b+1)*rpb) of each column (8 row lanes x 32 columns, fixed order)
+// stage 1: block b sums rows [b*rpb, (b+1)*rpb) of each column; CW = min(32, pow2 >= F) column lanes x 256/CW row
+// lanes (all lanes busy for narrow F), fixed order.  fp64 accumulation: the bias gradients are column sums of
+// (softmax - onehot) / N, which cancel to ~1/sqrt(N) of their terms' total, so fp32 chains of ~10^3 terms cost
+// ~1e-5 relative (bgs-shaped db2, r2 test_gpu_fullsize)
 __global__ void __launch_bounds__(256) k_colsum1(const float* __restrict__ X, int64_t M, int64_t F, int64_t ld,
-                                                 int64_t rpb, float* __restrict__ part) {
-    __shared__ float red[8][33];
+                                                 int64_t rpb, int CW, float* __restrict__ part) {
+    __shared__ double red[256];
     const int64_t r0 = blockIdx.x * rpb, r1 = min(M, r0 + rpb);
-    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
-    for (int64_t cb = 0; cb < F; cb += 32) {
+    const int RLN = 256 / CW;
+    const int tx = threadIdx.x % CW, ty = threadIdx.x / CW;
+    for (int64_t cb = 0; cb < F; cb += CW) {
         const int64_t j = cb + tx;
-        float s = 0.f;
-        if (j < F)
-            for (int64_t r = r0 + ty; r < r1; r += 8) s += __ldg(X + r * ld + j);
-        red[ty][tx] = s;
+        double s = 0.0;
+        if (j < F) {
+            // four independent chains (fixed order), so four loads are in flight per thread
+            double s4[4] = {0.0, 0.0, 0.0, 0.0};
+            int64_t r = r0 + ty;
+            for (; r + 3 * RLN < r1; r += 4 * RLN) {
+                const float a0 = __ldg(X + r * ld + j), a1 = __ldg(X + (r + RLN) * ld + j);
+                const float a2 = __ldg(X + (r + 2 * RLN) * ld + j), a3 = __ldg(X + (r + 3 * RLN) * ld + j);
+                s4[0] += (double)a0; s4[1] += (double)a1; s4[2] += (double)a2; s4[3] += (double)a3;
+            }
+            for (int k = 0; r < r1; r += RLN, ++k) s4[k & 3] += (double)__ldg(X + r * ld + j);
+            s = (s4[0] + s4[1]) + (s4[2] + s4[3]);
+        }
+        red[threadIdx.x] = s;
         __syncthreads();
         if (ty == 0 && j < F) {
-            float x = 0.f;
-            for (int k = 0; k < 8; ++k) x += red[k][tx];
-            part[blockIdx.x * F + j] = x;
+            double x = 0.0;
+            for (int k = 0; k < RLN; ++k) x += red[k * CW + tx];
+            part[blockIdx.x * F + j] = (float)x;
         }
         __syncthreads();
     }
@@ -87,7 +101,8 @@ seastar_status colsum_impl(const float* X, int64_t M, int64_t F, int64_t ld, flo
     const int64_t nblk = colsum_blocks(M);
     const int64_t rpb = M > 0 ? (M + nblk - 1) / nblk : 1;
     float* part = static_cast<float*>(ws);
-    k_colsum1<<<(unsigned)nblk, 256, 0, s>>>(X, M, F, ld, rpb, part);
+    const int CW = F >= 32 ? 32 : pow2_ceil((int)F);
+    k_colsum1<<<(unsigned)nblk, 256, 0, s>>>(X, M, F, ld, rpb, CW, part);
     reduce_splits(part, nblk, F, F, F, F, out, s);
     return check_launch("k_colsum");
 }
@@ -203,6 +218,69 @@ __global__ void __launch_bounds__(256) k_softmax_xent4(const float* __restrict__
     }
 }
 
+// a quad of lanes per row for narrow class counts (C <= 16; the AM R-GCN output has 1.9 M rows x 11 classes):
+// lane c of the quad owns float4 chunk c of the row, so a warp reads and writes 8 consecutive rows as contiguous
+// 128-bit accesses; max / sum / label logit by 2-step xor shuffles inside the quad.  The softmax itself runs in
+// fp64 (exp / log of the fp32 logits): the bias gradient of the output layer is a column sum of these rows that
+// cancels to ~1/sqrt(N) of its terms, and fp32 softmax rounding left it at 1.0e-5 of the fp64 oracle on the
+// bgs-shaped graph (r2).  Padding columns are never written.
+__global__ void __launch_bounds__(256) k_softmax_xent_q(const float* __restrict__ Z, int64_t M, int64_t n_total,
+                                                        int C, int64_t ldz, const int64_t* __restrict__ labels,
+                                                        float* __restrict__ dZ, int64_t lddz, float* __restrict__ part) {
+    __shared__ float wl[8];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, c = lane & 3;
+    const int64_t r = ((int64_t)blockIdx.x * 256 + threadIdx.x) >> 2;
+    const bool ok = r < M;
+    const bool mine = ok && 4 * c < C;
+    double z[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+    if (mine) {
+        const float4 v = ldg4(Z + r * ldz + 4 * c);
+        z[0] = v.x; z[1] = v.y; z[2] = v.z; z[3] = v.w;
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+            if (4 * c + i >= C) z[i] = -INFINITY;
+    }
+    const int64_t lab = ok ? labels[r] : -1;
+    double m = fmax(fmax(z[0], z[1]), fmax(z[2], z[3]));
+    m = fmax(m, __shfl_xor_sync(0xffffffffu, m, 1));
+    m = fmax(m, __shfl_xor_sync(0xffffffffu, m, 2));
+    double sum = 0.0, zl = 0.0;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int j = 4 * c + i;
+        sum += (mine && j < C) ? exp(z[i] - m) : 0.0;
+        zl += (mine && j == lab) ? z[i] : 0.0;
+    }
+    sum += __shfl_xor_sync(0xffffffffu, sum, 1);
+    sum += __shfl_xor_sync(0xffffffffu, sum, 2);
+    zl += __shfl_xor_sync(0xffffffffu, zl, 1);
+    zl += __shfl_xor_sync(0xffffffffu, zl, 2);
+    const double lse = m + log(sum);
+    float loss = (ok && c == 0) ? (float)(lse - zl) : 0.f;
+    if (dZ && mine) {
+        const double inv = 1.0 / (double)n_total;
+        float d[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) d[i] = (float)((exp(z[i] - lse) - (4 * c + i == lab ? 1.0 : 0.0)) * inv);
+        float* o = dZ + r * lddz + 4 * c;
+        if (4 * c + 4 <= C && (lddz % 4) == 0 && ((reinterpret_cast<uintptr_t>(dZ) & 15u) == 0)) {
+            *reinterpret_cast<float4*>(o) = make_float4(d[0], d[1], d[2], d[3]);
+        } else {
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+                if (4 * c + i < C) o[i] = d[i];
+        }
+    }
+    for (int o = 16; o; o >>= 1) loss += __shfl_xor_sync(0xffffffffu, loss, o);
+    if (lane == 0) wl[w] = loss;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        float x = 0.f;
+        for (int k = 0; k < 8; ++k) x += wl[k];
+        part[blockIdx.x] = x;
+    }
+}
+
 __global__ void k_loss_final(const float* __restrict__ part, int64_t n, int64_t n_total, float* __restrict__ loss) {
     __shared__ double red[256];
     double x = 0.0;
@@ -307,7 +385,10 @@ seastar_status seastar_softmax_xent(const float* Z, int64_t M, int64_t n_total, 
     cudaStream_t s = to_stream(stream);
     float* part = static_cast<float*>(workspace);
     int64_t nblk;
-    if (C <= 64) {
+    if (C <= 16 && ldz % 4 == 0 && aligned16(Z)) {
+        nblk = (M + 63) / 64;
+        k_softmax_xent_q<<<(unsigned)nblk, 256, 0, s>>>(Z, M, n_total, C, ldz, labels, dZ, lddz, part);
+    } else if (C <= 64) {
         nblk = (M + 31) / 32;
         k_softmax_xent4<<<(unsigned)nblk, 256, 0, s>>>(Z, M, n_total, C, ldz, labels, dZ, lddz, part);
     } else {

@@ -521,14 +521,16 @@ class RGCN2:
 
     def forward(self):
         g, p, n = self.g, self.P, self.n
+        ws = self.ws.need(max(L.seastar_rgcn_fwd_workspace(g.handle, self.Fin, self.Hd),
+                              L.seastar_rgcn_fwd_workspace(g.handle, self.Hd, self.C), 256))
         self._X_all = self.comm.all_gather(self.X_all, self.X)
         self._t("rgcn_fwd1")
         L.seastar_rgcn_fwd(g.handle, self._X_all, self.Fin, self.X.stride(0), p.p("W1"), self.Hd, None, p.p("b1"),
-                           "relu", self.H1, self.ldh)
+                           "relu", self.H1, self.ldh, ws, ws.numel())
         self._t("rgcn_fwd1_end")
         self._H1_all = self.comm.all_gather(self.H1_all, self.H1)
         L.seastar_rgcn_fwd(g.handle, self._H1_all, self.Hd, self.ldh, p.p("W2"), self.C, None, p.p("b2"), "none",
-                           self.logits, self.ldc)
+                           self.logits, self.ldc, ws, ws.numel())
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
         L.seastar_softmax_xent(self.logits, n, self.g.N, self.C, self.ldc, self.lab, self.loss, self.dlog, self.ldc,
                                ws, ws.numel())
@@ -624,8 +626,9 @@ class RGCNBasis2:
         self._t("rgcnb_fwd1_end")
         L.seastar_basis_combine(p.p("a2"), p.p("V2"), self.R, self.B2, self.Hd * self.C, self.W2)
         self._H1_all = self.comm.all_gather(self.H1_all, self.H1)
+        ws = self.ws.need(max(L.seastar_rgcn_fwd_workspace(g.handle, self.Hd, self.C), 256))
         L.seastar_rgcn_fwd(g.handle, self._H1_all, self.Hd, self.ldh, self.W2, self.C, None, p.p("b2"), "none",
-                           self.logits, self.ldc)
+                           self.logits, self.ldc, ws, ws.numel())
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
         L.seastar_softmax_xent(self.logits, n, self.g.N, self.C, self.ldc, self.lab, self.loss, self.dlog, self.ldc,
                                ws, ws.numel())
@@ -667,7 +670,7 @@ class CapturedEpoch:
 
     def __init__(self, model):
         self.model = model
-        self.graph = torch.cuda.CUDAGraph()
+        self.graph = torch.cuda.CUDAGraph(keep_graph=True)      # kept for kernel_names()
         s = torch.cuda.Stream()
         s.wait_stream(torch.cuda.current_stream())
         with torch.cuda.graph(self.graph, stream=s):
@@ -677,6 +680,28 @@ class CapturedEpoch:
     def epoch(self):
         self.graph.replay()
         return self.loss
+
+    def kernel_names(self) -> list:
+        """Names of the kernel nodes one replay launches (read back from the captured cudaGraph_t through
+        the driver API): the measured per-epoch launch list behind bench.py's ``gpu_launches``."""
+        from cuda.bindings import driver as cu
+        g = cu.CUgraph(int(self.graph.raw_cuda_graph()))
+        err, _, n = cu.cuGraphGetNodes(g, 0)
+        err, nodes, n = cu.cuGraphGetNodes(g, n)
+        assert err == cu.CUresult.CUDA_SUCCESS, err
+        names = []
+        for nd in nodes[:n]:
+            err, t = cu.cuGraphNodeGetType(nd)
+            if t != cu.CUgraphNodeType.CU_GRAPH_NODE_TYPE_KERNEL:
+                continue
+            err, prm = cu.cuGraphKernelNodeGetParams(nd)
+            name = None
+            if int(prm.func):
+                err, name = cu.cuFuncGetName(prm.func)
+            if not name and int(prm.kern):
+                err, name = cu.cuKernelGetName(prm.kern)
+            names.append(name.decode() if isinstance(name, bytes) else str(name))
+        return names
 
 
 class PrefetchedInput:

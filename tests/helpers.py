@@ -28,3 +28,23 @@ def padded(a, ld):
     out = np.full((M, ld), np.nan, np.float32)
     out[:, :F] = a
     return out
+
+
+BORDER_DEGREES = (0, 1, 31, 32, 33, 1023, 1024, 1025, 4096)
+
+
+def border_graph(N=6000, E_bg=24000, seed=11):
+    """Random background edges plus, for every d in BORDER_DEGREES, one destination with exactly d extra in-edges
+    and one source with exactly d extra out-edges, at the bucket borders of a3 (1 / 32 / 1024).
+    The border vertices take no background edges, so their degrees are exactly d (in) and d (out)."""
+    nb = len(BORDER_DEGREES)
+    dst_v = np.arange(nb)                    # vertices 0..nb-1: in-degree d_i
+    src_v = np.arange(nb, 2 * nb)            # vertices nb..2nb-1: out-degree d_i
+    lo = 2 * nb
+    pick = lambda s, n: lo + (synth.uniform(s, (n,), 0, 1).astype(np.float64) * (N - lo)).astype(np.int64).clip(0, N - lo - 1)
+    src = [pick(seed, E_bg)]
+    dst = [pick(seed + 1, E_bg)]
+    for i, d in enumerate(BORDER_DEGREES):
+        src.append(pick(seed + 10 + i, d)); dst.append(np.full(d, dst_v[i]))       # in-degree d
+        src.append(np.full(d, src_v[i])); dst.append(pick(seed + 30 + i, d))       # out-degree d
+    return synth.csr_from_edges(N, np.concatenate(src), np.concatenate(dst))

@@ -35,7 +35,7 @@ def test_every_declared_symbol_is_exported_and_bound(lib):
 
 
 def test_abi_version_and_no_cpu_fallback(lib):
-    assert lib.seastar_abi_version() == 1
+    assert lib.seastar_abi_version() == 2
     import torch
     if not torch.cuda.is_available():
         # without a GPU every compute entry must fail loudly, never fall back to the CPU

@@ -79,3 +79,74 @@ def test_rgcn_bwd(env, Fin, Fout):
                        dev(env, W), None, None, "none", dX2, dW2, ws, ws_b)
     assert torch.equal(dW, dW2)
     assert rel_err(dX2.cpu().numpy()[:, :Fin], rdX) <= TOL
+
+
+@pytest.fixture
+def onepass(request, monkeypatch):
+    """The one-pass kernels (default) when True, the opt-in two-phase path (SEASTAR_RGCN_TWOPHASE=1) when False."""
+    if request.param:
+        monkeypatch.delenv("SEASTAR_RGCN_TWOPHASE", raising=False)
+    else:
+        monkeypatch.setenv("SEASTAR_RGCN_TWOPHASE", "1")
+    return request.param
+
+
+@pytest.mark.parametrize("onepass", [False, True], indirect=True)
+@pytest.mark.parametrize("Fin,Fout", [(16, 16), (16, 11), (3, 7)])
+def test_rgcn_two_phase_and_one_pass(env, onepass, Fin, Fout):
+    """Both R-GCN paths (one pass with W_r in shared memory per type run; opt-in two-phase lane-per-edge products in
+    type-major order + per-row sums) against the oracle, forward and dX, with a hub row of 1,500 typed in-edges."""
+    torch, L, g, N, R = env["torch"], env["L"], env["g"], env["N"], env["R"]
+    ws_f = L.seastar_rgcn_fwd_workspace(g.handle, Fin, Fout)
+    assert (ws_f == 0) == onepass
+    ldx, ldy = (Fin + 3) // 4 * 4, (Fout + 3) // 4 * 4
+    X, W, b = rnd(21, (N, Fin)), rnd(22, (R, Fin, Fout)), rnd(23, (Fout,))
+    Y = torch.full((N, ldy), float("nan"), device="cuda")
+    L.seastar_rgcn_fwd(g.handle, dev(env, padded(X, ldx)), Fin, ldx, dev(env, W), Fout, None, dev(env, b), "elu", Y,
+                       ldy)
+    ref = oracle.act_fwd("elu", oracle.rgcn_fwd(env["ip"], env["ix"], env["et"], X, W) + b)
+    assert rel_err(Y.cpu().numpy()[:, :Fout], ref) <= TOL
+    dA = rnd(24, (N, Fout))
+    dX = torch.full((N, ldx), float("nan"), device="cuda")
+    ws_b = L.seastar_rgcn_bwd_workspace(g.handle, Fin, Fout)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    L.seastar_rgcn_bwd(g.handle, dev(env, padded(X, ldx)), Fin, ldx, dev(env, padded(dA, ldy)), Fout, ldy,
+                       dev(env, W), None, None, "none", dX, None, ws, ws_b)
+    rdX, _ = oracle.rgcn_bwd(env["ip"], env["ix"], env["et"], X, W, dA, need_dW=False)
+    assert rel_err(dX.cpu().numpy()[:, :Fin], rdX) <= TOL
+
+
+def test_rgcn_fwd_workspace_required(env, monkeypatch):
+    monkeypatch.setenv("SEASTAR_RGCN_TWOPHASE", "1")
+    torch, L, g = env["torch"], env["L"], env["g"]
+    need = L.seastar_rgcn_fwd_workspace(g.handle, 16, 16)
+    assert need > 0
+    X = torch.zeros((env["N"], 16), device="cuda")
+    W = torch.zeros((env["R"], 16, 16), device="cuda")
+    Y = torch.zeros((env["N"], 16), device="cuda")
+    small = torch.empty(need - 256, dtype=torch.uint8, device="cuda")
+    with pytest.raises(RuntimeError, match="workspace"):
+        L.seastar_rgcn_fwd(g.handle, X, 16, 16, W, 16, None, None, "none", Y, 16, small, small.numel())
+
+
+@pytest.mark.parametrize("R,Fin,Fout,ok", [(210, 32, 8, True), (240, 32, 8, False), (1200, 4, 4, True)])
+def test_rgcn_shared_memory_limit(R, Fin, Fout, ok):
+    """ADVICE r1: at R = 210 the padded W table (stride 272 floats) no longer fits but the dense one (256) does;
+    R = 240 exceeds the shared memory of an SM (UNSUPPORTED); narrow layers with many relations (R = 1200, 4 x 4:
+    76 KB padded, 77 KB) fit."""
+    import torch
+    from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
+    from paper_conf_eurosys_wumcjlzcy21_b200.graph import Graph
+    N = 3000
+    ip, ix, et = synth.powerlaw_directed_typed(N, 20000, 0.6, 0.6, R, 1.0, 23)
+    g = Graph(ip, ix, et, num_etypes=R, rgcn_norm=True)
+    X, W = rnd(31, (N, Fin)), rnd(32, (R, Fin, Fout))
+    Y = torch.empty((N, Fout), device="cuda")
+    if not ok:
+        with pytest.raises(RuntimeError, match="does not fit"):
+            L.seastar_rgcn_fwd(g.handle, torch.from_numpy(X).cuda(), Fin, Fin, torch.from_numpy(W).cuda(), Fout, None,
+                               None, "none", Y, Fout)
+        return
+    L.seastar_rgcn_fwd(g.handle, torch.from_numpy(X).cuda(), Fin, Fin, torch.from_numpy(W).cuda(), Fout, None, None,
+                       "none", Y, Fout)
+    assert rel_err(Y.cpu().numpy(), oracle.rgcn_fwd(ip, ix, et, X, W)) <= TOL

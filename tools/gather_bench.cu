@@ -118,6 +118,26 @@ static void row_size(const char* dist, size_t mb, long n, int* d_idx, float4* T,
     }
 }
 
+template <int L>
+static void reddit_rows(const char* kname, long n, int* d_idx, float4* T, float* out, int sms, std::vector<int>& h,
+                        bool& first) {
+    const int rows = 232965;      // configs[4] vertex count: the gathered table is N x row_B
+    for (int pl = 0; pl < 2; ++pl) {
+        make_indices(h, rows, pl == 1);
+        CK(cudaMemcpy(d_idx, h.data(), n * 4, cudaMemcpyHostToDevice));
+        double best = 0;
+        for (int blocks : {sms * 8, sms * 16}) {
+            best = std::max(best, run<L, 2>(T, d_idx, n, blocks, out));
+            best = std::max(best, run<L, 4>(T, d_idx, n, blocks, out));
+        }
+        printf("%s    {\"dist\": \"%s\", \"table_MB\": %.1f, \"row_B\": %d, \"reddit_rows\": %d, \"for\": \"%s\", "
+               "\"GBs_best\": %.0f}", first ? "" : ",\n", pl ? "powerlaw" : "uniform", rows * 16.0 * L / (1 << 20),
+               16 * L, rows, kname, best);
+        first = false;
+    }
+    fflush(stdout);
+}
+
 int main() {
     const long n = 100l * 1000 * 1000;
     int sms;
@@ -136,24 +156,26 @@ int main() {
     printf("{\"what\": \"random-row gather ceiling: GB/s = edges*(row_B+4)/time, best of 5, 256-thread CTAs\",\n"
            " \"sms\": %d, \"l2_bytes\": %d, \"edges\": %ld,\n \"rows\": [\n", sms, l2, n);
     bool first = true;
+    // 1. the Reddit kernels' own gathered tables (N = 232,965 rows of the kernel's row size)
+    reddit_rows<4>("gcn F=16 (T, dP rows)", n, d_idx, T, out, sms, h, first);
+    reddit_rows<11>("gat layer 2 T row (ld 44)", n, d_idx, T, out, sms, h, first);
+    reddit_rows<12>("gat layer 2 backward record (ld 48)", n, d_idx, T, out, sms, h, first);
+    reddit_rows<16>("gat layer 1 T row (8x8)", n, d_idx, T, out, sms, h, first);
+    reddit_rows<18>("gat layer 1 T row + el packed (72 floats)", n, d_idx, T, out, sms, h, first);
+    reddit_rows<22>("gat layer 1 backward record (ld 88)", n, d_idx, T, out, sms, h, first);
+    // 2. fixed table sizes (L2 capacity sweep)
     const size_t sizes_mb[] = {15, 41, 60, 67, 200, 1024};
-    for (int pl = 0; pl < 2; ++pl) {
-        for (size_t mb : sizes_mb) {
-            if (pl == 1 && mb > 67) continue;   // the power-law streams only at the Reddit table sizes
-            // one index stream per (dist, table size, row size); rows = table / row bytes
-            auto go = [&](auto Ltag) {
-                constexpr int L = decltype(Ltag)::value;
-                int rows = (int)((mb << 20) / (16 * L));
-                make_indices(h, rows, pl == 1);
-                CK(cudaMemcpy(d_idx, h.data(), n * 4, cudaMemcpyHostToDevice));
-                row_size<L>(pl ? "powerlaw" : "uniform", mb, n, d_idx, T, out, sms, first);
-            };
-            go(std::integral_constant<int, 4>{});    // 64 B: GCN F = 16
-            go(std::integral_constant<int, 11>{});   // 176 B: GAT layer 2 (41 -> ld 44)
-            go(std::integral_constant<int, 16>{});   // 256 B: GAT layer 1 T row (8 x 8)
-            go(std::integral_constant<int, 24>{});   // 384 B: GAT layer 1 backward record (ld 88 -> 352 B + pad)
-            fflush(stdout);
-        }
+    for (size_t mb : sizes_mb) {
+        auto go = [&](auto Ltag) {
+            constexpr int L = decltype(Ltag)::value;
+            int rows = (int)((mb << 20) / (16 * L));
+            make_indices(h, rows, false);
+            CK(cudaMemcpy(d_idx, h.data(), n * 4, cudaMemcpyHostToDevice));
+            row_size<L>("uniform", mb, n, d_idx, T, out, sms, first);
+        };
+        go(std::integral_constant<int, 4>{});
+        go(std::integral_constant<int, 16>{});
+        fflush(stdout);
     }
     printf("\n ]}\n");
     return 0;
