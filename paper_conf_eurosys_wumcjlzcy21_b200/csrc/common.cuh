@@ -202,9 +202,10 @@ inline void set_drop(Args& a, const seastar_dropout_spec* d, const int32_t* eid)
 // ----------------------------------------------------------------------------------------------
 // L2 residency of the gathered table.  Every edge of a graph kernel gathers a row of one table
 // (T, dP, the GAT record D, X ...) that is 15-90 MB and therefore *could* live in the 126 MB L2, while
-// the edge-index stream (4-8 B per edge, 0.5-1 GB) and the outputs stream through once.  Graph kernels
-// are launched with an access-policy window over the gathered table (hits persist, misses stream) and
-// read their index streams with evict-first loads (__ldcs).
+// the edge-index stream (4-8 B per edge, 0.5-1 GB) and the outputs stream through once.  Graph kernels read
+// their index streams with evict-first loads (__ldcs).  The GAT backward and R-GCN launches can also carry an
+// access-policy window over the gathered table (hits persist, misses stream) -- opt-in (SEASTAR_L2_PERSIST=1,
+// l2_persist_bytes()): the persisting set-aside is device-wide and shrinks the L2 of every other kernel.
 // ----------------------------------------------------------------------------------------------
 struct L2Window {
     const void* base = nullptr;

@@ -79,7 +79,7 @@ __global__ void __launch_bounds__(256) k_gat_fwd(const GatFwdArgs a) {
                 const int u = __shfl_sync(gmask, my, k & (RL - 1), RL);
                 mk[jj] = 1.f;
                 if (k < n && active) {
-                    z[jj] = lrelu(__ldg(a.el + (int64_t)u * a.H + h) + erv, a.slope);
+                    z[jj] = lrelu(__ldg(a.el + (int64_t)u * a.ldel + h) + erv, a.slope);
                     load_vec<VEC>(a.T + (int64_t)u * a.ld + col, val[jj]);
                     if (DROP)
                         mk[jj] = drop_mult(dkey, (uint64_t)__ldg(a.deid + base + k) * a.H + h, a.dthr, a.dscale);
@@ -196,7 +196,7 @@ __global__ void __launch_bounds__(256) k_gat_bwd(const GatBwdArgs a) {
 #pragma unroll
     for (int i = 0; i < VEC; ++i)   // padding columns never enter the head dot products
         if (!(valid && active) || col + i >= W) t[i] = 0.f;
-    const float elu = (valid && active) ? __ldg(a.el + u * a.H + h) : 0.f;
+    const float elu = (valid && active) ? __ldg(a.el + u * a.ldel + h) : 0.f;
     float acc[VEC], dl = 0.f;
 #pragma unroll
     for (int i = 0; i < VEC; ++i) acc[i] = 0.f;
@@ -327,7 +327,7 @@ __global__ void __launch_bounds__(256) k_gat_der(const GatBwdArgs a) {
 #pragma unroll
                     for (int i = 0; i < VEC; ++i)
                         if (col + i >= W) t[jj][i] = 0.f;
-                    elu[jj] = __ldg(a.el + (int64_t)u * a.H + h);
+                    elu[jj] = __ldg(a.el + (int64_t)u * a.ldel + h);
                 } else {
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) t[jj][i] = 0.f;
@@ -368,7 +368,7 @@ __global__ void __launch_bounds__(256) k_gat_der(const GatBwdArgs a) {
 // thread per (u,h): el/er projections
 __global__ void k_gat_attn_proj(const float* __restrict__ T, int64_t M, int H, int F, int64_t ldt,
                                 const float* __restrict__ a_l, const float* __restrict__ a_r, float* __restrict__ el,
-                                float* __restrict__ er) {
+                                float* __restrict__ er, int64_t ldel) {
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i >= M * H) return;
     const int64_t u = i / H;
@@ -380,7 +380,7 @@ __global__ void k_gat_attn_proj(const float* __restrict__ T, int64_t M, int H, i
         sl = fmaf(x, __ldg(a_l + h * F + f), sl);
         sr = fmaf(x, __ldg(a_r + h * F + f), sr);
     }
-    if (el) el[i] = sl;
+    if (el) el[u * ldel + h] = sl;
     if (er) er[i] = sr;
 }
 
@@ -705,7 +705,10 @@ seastar_status seastar_gat_attn_proj(const float* T, int64_t M, int32_t H, int32
     SS_TRY(check_device());
     if (M == 0) return SEASTAR_OK;
     const int64_t n = M * H;
-    k_gat_attn_proj<<<(unsigned)((n + 255) / 256), 256, 0, to_stream(stream)>>>(T, M, H, F, ldt, a_l, a_r, el, er);
+    const int64_t ldel = el_stride(T, el, H, F, ldt);
+    SS_ARG(ldel == H || ldt >= (int64_t)H * F + H, "gat_attn_proj: el packed into T needs ldt >= H*F + H");
+    k_gat_attn_proj<<<(unsigned)((n + 255) / 256), 256, 0, to_stream(stream)>>>(T, M, H, F, ldt, a_l, a_r, el, er,
+                                                                                ldel);
     return check_launch("k_gat_attn_proj");
 }
 
@@ -725,6 +728,8 @@ seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float*
     a.perm = g->fwd.perm; a.off = g->fwd.off; a.nbr = g->fwd.nbr;
     a.vbase = g->row_begin;
     a.T = T_all; a.el = el_all; a.er = er_loc;
+    a.ldel = el_stride(T_all, el_all, H, F, ldt);
+    SS_ARG(a.ldel == H || ldt >= (int64_t)H * F + H, "gat_fwd: el packed into T needs ldt >= H*F + H");
     a.H = H; a.F = F; a.ld = ldt; a.slope = slope; a.bias = bias; a.act = act;
     a.A = A_loc; a.Y = Y_loc; a.lse = lse_loc; a.B = B_loc; a.bsum = b_loc;
     a.row_begin = 0; a.row_end = g->fwd.n_rows;
@@ -796,6 +801,8 @@ seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float*
     a.perm = g->rev.perm; a.off = g->rev.off; a.nbr = g->rev.nbr;
     a.vbase = g->row_begin;
     a.T = T_loc; a.el = el_loc; a.D = D_all;
+    a.ldel = el_stride(T_loc, el_loc, H, F, ldt);
+    SS_ARG(a.ldel == H || ldt >= (int64_t)H * F + H, "gat_bwd: el packed into T needs ldt >= H*F + H");
     a.H = H; a.F = F; a.ldt = ldt; a.ldd = seastar_gat_record_ld(H, F); a.slope = slope;
     a.dT = dT_loc; a.del = del_loc;
     ScopedL2Window win(D_all, (size_t)g->N * a.ldd * sizeof(float));
@@ -827,6 +834,8 @@ seastar_status seastar_gat_der(seastar_graph g, const float* T_all, const float*
     a.perm = g->fwd.perm; a.off = g->fwd.off; a.nbr = g->fwd.nbr;
     a.vbase = g->row_begin;
     a.T = T_all; a.el = el_all; a.D = D_loc;
+    a.ldel = el_stride(T_all, el_all, H, F, ldt);
+    SS_ARG(a.ldel == H || ldt >= (int64_t)H * F + H, "gat_der: el packed into T needs ldt >= H*F + H");
     a.H = H; a.F = F; a.ldt = ldt; a.ldd = seastar_gat_record_ld(H, F); a.slope = slope;
     a.der = der_loc;
     a.row_begin = 0; a.row_end = g->fwd.n_rows;

@@ -35,6 +35,7 @@ struct GatFwdArgs {
     int64_t row_begin, row_end, vbase;
     const float* T; const float* el; const float* er;
     int H, F; int64_t ld; float slope;
+    int64_t ldel;            // row stride of el (H, or ld when el is packed into T's padding: el == T + H*F)
     const float* bias; int act;
     float* A; float* Y; float* lse;
     float* B; float* bsum;   // optional: der factors (see k_gat_fwd_hpl)
@@ -51,6 +52,7 @@ struct GatBwdArgs {
     const float* el;     // gathered (der) or owned (src-major)
     const float* D;      // packed records: gathered (src-major) or owned (der)
     int H, F; int64_t ldt, ldd; float slope;
+    int64_t ldel;        // row stride of el (see GatFwdArgs)
     float* dT; float* del;   // src-major outputs
     float* der;              // der output
     const int32_t* deid; uint64_t dseed; const int32_t* dstep; uint32_t dsite, dthr; float dscale;   // as GatFwdArgs
@@ -59,13 +61,20 @@ struct GatBwdArgs {
 
 
 // packed backward record D[v] = [dA (H*F, zero-padded to a multiple of 4) | per head (er, lse, c, nl2)]
-// with nl2 = -lse * log2(e), so a_e = ex2(LReLU(s_e) log2 e + nl2) is one FFMA + one SFU op
-__device__ __forceinline__ int rec_aux_offset(int W) { return (W + 3) & ~3; }
+// with nl2 = -lse * log2(e), so a_e = ex2(LReLU(s_e) log2 e + nl2) is one FFMA + one SFU op.  (Measured in r2: a
+// 3-scalar layout [er | c | nl2] without lse saves one of the 12 sectors of the 8x8 record but needs three 32-bit
+// loads per head instead of one 128-bit load, and the layer-1 backward went from 2.62 to 2.96 ms -- it is L1-bound.)
+__host__ __device__ __forceinline__ int rec_aux_offset(int W) { return (W + 3) & ~3; }
 
 // 32-bit row offset -> 64-bit address in one IMAD.WIDE.U32 (row strides are < 2^31 floats, checked
 // at the ABI)
 __device__ __forceinline__ const float* row_ptr(const float* base, int r, int64_t ld) {
     return base + (size_t)(uint32_t)r * (uint32_t)ld;
+}
+
+// el packed into the first padding columns of T (el == T + H*F, row stride ldt) or a separate [rows, H] table
+inline int64_t el_stride(const float* T, const float* el, int H, int F, int64_t ldt) {
+    return (el == T + (int64_t)H * F) ? ldt : (int64_t)H;
 }
 
 // launchers (return false when the geometry does not apply)

@@ -87,7 +87,7 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
                 const int k = (b * UE + jj) * S + slot;     // < RL
                 const int u = __shfl_sync(gmask, my, k, RL);
                 load_lane_chunks<VPL, L>(row_ptr(Tc, u, a.ld), qv, x[jj]);
-                const float s = __ldg(a.el + u) + erv;
+                const float s = __ldg(a.el + (size_t)(uint32_t)u * (size_t)a.ldel) + erv;
                 z[jj] = k < n ? lrelu(s, slope) : -INFINITY;
             }
             float mb = m;
@@ -255,7 +255,7 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdA
     float4 k4 = make_float4(0.f, 0.f, 0.f, 0.f);   // src-major: (el_u, -, -, -); der: (er, lse, c, nl2)_v
     if (!DER) {
         load_lane_chunks<VPL, L>(a.T + w * a.ldt + col0, qv, own);
-        if (valid) k4.x = __ldg(a.el + w);
+        if (valid) k4.x = __ldg(a.el + w * a.ldel);
     } else {
         load_lane_chunks<VPL, L>(a.D + w * a.ldd + col0, qv, own);
         if (valid) k4 = ldg4(a.D + w * a.ldd + aux0);
@@ -290,7 +290,7 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdA
                 if (!DER) {
                     e[jj] = ldg4(row_ptr(a.D + aux0, o, a.ldd));          // (er, lse, c, nl2)_v
                 } else {
-                    e[jj] = make_float4(__ldg(a.el + o), 0.f, 0.f, 0.f);  // el_u
+                    e[jj] = make_float4(__ldg(a.el + (size_t)(uint32_t)o * (size_t)a.ldel), 0.f, 0.f, 0.f);  // el_u
                     // gathered T rows may carry non-finite padding (NaN * 0 = NaN): zero it
 #pragma unroll
                     for (int q = 0; q < VPL; ++q) x[jj][q] = mask_tail(x[jj][q], nvalid[q]);

@@ -429,9 +429,11 @@ constexpr int kHubWarpsGat = 8;
         default: SS_HPL_F4B(KERNEL, 32, f4, __VA_ARGS__) break;      \
     }
 
+// the head-per-lane kernels read el at the compile-time row stride H (a runtime stride in the hot loop cost the
+// layer-1 backward a spill reload and 50 % on Reddit, r2): an el packed into T's padding takes the generic kernels
 bool launch_gat_fwd_hpl(const GatFwdArgs& a0, int64_t hub, cudaStream_t s) {
     const int f4 = hpl_f4(a0.H, a0.F, a0.ld, aligned16(a0.T) && aligned16(a0.A) && aligned16(a0.Y));
-    if (!f4) return false;
+    if (!f4 || a0.ldel != a0.H) return false;
     static_assert(32 * kHubWarpsGat == 256, "long-row CTAs are the launch's 256-thread blocks");
     GatFwdArgs a = a0;
     a.nlong = std::min<int64_t>(std::max<int64_t>(hub - a0.row_begin, 0), a0.row_end - a0.row_begin);
@@ -449,7 +451,7 @@ bool launch_gat_fwd_hpl(const GatFwdArgs& a0, int64_t hub, cudaStream_t s) {
 
 bool launch_gat_bwd_hpl(const GatBwdArgs& a0, int64_t hub, cudaStream_t s) {
     const int f4 = hpl_f4(a0.H, a0.F, a0.ldt, aligned16(a0.T) && aligned16(a0.D) && aligned16(a0.dT));
-    if (!f4) return false;
+    if (!f4 || a0.ldel != a0.H) return false;
     GatBwdArgs a = a0;
     a.nlong = std::min<int64_t>(std::max<int64_t>(hub - a0.row_begin, 0), a0.row_end - a0.row_begin);
     const unsigned grid = (unsigned)(a.nlong + (a.row_end - a.row_begin - a.nlong + 7) / 8);
@@ -461,7 +463,7 @@ bool launch_gat_bwd_hpl(const GatBwdArgs& a0, int64_t hub, cudaStream_t s) {
 
 bool launch_gat_der_hpl(const GatBwdArgs& a, cudaStream_t s) {
     const int f4 = hpl_f4(a.H, a.F, a.ldt, aligned16(a.T) && aligned16(a.D));
-    if (!f4) return false;
+    if (!f4 || a.ldel != a.H) return false;
     const unsigned grid = (unsigned)((a.row_end - a.row_begin + 7) / 8);
     if (grid) { SS_HPL_H(k_gat_der_hpl, a.H, f4) }
     return true;

@@ -51,7 +51,11 @@ size_t l2_persist_bytes() {
         init[dev] = true;
         per_dev[dev] = 0;
         int maxp = 0;
-        if (getenv("SEASTAR_NO_L2_PERSIST") == nullptr &&
+        // opt-in (SEASTAR_L2_PERSIST=1): the set-aside is device-wide and not stream-ordered, so once reserved it
+        // shrinks the normal L2 for every later kernel -- measured on Reddit (r2): 13.92 ms/step with the window on
+        // the GAT backward's records, 13.37 ms without it (stale persisting lines)
+        const char* on = getenv("SEASTAR_L2_PERSIST");
+        if (on != nullptr && on[0] == '1' &&
             cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev) == cudaSuccess && maxp > 0 &&
             cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp) == cudaSuccess)
             per_dev[dev] = maxp;

@@ -268,12 +268,16 @@ class GAT2:
         self.ad = {"1": L.dropout_spec(attn_dropout, 3, seed, self.P.step),
                    "2": L.dropout_spec(attn_dropout, 4, seed, self.P.step)}
         n, W1w, C = _local_rows(self), self.W1w, self.C
-        self.ld1, self.ld2 = _ld(W1w), _ld(C)
+        # layer 2 (one head): el2 lives in T2's first padding column (seastar_gat_fwd: el_all == T_all + H*F) and the
+        # row stride is a whole number of 32-byte sectors, so a gathered T2 row brings its el2 along -- 6 sectors per
+        # edge on Reddit (C = 41, ld 48) instead of 6.5 + 1 for a separate el table
+        self.ld1, self.ld2 = _ld(W1w), (C + 1 + 7) // 8 * 8
         e = lambda r, c: torch.zeros((r, c), device=dev)
         self.T1, self.A1, self.Y1 = e(n, self.ld1), e(n, self.ld1), e(n, self.ld1)
         self.el1, self.er1, self.lse1 = e(n, heads), e(n, heads), e(n, heads)
         self.T2, self.A2, self.Y2 = e(n, self.ld2), e(n, self.ld2), e(n, self.ld2)
-        self.el2, self.er2, self.lse2 = e(n, 1), e(n, 1), e(n, 1)
+        self.el2 = self.T2[:, C:C + 1]
+        self.er2, self.lse2 = e(n, 1), e(n, 1)
         self.dY2 = e(n, self.ld2)
         self.ldd1, self.ldd2 = L.seastar_gat_record_ld(heads, hidden), L.seastar_gat_record_ld(1, C)
         self.D1, self.D2 = e(n, self.ldd1), e(n, self.ldd2)
@@ -295,7 +299,7 @@ class GAT2:
         self.T1_all = e(R, self.ld1) if P > 1 else None
         self.el1_all = e(R, heads) if P > 1 else None
         self.T2_all = e(R, self.ld2) if P > 1 else None
-        self.el2_all = e(R, 1) if P > 1 else None
+        self.el2_all = None                                   # packed into T2_all's rows
         self.D1_all = e(R, self.ldd1) if P > 1 else None
         self.D2_all = e(R, self.ldd2) if P > 1 else None
         self.timer = None
@@ -326,7 +330,7 @@ class GAT2:
         _linear(self.ws, self.Y1d, n, W, self.ld1, p.p("W2"), C, None, None, "none", self.T2, self.ld2)
         L.seastar_gat_attn_proj(self.T2, n, 1, C, self.ld2, p.p("al2"), p.p("ar2"), self.el2, self.er2)
         T2_all = self.comm.all_gather(self.T2_all, self.T2)
-        el2_all = self.comm.all_gather(self.el2_all, self.el2)
+        el2_all = T2_all[:, C:C + 1]                          # el2 travels inside the gathered T2 rows
         self._gathered2 = (T2_all, el2_all)
         self._t("gat_fwd2")
         L.seastar_gat_fwd(g.handle, T2_all, el2_all, self.er2, 1, C, self.ld2, self.slope, p.p("b2"), "none", self.A2,
