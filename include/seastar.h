@@ -215,6 +215,29 @@ seastar_status seastar_gcn_bwd(seastar_graph g, const float* dP_all, int64_t F, 
                                float scale, const float* Yact_loc, seastar_act act, const float* post_scale,
                                float* dA_loc, float* dP_loc, const seastar_dropout_spec* edge_drop,
                                seastar_stream stream);
+/*
+ * NEXT-1 (multi-GPU overlap): seastar_gcn_fwd / seastar_gcn_bwd of a row-partitioned graph in two
+ * phases around the all-gather of the source table.  graph_create keeps, per owned row, its edges re-ordered with
+ * the edges whose neighbour is an owned vertex first.
+ *   phase 1: part[v, :F] = sum over the owned-neighbour edges of the row, read from the rank's OWN rows (T_loc /
+ *            dP_loc_in [n_loc, F] ld ldloc, row i = vertex row_begin + i) -- it needs no gathered data, so it runs
+ *            while the all-gather is in flight; no epilogue.  T_all / dP_all and the outputs are ignored.
+ *   phase 2: the remaining edges from the gathered table (T_all / dP_all), + part, then the same epilogue as
+ *            seastar_gcn_fwd / seastar_gcn_bwd (all their arguments keep their meaning).  T_loc is ignored.
+ *   part: [n_loc, F] ld ldp (dev, caller-owned scratch, written by phase 1 and read by phase 2).
+ * The sum is taken in (owned part, rest) order: deterministic, and within the tolerance of the one-phase call
+ * (the order of a row's terms differs).  INVALID_ARGUMENT for an unpartitioned graph.
+ */
+seastar_status seastar_gcn_fwd_split(seastar_graph g, int32_t phase, const float* T_loc, int64_t ldloc,
+                                     const float* T_all, int64_t F, int64_t ld, const float* dst_norm,
+                                     const float* bias, seastar_act act, float alpha, const float* H0_loc,
+                                     float* Y_loc, const float* out_scale, float* Ys_loc, float* part, int64_t ldp,
+                                     const seastar_dropout_spec* edge_drop, seastar_stream stream);
+seastar_status seastar_gcn_bwd_split(seastar_graph g, int32_t phase, const float* dP_loc_in, int64_t ldloc,
+                                     const float* dP_all, int64_t F, int64_t ld, const float* src_norm, float scale,
+                                     const float* Yact_loc, seastar_act act, const float* post_scale, float* dA_loc,
+                                     float* dP_loc, float* part, int64_t ldp, const seastar_dropout_spec* edge_drop,
+                                     seastar_stream stream);
 
 /* ------------------------------------------------------------------------------------------ */
 /* a6 / a9: GAT (Fig. 2 L95-L123, Fig. 3, FSM units L391-L393)                   */
@@ -399,6 +422,10 @@ seastar_status seastar_colsum(const float* X, int64_t M, int64_t F, int64_t ld, 
 size_t seastar_colsum_workspace(int64_t M, int64_t F);
 /* y = a * x + b * y over n floats */
 seastar_status seastar_axpby(int64_t n, float a, const float* x, float b, float* y, seastar_stream stream);
+/* Y[i, :F] = scale[i] * X[i, :F] for i < M (dev; ldx, ldy >= F; Y may alias X) -- the APPNP propagation's
+ * n (.) pre-scaling of a table (reading #23), without a dense transform */
+seastar_status seastar_row_scale(const float* X, int64_t M, int64_t F, int64_t ldx, const float* scale, float* Y,
+                                 int64_t ldy, seastar_stream stream);
 /*
  * One Adam step over a flat parameter buffer (Kingma & Ba Alg. 1), step number read from
  * *step (dev int32, >= 1) so the call can be captured in a CUDA graph; see seastar_step_inc.

@@ -66,6 +66,10 @@ _SIGS = {
     "seastar_linear_bwd_weight_workspace": ([_I64, _I64, _I64], _SZ),
     "seastar_gcn_fwd": ([_P, _P, _I64, _I64, _P, _P, _I32, _F, _P, _P, _P, _P, _P, _P], _ST),
     "seastar_gcn_bwd": ([_P, _P, _I64, _I64, _P, _F, _P, _I32, _P, _P, _P, _P, _P], _ST),
+    "seastar_gcn_fwd_split": ([_P, _I32, _P, _I64, _P, _I64, _I64, _P, _P, _I32, _F, _P, _P, _P, _P, _P, _I64, _P, _P],
+                              _ST),
+    "seastar_gcn_bwd_split": ([_P, _I32, _P, _I64, _P, _I64, _I64, _P, _F, _P, _I32, _P, _P, _P, _P, _I64, _P, _P],
+                              _ST),
     "seastar_gat_attn_proj": ([_P, _I64, _I32, _I32, _I64, _P, _P, _P, _P, _P], _ST),
     "seastar_gat_fwd": ([_P, _P, _P, _P, _I32, _I32, _I64, _F, _P, _I32, _P, _P, _P, _P, _P, _P, _P], _ST),
     "seastar_gat_record_ld": ([_I32, _I32], _I64),
@@ -89,6 +93,7 @@ _SIGS = {
     "seastar_colsum": ([_P, _I64, _I64, _I64, _P, _P, _SZ, _P], _ST),
     "seastar_colsum_workspace": ([_I64, _I64], _SZ),
     "seastar_axpby": ([_I64, _F, _P, _F, _P, _P], _ST),
+    "seastar_row_scale": ([_P, _I64, _I64, _I64, _P, _P, _I64, _P], _ST),
     "seastar_adam": ([_P, _P, _P, _P, _I64, _F, _F, _F, _F, _P, _P], _ST),
     "seastar_step_inc": ([_P, _P], _ST),
 }
@@ -245,6 +250,22 @@ def seastar_gcn_bwd(g, dP_all, F, ld, src_norm, scale, Yact_loc, act, post_scale
           _dptr(dP_loc, "dP"), _spec(edge_drop), _stream(stream))
 
 
+def seastar_gcn_fwd_split(g, phase, T_loc, ldloc, T_all, F, ld, dst_norm, bias, act, alpha, H0_loc, Y_loc,
+                          out_scale, Ys_loc, part, ldp, stream=None, edge_drop=None) -> None:
+    _call("seastar_gcn_fwd_split", g, int(phase), _dptr(T_loc, "T_loc"), ldloc, _dptr(T_all, "T_all"), F, ld,
+          _dptr(dst_norm, "dst_norm"), _dptr(bias, "bias"), _act(act), float(alpha), _dptr(H0_loc, "H0"),
+          _dptr(Y_loc, "Y"), _dptr(out_scale, "out_scale"), _dptr(Ys_loc, "Ys"), _dptr(part, "part"), ldp,
+          _spec(edge_drop), _stream(stream))
+
+
+def seastar_gcn_bwd_split(g, phase, dP_loc_in, ldloc, dP_all, F, ld, src_norm, scale, Yact_loc, act, post_scale,
+                          dA_loc, dP_loc, part, ldp, stream=None, edge_drop=None) -> None:
+    _call("seastar_gcn_bwd_split", g, int(phase), _dptr(dP_loc_in, "dP_loc_in"), ldloc, _dptr(dP_all, "dP_all"), F,
+          ld, _dptr(src_norm, "src_norm"), float(scale), _dptr(Yact_loc, "Yact"), _act(act),
+          _dptr(post_scale, "post_scale"), _dptr(dA_loc, "dA"), _dptr(dP_loc, "dP"), _dptr(part, "part"), ldp,
+          _spec(edge_drop), _stream(stream))
+
+
 # ----------------------------------------------------------------------------------- GAT
 def seastar_gat_attn_proj(T, M, H, F, ldt, a_l, a_r, el, er, stream=None) -> None:
     _call("seastar_gat_attn_proj", _dptr(T, "T"), M, H, F, ldt, _dptr(a_l, "a_l"), _dptr(a_r, "a_r"),
@@ -388,6 +409,10 @@ def seastar_colsum_workspace(M, F) -> int:
 def seastar_colsum(X, M, F, ld, out, workspace, ws_bytes, stream=None) -> None:
     _call("seastar_colsum", _dptr(X, "X"), M, F, ld, _dptr(out, "out"), _dptr(workspace, "workspace"), ws_bytes,
           _stream(stream))
+
+
+def seastar_row_scale(X, M, F, ldx, scale, Y, ldy, stream=None) -> None:
+    _call("seastar_row_scale", _dptr(X, "X"), M, F, ldx, _dptr(scale, "scale"), _dptr(Y, "Y"), ldy, _stream(stream))
 
 
 def seastar_axpby(n, a, x, b, y, stream=None) -> None:

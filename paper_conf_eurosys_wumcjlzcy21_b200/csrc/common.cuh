@@ -76,6 +76,15 @@ struct TypeMajor {
     int32_t* dst = nullptr;       // [Ef] destination vertex id of each edge (run boundaries = changes of dst in a task)
     int64_t n_runs = 0, n_tasks = 0;
 };
+// NEXT-1: an index set's rows with their edges re-ordered so that the edges whose neighbour is an
+// owned vertex come first (stable, eid order inside each part).  The partitioned aggregation runs the owned-neighbour
+// part from the rank's own table while the all-gather of the other ranks' rows is in flight, then the rest.
+struct LocalSplit {
+    int32_t* nbr = nullptr;    // [E] neighbour id, row-major like the index set (same off[])
+    int32_t* eid = nullptr;    // [E] user edge id
+    int32_t* lcnt = nullptr;   // [n_rows] owned-neighbour edges at the front of each row
+};
+
 constexpr int kTaskEdges = 512;   // edges per dW task (a task may exceed it only inside one run)
 
 // Two-phase R-GCN (a7 forward on FWD, a10 dX on REV; rgcn.cu): an index set's edges in type-major order
@@ -101,6 +110,7 @@ struct seastar_graph_s {
     uint32_t flags = 0;
     bool partitioned = false;
     seastar::IndexSet fwd, rev, lsf;
+    seastar::LocalSplit fsplit, rsplit;  // partitioned only: rows' edges with owned neighbours first (NEXT-1)
     seastar::TypeMajor tm;
     seastar::EdgeMajor fem, rem;     // two-phase R-GCN: FWD (forward) and REV (dX) edges in type-major order
     int32_t* rtm_nbr = nullptr;      // REV edges in type-major order (rem's edge arrays)

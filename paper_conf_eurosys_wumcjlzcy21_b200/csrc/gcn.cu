@@ -40,6 +40,10 @@ struct AggArgs {
     // NEXT-3 edge dropout (deid == nullptr: off): edge k's message is scaled by drop_mult(key, eid[k])
     const int32_t* deid; uint64_t dseed; const int32_t* dstep; uint32_t dsite, dthr; float dscale;
     int64_t nlong;         // WPR > 1 launches: blocks [0, nlong) are long rows (a CTA each), the rest 8 warp-rows
+    // NEXT-1 split phases over a LocalSplit (phase 0: whole rows, no split): phase 1 sums each row's owned-neighbour
+    // edges from tloc (the rank's own rows, ld ldloc) into part (ld ldp, no epilogue) while the all-gather of the
+    // table runs; phase 2 sums the remaining edges from the gathered table, adds part, and runs the epilogue
+    int phase; const int32_t* lcnt; const float* tloc; int64_t ldloc; float* part; int64_t ldp;
 };
 
 // minimum resident blocks (0: compiler's choice, 48 registers at F = 16).  Measured on Reddit: forcing 6 blocks
@@ -81,6 +85,12 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
     const bool valid = row < a.row_end;
     int beg = valid ? __ldg(a.off + row) : 0;
     int end = valid ? __ldg(a.off + row + 1) : 0;
+    if (a.phase && valid) {                      // NEXT-1: owned-neighbour edges lead every split row
+        const int lc = __ldg(a.lcnt + row);
+        if (a.phase == 1) end = beg + lc; else beg += lc;
+    }
+    const float* tab = a.phase == 1 ? a.tloc - a.vbase * a.ldloc : a.table;   // phase 1: the rank's own rows
+    const int64_t tld = a.phase == 1 ? a.ldloc : a.ld;
     if (hubblk) {
         const int64_t len = end - beg;
         const int b0 = beg + (int)(len * wib / WPR);
@@ -125,7 +135,7 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
                         const int k = (j0 + jj) * S + slot;
                         const int u = __shfl_sync(gmask, my[h], k & (RL - 1), RL);
                         if (k < n[h] && active) {
-                            load_vec<VEC>(a.table + (int64_t)u * a.ld + col, val[h][jj]);
+                            load_vec<VEC>(tab + (int64_t)u * tld + col, val[h][jj]);
                             if (DROP) {
                                 const float w = drop_mult(dkey, (uint64_t)__ldg(a.deid + base + h * RL + k), a.dthr,
                                                           a.dscale);
@@ -169,6 +179,18 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
         }
 
         if (!valid || slot != 0 || !active) continue;
+        if (a.phase == 1) {                          // partial row sum, finished by phase 2
+            float* pp = a.part + v * a.ldp + col;
+            if (col + VEC <= a.F) store_vec<VEC>(pp, acc);
+            else for (int i = 0; i < VEC && col + i < a.F; ++i) pp[i] = acc[i];
+            continue;
+        }
+        if (a.phase == 2) {
+            const float* pp = a.part + v * a.ldp + col;
+#pragma unroll
+            for (int i = 0; i < VEC; ++i)
+                if (col + i < a.F) acc[i] += pp[i];
+        }
         const float rs = (a.rscale ? __ldg(a.rscale + v) : 1.f) * a.gscale;
         float out[VEC], out2[VEC];
         if (!a.bwd) {
@@ -266,15 +288,18 @@ static void launch_vec(AggArgs a, int L, bool warp_rows, cudaStream_t s, bool hu
 }
 
 // launch over the two degree classes of an index set: rows with degree >= 32 get a warp each,
-// the rest (incl. empty rows, which still need their epilogue) get sub-warp row groups
-seastar_status launch_aggregate(const IndexSet& x, AggArgs a, bool vec4, cudaStream_t s) {
+// the rest (incl. empty rows, which still need their epilogue) get sub-warp row groups; sp: the local-first split
+// of x (NEXT-1 phases 1 / 2) or nullptr
+seastar_status launch_aggregate(const IndexSet& x, AggArgs a, bool vec4, cudaStream_t s,
+                                const LocalSplit* sp = nullptr) {
     const int VEC = vec4 ? 4 : 1;
     const int C = (a.F + VEC - 1) / VEC;
     const int L = C >= 32 ? 32 : pow2_ceil(C);
     const int64_t split = x.bucket_rows[1];   // # rows with degree >= 32
     a.perm = x.perm;
     a.off = x.off;
-    a.nbr = x.nbr;
+    a.nbr = sp ? sp->nbr : x.nbr;
+    a.lcnt = sp ? sp->lcnt : nullptr;
     AggArgs hi = a, lo = a;
     hi.row_begin = 0; hi.row_end = split;
     hi.nlong = std::min<int64_t>(long_rows(x), split);     // long rows lead the degree-sorted order
@@ -340,6 +365,66 @@ seastar_status seastar_gcn_bwd(seastar_graph g, const float* dP_all, int64_t F, 
     bool vec4 = (ld % 4 == 0) && aligned16(dP_all) && (!dA_loc || aligned16(dA_loc)) && (!dP_loc || aligned16(dP_loc)) &&
                 (!Yact_loc || aligned16(Yact_loc));
     return launch_aggregate(g->rev, a, vec4, to_stream(stream));
+}
+
+// NEXT-1: the partitioned aggregation in two phases around the all-gather (seastar.h)
+seastar_status seastar_gcn_fwd_split(seastar_graph g, int32_t phase, const float* T_loc, int64_t ldloc,
+                                     const float* T_all, int64_t F, int64_t ld, const float* dst_norm,
+                                     const float* bias, seastar_act act, float alpha, const float* H0_loc,
+                                     float* Y_loc, const float* out_scale, float* Ys_loc, float* part, int64_t ldp,
+                                     const seastar_dropout_spec* edge_drop, seastar_stream stream) {
+    SS_ARG(g != nullptr, "gcn_fwd_split: graph is NULL");
+    SS_ARG(g->partitioned, "gcn_fwd_split: the graph is not row-partitioned (use seastar_gcn_fwd)");
+    SS_ARG(phase == 1 || phase == 2, "gcn_fwd_split: phase must be 1 or 2");
+    SS_ARG(F >= 1 && ld >= F && ldp >= F, "gcn_fwd_split: bad sizes");
+    SS_ARG(part != nullptr, "gcn_fwd_split: part is NULL");
+    SS_ARG(phase == 2 || (T_loc && ldloc >= F), "gcn_fwd_split: phase 1 needs T_loc (ldloc >= F)");
+    SS_ARG(phase == 1 || (T_all && Y_loc), "gcn_fwd_split: phase 2 needs T_all and Y_loc");
+    SS_ARG(!Ys_loc || out_scale, "gcn_fwd_split: Ys_loc requires out_scale");
+    SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "gcn_fwd_split: bad activation %d", (int)act);
+    SS_ARG(!edge_drop || (edge_drop->p >= 0.f && edge_drop->p < 1.f), "gcn_fwd_split: need 0 <= edge_drop->p < 1");
+    SS_TRY(check_device());
+    AggArgs a{};
+    a.vbase = g->row_begin;
+    a.table = T_all; a.ld = ld; a.F = (int)F; a.bwd = 0;
+    a.rscale = dst_norm; a.gscale = 1.f;
+    a.H0 = H0_loc; a.alpha = alpha; a.bias = bias; a.act = act; a.Y = Y_loc; a.out_scale = out_scale; a.Ys = Ys_loc;
+    a.phase = phase; a.tloc = T_loc; a.ldloc = ldloc; a.part = part; a.ldp = ldp;
+    set_drop(a, edge_drop, g->fsplit.eid);
+    const bool vec4 = (ld % 4 == 0) && (ldp % 4 == 0) && aligned16(part) &&
+                      (phase == 2 ? aligned16(T_all) && aligned16(Y_loc) && (!H0_loc || aligned16(H0_loc)) &&
+                                        (!Ys_loc || aligned16(Ys_loc))
+                                  : (ldloc % 4 == 0) && aligned16(T_loc));
+    return launch_aggregate(g->fwd, a, vec4, to_stream(stream), &g->fsplit);
+}
+
+seastar_status seastar_gcn_bwd_split(seastar_graph g, int32_t phase, const float* dP_loc_in, int64_t ldloc,
+                                     const float* dP_all, int64_t F, int64_t ld, const float* src_norm, float scale,
+                                     const float* Yact_loc, seastar_act act, const float* post_scale, float* dA_loc,
+                                     float* dP_loc, float* part, int64_t ldp, const seastar_dropout_spec* edge_drop,
+                                     seastar_stream stream) {
+    SS_ARG(g != nullptr, "gcn_bwd_split: graph is NULL");
+    SS_ARG(g->partitioned, "gcn_bwd_split: the graph is not row-partitioned (use seastar_gcn_bwd)");
+    SS_ARG(phase == 1 || phase == 2, "gcn_bwd_split: phase must be 1 or 2");
+    SS_ARG(F >= 1 && ld >= F && ldp >= F, "gcn_bwd_split: bad sizes");
+    SS_ARG(part != nullptr, "gcn_bwd_split: part is NULL");
+    SS_ARG(phase == 2 || (dP_loc_in && ldloc >= F), "gcn_bwd_split: phase 1 needs dP_loc_in (ldloc >= F)");
+    SS_ARG(phase == 1 || (dP_all && (dA_loc || dP_loc)), "gcn_bwd_split: phase 2 needs dP_all and an output");
+    SS_ARG(act >= SEASTAR_ACT_NONE && act <= SEASTAR_ACT_SIGMOID, "gcn_bwd_split: bad activation %d", (int)act);
+    SS_ARG(!edge_drop || (edge_drop->p >= 0.f && edge_drop->p < 1.f), "gcn_bwd_split: need 0 <= edge_drop->p < 1");
+    SS_TRY(check_device());
+    AggArgs a{};
+    a.vbase = g->row_begin;
+    a.table = dP_all; a.ld = ld; a.F = (int)F; a.bwd = 1;
+    a.rscale = src_norm; a.gscale = scale;
+    a.Yact = Yact_loc; a.act = act; a.dA = dA_loc; a.post_scale = post_scale; a.dP = dP_loc;
+    a.phase = phase; a.tloc = dP_loc_in; a.ldloc = ldloc; a.part = part; a.ldp = ldp;
+    set_drop(a, edge_drop, g->rsplit.eid);
+    const bool vec4 = (ld % 4 == 0) && (ldp % 4 == 0) && aligned16(part) &&
+                      (phase == 2 ? aligned16(dP_all) && (!dA_loc || aligned16(dA_loc)) &&
+                                        (!dP_loc || aligned16(dP_loc)) && (!Yact_loc || aligned16(Yact_loc))
+                                  : (ldloc % 4 == 0) && aligned16(dP_loc_in));
+    return launch_aggregate(g->rev, a, vec4, to_stream(stream), &g->rsplit);
 }
 
 }  // extern "C"

@@ -361,6 +361,17 @@ __global__ void k_tm_tasks(int64_t bound, long long* __restrict__ meta, const in
     }
 }
 
+// ---- NEXT-1 local-first split: key = row << 1 | (neighbour not owned); owned-neighbour counts per row
+__global__ void k_split_keys(int64_t n, const int32_t* __restrict__ rowidx, const int32_t* __restrict__ nbr,
+                             int64_t rb, int64_t re, uint64_t* __restrict__ key, int32_t* __restrict__ lcnt) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const int64_t u = nbr[i];
+    const bool own = u >= rb && u < re;
+    key[i] = ((uint64_t)rowidx[i] << 1) | (own ? 0u : 1u);
+    if (own) atomicAdd(&lcnt[rowidx[i]], 1);   // integer count per row: order-independent
+}
+
 // ---- two-phase R-GCN edge-major views: the type of every type-major edge (from its sort key)
 __global__ void k_em_type(int64_t n, const uint64_t* __restrict__ key, int rbits, int32_t* __restrict__ type) {
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -561,6 +572,12 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
         want(&g->rev.norm, Er, want_norm);
         want(&g->lsf.off, N + 1, part);
         want(&g->lsf.eid, Er, part);
+        want(&g->fsplit.nbr, Ef, part);
+        want(&g->fsplit.eid, Ef, part);
+        want(&g->fsplit.lcnt, n_loc, part);
+        want(&g->rsplit.nbr, Er, part);
+        want(&g->rsplit.eid, Er, part);
+        want(&g->rsplit.lcnt, n_loc, part);
         want(&g->indeg_loc, n_loc, true);
         want(&g->outdeg_loc, n_loc, true);
         const bool tm_on = etypes != nullptr && Ef > 0;
@@ -794,6 +811,33 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
             k_em_type<<<grid_for(Er, 256), 256, 0, s>>>(Er, k1, rbits, g->rem.type);
             CK(cudaMemcpyAsync(g->rem.pos, pos, sizeof(int32_t) * Er, cudaMemcpyDeviceToDevice, s));
             CKS_LAUNCH("k_em_type(rev)");
+        }
+
+        // ---- NEXT-1: local-first splits of FWD and REV (partitioned graphs) -------------------------
+        if (part && n_loc > 0) {
+            const int rbits1 = bit_width((uint64_t)n_loc) + 1;
+            auto split = [&](const IndexSet& x, LocalSplit& sp) -> seastar_status {
+                const int64_t ne = x.n_edges;
+                SS_CUDA(cudaMemsetAsync(sp.lcnt, 0, sizeof(int32_t) * n_loc, s));
+                if (ne == 0) return SEASTAR_OK;
+                int32_t *rowidx, *iota, *perm;
+                uint64_t *k0, *k1;
+                SS_CUDA(t.alloc(&rowidx, ne));
+                SS_CUDA(t.alloc(&iota, ne));
+                SS_CUDA(t.alloc(&perm, ne));
+                SS_CUDA(t.alloc(&k0, ne));
+                SS_CUDA(t.alloc(&k1, ne));
+                k_row_index<<<8 * num_sms(), 256, 0, s>>>(n_loc, x.off, rowidx);
+                k_split_keys<<<grid_for(ne, 256), 256, 0, s>>>(ne, rowidx, x.nbr, row_begin, row_end, k0, sp.lcnt);
+                k_iota<<<grid_for(ne, 256), 256, 0, s>>>(ne, iota);
+                SS_TRY(check_launch("k_split_keys"));
+                SS_TRY(radix_sort_pairs<uint64_t>(t, k0, k1, iota, perm, ne, rbits1));
+                k_gather_i32<<<grid_for(ne, 256), 256, 0, s>>>(ne, perm, x.nbr, sp.nbr);
+                k_gather_i32<<<grid_for(ne, 256), 256, 0, s>>>(ne, perm, x.eid, sp.eid);
+                return check_launch("k_gather(split)");
+            };
+            CKS(split(g->fwd, g->fsplit));
+            CKS(split(g->rev, g->rsplit));
         }
 
         // ---- a3: degree buckets (second and last sync) --------------------------------------------

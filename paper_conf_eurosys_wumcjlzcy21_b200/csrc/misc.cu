@@ -3,6 +3,8 @@
 // and a flat-buffer Adam step (DGL's default training loop).
 #include <math.h>
 
+#include <algorithm>
+
 #include "common.cuh"
 #include <cmath>
 
@@ -397,6 +399,34 @@ seastar_status seastar_softmax_xent(const float* Z, int64_t M, int64_t n_total, 
     }
     k_loss_final<<<1, 256, 0, s>>>(part, nblk, n_total, loss);
     return check_launch("k_softmax_xent");
+}
+
+}  // extern "C"
+
+namespace seastar {
+__global__ void k_row_scale(const float* __restrict__ X, int64_t M, int64_t F, int64_t ldx,
+                            const float* __restrict__ scale, float* Y, int64_t ldy) {
+    const int64_t n = M * F;
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = k / F, j = k % F;
+        Y[i * ldy + j] = __ldg(scale + i) * X[i * ldx + j];
+    }
+}
+}  // namespace seastar
+
+extern "C" {
+
+seastar_status seastar_row_scale(const float* X, int64_t M, int64_t F, int64_t ldx, const float* scale, float* Y,
+                                 int64_t ldy, seastar_stream stream) {
+    SS_ARG(X && scale && Y, "row_scale: NULL argument");
+    SS_ARG(M >= 0 && F >= 1 && ldx >= F && ldy >= F, "row_scale: bad sizes");
+    SS_ARG((void*)X != (void*)Y || ldx == ldy, "row_scale: in-place needs ldx == ldy");
+    SS_TRY(check_device());
+    if (M == 0) return SEASTAR_OK;
+    const int64_t n = M * F;
+    const int64_t blocks = std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 16);
+    k_row_scale<<<(unsigned)blocks, 256, 0, to_stream(stream)>>>(X, M, F, ldx, scale, Y, ldy);
+    return check_launch("k_row_scale");
 }
 
 seastar_status seastar_axpby(int64_t n, float a, const float* x, float b, float* y, seastar_stream stream) {

@@ -69,16 +69,20 @@ class Comm:
             torch.distributed.all_gather_into_tensor(out_all, loc, group=self.group)
         return out_all
 
-    def reduce_scatter(self, out_loc: torch.Tensor, part_all: torch.Tensor):
-        if self.world == 1:
-            return part_all
-        if self.staged:
-            h = part_all.cpu()
-            torch.distributed.all_reduce(h, group=self.group)
-            out_loc.copy_(h.view(self.world, *out_loc.shape)[self.rank])
-        else:
-            torch.distributed.reduce_scatter_tensor(out_loc, part_all, group=self.group)
-        return out_loc
+    class _Done:
+        def wait(self):
+            return None
+
+    def all_gather_async(self, out_all: torch.Tensor, loc: torch.Tensor):
+        """NEXT-1: start the all-gather and return a handle whose wait() makes the current stream wait for it; the
+        caller launches the owned-neighbour phase of the aggregation in between (NCCL runs on its own stream).
+        The staged gloo path is synchronous (the handle is already complete)."""
+        if self.world == 1 or self.staged:
+            self.all_gather(out_all, loc)
+            return Comm._Done()
+        loc = self._rows(loc)
+        assert out_all.is_contiguous() and out_all.numel() == loc.numel() * self.world, (out_all.shape, loc.shape)
+        return torch.distributed.all_gather_into_tensor(out_all, loc, group=self.group, async_op=True)
 
     def all_reduce(self, flat: torch.Tensor):
         if self.world > 1:
@@ -151,7 +155,8 @@ class GCN2:
     next-layer norm into the backward aggregation's epilogue."""
 
     def __init__(self, g: Graph, X_loc: torch.Tensor, labels_loc: torch.Tensor, params: dict, lr=0.01,
-                 comm: Comm | None = None, n_pad_rows: int | None = None, dropout: float = 0.0, seed: int = 0):
+                 comm: Comm | None = None, n_pad_rows: int | None = None, dropout: float = 0.0, seed: int = 0,
+                 overlap: bool | None = None):
         self.g, self.X, self.lab, self.lr = g, X_loc, labels_loc, lr
         self.drop_p, self.drop_seed = float(dropout), int(seed)     # NEXT-3: dropout on the hidden layer (DGL: 0.5)
         self.comm = comm or Comm()
@@ -185,7 +190,37 @@ class GCN2:
         self.H1s_all = e(self.rows_all, H) if P > 1 else None
         self.dP2_all = e(self.rows_all, H) if P > 1 else None
         self.dP1_all = e(self.rows_all, H) if P > 1 else None
+        # NEXT-1: partitioned aggregations in two phases around each all-gather (owned-neighbour edges first)
+        self.overlap = (P > 1) if overlap is None else (bool(overlap) and P > 1)
+        self.part = e(n, H) if self.overlap else None
         self.timer = None
+
+    def _agg_fwd(self, loc, tab_all_buf, dst_norm, bias, act, out, out_scale=None, outs=None):
+        """forward aggregation of the gathered `loc` rows (one phase, or NEXT-1's two phases around the gather)"""
+        g, H = self.g, self.H
+        if not self.overlap:
+            tab = self.comm.all_gather(tab_all_buf, loc)
+            L.seastar_gcn_fwd(g.handle, tab, H, H, dst_norm, bias, act, 0.0, None, out, out_scale, outs)
+            return
+        h = self.comm.all_gather_async(tab_all_buf, loc)
+        L.seastar_gcn_fwd_split(g.handle, 1, loc, H, None, H, H, None, None, "none", 0.0, None, None, None, None,
+                                self.part, H)
+        h.wait()
+        L.seastar_gcn_fwd_split(g.handle, 2, None, 0, tab_all_buf, H, H, dst_norm, bias, act, 0.0, None, out,
+                                out_scale, outs, self.part, H)
+
+    def _agg_bwd(self, loc, tab_all_buf, Yact, act, post_scale, dA, dP):
+        g, H = self.g, self.H
+        if not self.overlap:
+            tab = self.comm.all_gather(tab_all_buf, loc)
+            L.seastar_gcn_bwd(g.handle, tab, H, H, self.src_n, 1.0, Yact, act, post_scale, dA, dP)
+            return
+        h = self.comm.all_gather_async(tab_all_buf, loc)
+        L.seastar_gcn_bwd_split(g.handle, 1, loc, H, None, H, H, None, 1.0, None, "none", None, None, None,
+                                self.part, H)
+        h.wait()
+        L.seastar_gcn_bwd_split(g.handle, 2, None, 0, tab_all_buf, H, H, self.src_n, 1.0, Yact, act, post_scale, dA,
+                                dP, self.part, H)
 
     def _t(self, name):
         if self.timer is not None:
@@ -195,15 +230,12 @@ class GCN2:
         g, p, H, C, n = self.g, self.P, self.H, self.C, self.n
         _linear(self.ws, self.X, n, self.Fin, self.X.stride(0), p.p("W1"), H, None, self.src_n, "none",
                              self.T1, H)
-        T1_all = self.comm.all_gather(self.T1_all, self.T1)
         self._t("gcn_fwd1")
-        L.seastar_gcn_fwd(g.handle, T1_all, H, H, self.dst_n, p.p("b1"), "relu", 0.0, None, self.H1, self.src_n,
-                          self.H1s)
+        self._agg_fwd(self.T1, self.T1_all, self.dst_n, p.p("b1"), "relu", self.H1, self.src_n, self.H1s)
         self._t("gcn_fwd1_end")
         if self.drop_p > 0:      # layer-2 input src_n * drop(H1): the mask commutes with the row scale
             L.seastar_dropout(self.H1s, n, H, H, g.row_begin, self.drop_p, self.drop_seed, 1, p.step, self.H1s, H)
-        H1s_all = self.comm.all_gather(self.H1s_all, self.H1s)
-        L.seastar_gcn_fwd(g.handle, H1s_all, H, H, self.dst_n, None, "none", 0.0, None, self.P2)
+        self._agg_fwd(self.H1s, self.H1s_all, self.dst_n, None, "none", self.P2)
         _linear(self.ws, self.P2, n, H, H, p.p("W2"), C, p.p("b2"), None, "none", self.logits, self.ldc)
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
         L.seastar_softmax_xent(self.logits, n, self.g.N, C, self.ldc, self.lab, self.loss, self.dlogits, self.ldc,
@@ -218,16 +250,14 @@ class GCN2:
         L.seastar_linear_bwd_weight(self.P2, n, H, H, self.dlogits, C, self.ldc, p.g("W2"), p.g("b2"), ws,
                                     ws.numel())
         L.seastar_linear_bwd_data(self.dlogits, n, C, self.ldc, p.p("W2"), H, self.dst_n, None, "none", self.dP2, H)
-        dP2_all = self.comm.all_gather(self.dP2_all, self.dP2)
         self._t("gcn_bwd2")
-        L.seastar_gcn_bwd(g.handle, dP2_all, H, H, self.src_n, 1.0, self.H1, "relu", self.dst_n, self.dA1, self.dP1)
+        self._agg_bwd(self.dP2, self.dP2_all, self.H1, "relu", self.dst_n, self.dA1, self.dP1)
         self._t("gcn_bwd2_end")
         if self.drop_p > 0:      # d drop(H1) -> dH1: the same mask, commuting with relu' and the dst_n scale
             for t in (self.dA1, self.dP1):
                 L.seastar_dropout(t, n, H, H, g.row_begin, self.drop_p, self.drop_seed, 1, p.step, t, H)
         L.seastar_colsum(self.dA1, n, H, H, p.g("b1"), ws, ws.numel())
-        dP1_all = self.comm.all_gather(self.dP1_all, self.dP1)
-        L.seastar_gcn_bwd(g.handle, dP1_all, H, H, self.src_n, 1.0, None, "none", None, self.dT1, None)
+        self._agg_bwd(self.dP1, self.dP1_all, None, "none", None, self.dT1, None)
         L.seastar_linear_bwd_weight(self.X, n, self.Fin, self.X.stride(0), self.dT1, H, H, p.g("W1"), None, ws,
                                     ws.numel())
         self.comm.all_reduce(self.P.grad)
@@ -392,7 +422,7 @@ class APPNPNet:
     Each propagation step is one fused gcn_fwd (APPNP epilogue, writes Z and n*Z for the next step)."""
 
     def __init__(self, g: Graph, X_loc, labels_loc, params: dict, K=10, alpha=0.1, lr=0.01, comm: Comm | None = None,
-                 n_pad_rows: int | None = None, edge_dropout: float = 0.0, seed: int = 0):
+                 n_pad_rows: int | None = None, edge_dropout: float = 0.0, seed: int = 0, overlap: bool | None = None):
         self.g, self.X, self.lab, self.K, self.alpha, self.lr = g, X_loc, labels_loc, K, alpha, lr
         self.comm = comm or Comm()
         dev = X_loc.device
@@ -423,6 +453,9 @@ class APPNPNet:
         P = self.comm.world
         self.Zs_all = e(self.rows_all, self.ldc) if P > 1 else None
         self.Gs_all = e(self.rows_all, self.ldc) if P > 1 else None
+        # NEXT-1: each propagation step's aggregation in two phases around its all-gather (see GCN2)
+        self.overlap = (P > 1) if overlap is None else (bool(overlap) and P > 1)
+        self.part = e(n, self.ldc) if self.overlap else None
         self.timer = None
 
     def _t(self, name):
@@ -434,12 +467,21 @@ class APPNPNet:
         _linear(self.ws, self.X, n, self.Fin, self.X.stride(0), p.p("W1"), Hd, p.p("b1"), None, "relu", self.Hh,
                              Hd)
         _linear(self.ws, self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), None, "none", self.H0, ld)
-        _linear(self.ws, self.Hh, n, Hd, Hd, p.p("W2"), C, p.p("b2"), self.nrm, "none", self.Zs[0], ld)
+        L.seastar_row_scale(self.H0, n, C, ld, self.nrm, self.Zs[0], ld)           # Z^0 = H0, pre-scaled by n
         for k in range(self.K):
-            Zs_all = self.comm.all_gather(self.Zs_all, self.Zs[k])
             self._t("appnp_fwd") if k == 0 else None
-            L.seastar_gcn_fwd(g.handle, Zs_all, C, ld, self.nrm, None, "none", self.alpha, self.H0, self.Z[k + 1],
-                              self.nrm, self.Zs[k + 1], edge_drop=self.ed[k])
+            if self.overlap:
+                h = self.comm.all_gather_async(self.Zs_all, self.Zs[k])
+                L.seastar_gcn_fwd_split(g.handle, 1, self.Zs[k], ld, None, C, ld, None, None, "none", 0.0, None, None,
+                                        None, None, self.part, ld, edge_drop=self.ed[k])
+                h.wait()
+                L.seastar_gcn_fwd_split(g.handle, 2, None, 0, self.Zs_all, C, ld, self.nrm, None, "none", self.alpha,
+                                        self.H0, self.Z[k + 1], self.nrm, self.Zs[k + 1], self.part, ld,
+                                        edge_drop=self.ed[k])
+            else:
+                Zs_all = self.comm.all_gather(self.Zs_all, self.Zs[k])
+                L.seastar_gcn_fwd(g.handle, Zs_all, C, ld, self.nrm, None, "none", self.alpha, self.H0, self.Z[k + 1],
+                                  self.nrm, self.Zs[k + 1], edge_drop=self.ed[k])
             self._t("appnp_fwd_end") if k == 0 else None
         out = self.Z[self.K] if self.K > 0 else self.H0
         ws = self.ws.need(L.seastar_softmax_xent_workspace(n))
@@ -450,17 +492,26 @@ class APPNPNet:
         g, p, n, Hd, C, ld, a = self.g, self.P, self.n, self.Hd, self.C, self.ldc, self.alpha
         # G = dL/dZ^K ; for k = K-1..0: dH0 += a G ; G <- (1-a) n sum_out n G
         self.dH0.zero_()
-        _linear(self.ws, self.G, n, C, ld, self._eye(C), C, None, self.nrm, "none", self.Gs[0], ld) \
-            if self.K > 0 else None
+        if self.K > 0:
+            L.seastar_row_scale(self.G, n, C, ld, self.nrm, self.Gs[0], ld)
         cur = 0
         G = self.G
         for k in range(self.K):
             L.seastar_axpby(n * ld, a, G, 1.0, self.dH0)
-            Gs_all = self.comm.all_gather(self.Gs_all, self.Gs[cur])
             nxt = self.Gtmp if G is self.G else self.G
             self._t("appnp_bwd") if k == 0 else None
-            L.seastar_gcn_bwd(g.handle, Gs_all, C, ld, self.nrm, 1.0 - a, None, "none", self.nrm, nxt, self.Gs[1 - cur],
-                              edge_drop=self.ed[self.K - 1 - k])
+            ed = self.ed[self.K - 1 - k]
+            if self.overlap:
+                h = self.comm.all_gather_async(self.Gs_all, self.Gs[cur])
+                L.seastar_gcn_bwd_split(g.handle, 1, self.Gs[cur], ld, None, C, ld, None, 1.0, None, "none", None, None,
+                                        None, self.part, ld, edge_drop=ed)
+                h.wait()
+                L.seastar_gcn_bwd_split(g.handle, 2, None, 0, self.Gs_all, C, ld, self.nrm, 1.0 - a, None, "none",
+                                        self.nrm, nxt, self.Gs[1 - cur], self.part, ld, edge_drop=ed)
+            else:
+                Gs_all = self.comm.all_gather(self.Gs_all, self.Gs[cur])
+                L.seastar_gcn_bwd(g.handle, Gs_all, C, ld, self.nrm, 1.0 - a, None, "none", self.nrm, nxt,
+                                  self.Gs[1 - cur], edge_drop=ed)
             self._t("appnp_bwd_end") if k == 0 else None
             G = nxt
             cur = 1 - cur
@@ -472,11 +523,6 @@ class APPNPNet:
         L.seastar_linear_bwd_weight(self.X, n, self.Fin, self.X.stride(0), self.dHh, Hd, Hd, p.g("W1"), p.g("b1"), ws,
                                     ws.numel())
         self.comm.all_reduce(self.P.grad)
-
-    def _eye(self, C):
-        if not hasattr(self, "_I") or self._I.shape[0] != C:
-            self._I = torch.eye(C, device=self.X.device)
-        return self._I
 
     def epoch(self):
         loss = self.forward()

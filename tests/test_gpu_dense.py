@@ -159,3 +159,19 @@ def test_linear_bwd_weight_tcgen05(env, M, K, N):
                                 ws_b)
     _, rdW2, _ = oracle.linear_bwd(X2, np.zeros((K, N), np.float32), dY)
     assert rel_err(dW.cpu().numpy(), rdW2) <= TOL
+
+
+def test_row_scale():
+    """seastar_row_scale (APPNP's n (.) pre-scaling): Y[i] = s[i] X[i], strided and in place."""
+    import torch
+    from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
+    import synth
+    M, F, ld = 1000, 5, 8
+    X = synth.uniform(1, (M, ld))
+    s = synth.uniform(2, (M,), 0.1, 2.0)
+    Xd, sd = torch.from_numpy(X).cuda(), torch.from_numpy(s).cuda()
+    Y = torch.full((M, ld), float("nan"), device="cuda")
+    L.seastar_row_scale(Xd, M, F, ld, sd, Y, ld)
+    np.testing.assert_array_equal(Y.cpu().numpy()[:, :F], (s[:, None] * X[:, :F]).astype(np.float32))
+    L.seastar_row_scale(Xd, M, F, ld, sd, Xd, ld)
+    np.testing.assert_array_equal(Xd.cpu().numpy()[:, :F], Y.cpu().numpy()[:, :F])

@@ -35,6 +35,15 @@ class ThreadComm:
         out_all.copy_(torch.cat(self._exchange(loc), 0))
         return out_all
 
+    def all_gather_async(self, out_all, loc):
+        """NEXT-1 interface: the lockstep exchange completes here; the handle's wait() is a no-op"""
+        self.all_gather(out_all, loc)
+
+        class _Done:
+            def wait(self):
+                return None
+        return _Done()
+
     def reduce_scatter(self, out_loc, part_all):
         raise AssertionError("the partitioned models never reduce-scatter")
 
@@ -81,8 +90,10 @@ def grads_of(model, keys):
     return {k: model.P.g(k).cpu().numpy().copy() for k in keys}
 
 
-@pytest.mark.parametrize("P", [2, 3])
-def test_gcn_gat_partitioned(env, P):
+@pytest.mark.parametrize("P,overlap", [(2, True), (3, True), (2, False)])
+def test_gcn_gat_partitioned(env, P, overlap):
+    """overlap: GCN2's aggregations run NEXT-1's two phases (owned-neighbour edges from the rank's own rows, then
+    the rest from the gathered table) -- the default when partitioned -- or one phase after the gather."""
     torch, models, part, Graph = env["torch"], env["models"], env["part"], env["Graph"]
     N, Fin = 3001, 120
     ip, ix = synth.powerlaw_sym(N, 30000, 0.5, 51)
@@ -102,7 +113,7 @@ def test_gcn_gat_partitioned(env, P):
         g = Graph(ip, ix, row_begin=rb, row_end=re)
         Xl = torch.from_numpy(X[rb:re]).cuda()
         mg = models.GCN2(g, Xl, torch.from_numpy(lab7[rb:re]).cuda(), pg, comm=comm,
-                         n_pad_rows=part.gathered_rows(N, P))
+                         n_pad_rows=part.gathered_rows(N, P), overlap=overlap)
         lg = mg.forward().item()
         mg.backward()
         ma = models.GAT2(g, Xl, torch.from_numpy(lab5[rb:re]).cuda(), pa, heads, hid, comm=comm,
@@ -182,3 +193,35 @@ def test_rgcnb_partitioned(env, P):
         else:
             got = res[0][1][k]
         assert rel_err(got, rg[k].reshape(got.shape)) <= TOL, k
+
+
+@pytest.mark.parametrize("overlap,edge_p", [(True, 0.0), (False, 0.0), (True, 0.2)])
+def test_appnp_partitioned(env, overlap, edge_p):
+    """APPNP row-partitioned over P = 2 ranks: every propagation step's aggregation (forward and backward) in NEXT-1's
+    two phases around its all-gather, or one phase; with and without edge dropout (masks keyed by user edge id)."""
+    torch, models, part, Graph = env["torch"], env["models"], env["part"], env["Graph"]
+    P, N, Fin, Hd, C, K = 2, 1601, 40, 16, 5, 4
+    ip, ix = synth.powerlaw_sym(N, 12000, 0.5, 61)
+    X, lab = synth.uniform(44, (N, Fin)), synth.labels(45, N, C)
+    p = {"W1": synth.glorot(46, Fin, Hd), "b1": synth.uniform(47, (Hd,), -0.1, 0.1),
+         "W2": synth.glorot(48, Hd, C), "b2": synth.uniform(49, (C,), -0.1, 0.1)}
+
+    def build(r, comm):
+        torch.cuda.set_device(0)
+        rb, re = part.row_range(N, P, r)
+        g = Graph(ip, ix, row_begin=rb, row_end=re)
+        m = models.APPNPNet(g, torch.from_numpy(X[rb:re]).cuda(), torch.from_numpy(lab[rb:re]).cuda(), p, K=K,
+                            alpha=0.1, comm=comm, n_pad_rows=part.gathered_rows(N, P), overlap=overlap,
+                            edge_dropout=edge_p, seed=9)
+        assert m.overlap == overlap
+        l = m.forward().item()
+        m.backward()
+        torch.cuda.synchronize()
+        return l, grads_of(m, p)
+
+    res = run_ranks(P, build)
+    drop = {"edge_p": edge_p, "seed": 9, "step": 0} if edge_p else None
+    rl, rg = model_ref.appnp(ip, ix, X, lab, {k: v.astype(np.float64) for k, v in p.items()}, K, 0.1, drop=drop)
+    assert abs(sum(r[0] for r in res) - rl) <= TOL * abs(rl)
+    for k in rg:
+        assert rel_err(res[0][1][k], rg[k].reshape(res[0][1][k].shape)) <= TOL, k
