@@ -1,6 +1,7 @@
 // common.cuh -- shared internals of libseastar.so (sm_100a).  Not part of the ABI.
 #pragma once
 #include <cmath>
+#include <cstdlib>
 
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -277,14 +278,22 @@ inline int num_sms() {
     return sms;
 }
 
-// "Long" rows of a row launch: a row whose edges exceed a quarter of one SM's share of the index set would keep
-// one warp busy past the rest of the launch (CoraFull-shaped: ~250 edges), so it gets a CTA of 8 warps (PAPER.md
-// L1253 CTA + Warp; the a3 hub class, made relative to the launch).  Returns the number of leading (highest-degree)
-// rows that qualify: rows with degree >= the power of two at or above max(E / (4 * #SMs), 128).
+// "Long" rows of a row launch get a CTA of 8 warps in the same launch as the warp rows (PAPER.md L1253 CTA + Warp):
+// every row whose edges exceed a quarter of one SM's share of the index set, which would keep one warp busy past
+// the rest of the launch (CoraFull-shaped: ~250 edges).  Returns the number of leading (highest-degree) rows that
+// qualify: degree >= the power of two at or above max(E / (4 #SMs), 128).  On the Reddit shape no row qualifies;
+// giving its a3 hub class (degree >= 1024) CTAs was measured slower in the product kernels (r2 same-box A/B,
+// profiles/r2/ab_long_rows.txt: GCN aggregation 0.68 -> 0.82 ms) although the NEXT-4 sweep's plain-sum kernel gains
+// (profiles/r2/ablation.md).  SEASTAR_LONG_ROW=<degree> overrides the threshold (A/B runs; 0 disables).
 inline int64_t long_rows(const IndexSet& x) {
-    const int64_t t = x.n_edges / (4 * (int64_t)num_sms());
+    int64_t t = x.n_edges / (4 * (int64_t)num_sms());
+    t = t > 128 ? t : 128;
+    if (const char* env = getenv("SEASTAR_LONG_ROW")) {
+        t = atoll(env);
+        if (t <= 0) return 0;
+    }
     int k = 0;
-    while (k < kPow2Classes && ((int64_t)1 << (kPow2Lo + k)) < (t > 128 ? t : 128)) ++k;
+    while (k < kPow2Classes && ((int64_t)1 << (kPow2Lo + k)) < t) ++k;
     return k < kPow2Classes ? x.pow2_rows[k] : 0;
 }
 

@@ -62,7 +62,9 @@ struct AggArgs {
 // edges, and the warps' partial sums are added in warp order through shared memory before warp 0 runs the epilogue
 // (deterministic) -- and every later block owns 8 rows, a warp each ("CTA + Warp").  One
 // launch for both classes: a separate hub launch cost more (kernel boundary) than it saved on the Reddit shape.
-template <int VEC, int L, int RL, int NB, bool DROP = false, int WPR = 1>
+// PH: NEXT-1 split phase (0: whole rows; 1 / 2: see AggArgs) as a template parameter -- a runtime phase cost the
+// whole-row kernel 14 registers (48 -> 62) and its occupancy (r2 sweep: 0.67 -> 0.81 ms at F = 16 on Reddit)
+template <int VEC, int L, int RL, int NB, bool DROP = false, int WPR = 1, int PH = 0>
 __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
     static_assert(WPR == 1 || RL == 32, "hub rows take whole warps");
     constexpr int S = RL / L;                    // edge slots per row group
@@ -85,12 +87,12 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
     const bool valid = row < a.row_end;
     int beg = valid ? __ldg(a.off + row) : 0;
     int end = valid ? __ldg(a.off + row + 1) : 0;
-    if (a.phase && valid) {                      // NEXT-1: owned-neighbour edges lead every split row
+    if (PH != 0 && valid) {                      // NEXT-1: owned-neighbour edges lead every split row
         const int lc = __ldg(a.lcnt + row);
-        if (a.phase == 1) end = beg + lc; else beg += lc;
+        if (PH == 1) end = beg + lc; else beg += lc;
     }
-    const float* tab = a.phase == 1 ? a.tloc - a.vbase * a.ldloc : a.table;   // phase 1: the rank's own rows
-    const int64_t tld = a.phase == 1 ? a.ldloc : a.ld;
+    const float* tab = PH == 1 ? a.tloc - a.vbase * a.ldloc : a.table;   // phase 1: the rank's own rows
+    const int64_t tld = PH == 1 ? a.ldloc : a.ld;
     if (hubblk) {
         const int64_t len = end - beg;
         const int b0 = beg + (int)(len * wib / WPR);
@@ -179,13 +181,13 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
         }
 
         if (!valid || slot != 0 || !active) continue;
-        if (a.phase == 1) {                          // partial row sum, finished by phase 2
+        if (PH == 1) {                               // partial row sum, finished by phase 2
             float* pp = a.part + v * a.ldp + col;
             if (col + VEC <= a.F) store_vec<VEC>(pp, acc);
             else for (int i = 0; i < VEC && col + i < a.F; ++i) pp[i] = acc[i];
             continue;
         }
-        if (a.phase == 2) {
+        if (PH == 2) {
             const float* pp = a.part + v * a.ldp + col;
 #pragma unroll
             for (int i = 0; i < VEC; ++i)
@@ -244,8 +246,8 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
 
 constexpr int kHubWarps = 8;       // warps per hub row (degree >= 1024: >= 128 edges per warp)
 
-template <int VEC, int L>
-static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s, bool hub = false) {
+template <int VEC, int L, int PH>
+static void launch_rl_ph(AggArgs a, bool warp_rows, cudaStream_t s, bool hub) {
     const int64_t rows = a.row_end - a.row_begin;
     if (rows <= 0) return;
     constexpr int threads = 256;
@@ -253,8 +255,8 @@ static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s, bool hub = fals
         static_assert(32 * kHubWarps == threads, "hub CTAs are the launch's 256-thread blocks");
         constexpr int NBW = L >= 4 ? 1 : 4 / L;
         const unsigned grid = (unsigned)(a.nlong + (rows - a.nlong + kHubWarps - 1) / kHubWarps);
-        if (a.deid) launch_k(k_aggregate<VEC, L, 32, NBW, true, kHubWarps>, dim3(grid), dim3(threads), 0, s, a);
-        else launch_k(k_aggregate<VEC, L, 32, NBW, false, kHubWarps>, dim3(grid), dim3(threads), 0, s, a);
+        if (a.deid) launch_k(k_aggregate<VEC, L, 32, NBW, true, kHubWarps, PH>, dim3(grid), dim3(threads), 0, s, a);
+        else launch_k(k_aggregate<VEC, L, 32, NBW, false, kHubWarps, PH>, dim3(grid), dim3(threads), 0, s, a);
         return;
     }
     if (warp_rows) {
@@ -264,14 +266,23 @@ static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s, bool hub = fals
         // narrow rows (L < 4 chunk lanes, F <= 8) take 4/L index chunks per iteration so every lane still has
         // 4 gathers in flight: F = 8 0.75 -> 0.50 ms, F = 1..4 0.54 -> 0.46 ms on Reddit (tools/ab_gcn.sh)
         constexpr int NBW = L >= 4 ? 1 : 4 / L;
-        if (a.deid) launch_k(k_aggregate<VEC, L, 32, NBW, true>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
-        else launch_k(k_aggregate<VEC, L, 32, NBW>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        if (a.deid) launch_k(k_aggregate<VEC, L, 32, NBW, true, 1, PH>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        else launch_k(k_aggregate<VEC, L, 32, NBW, false, 1, PH>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
     } else {
         constexpr int RL = L < 4 ? 4 : L;   // at least 4 lanes per row group keeps index loads useful
         const int64_t per_block = threads / RL;
         const int64_t blocks = (rows + per_block - 1) / per_block;
-        if (a.deid) launch_k(k_aggregate<VEC, L, RL, 1, true>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
-        else launch_k(k_aggregate<VEC, L, RL, 1>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        if (a.deid) launch_k(k_aggregate<VEC, L, RL, 1, true, 1, PH>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+        else launch_k(k_aggregate<VEC, L, RL, 1, false, 1, PH>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
+    }
+}
+
+template <int VEC, int L>
+static void launch_rl(AggArgs a, bool warp_rows, cudaStream_t s, bool hub = false) {
+    switch (a.phase) {
+        case 1: launch_rl_ph<VEC, L, 1>(a, warp_rows, s, hub); break;
+        case 2: launch_rl_ph<VEC, L, 2>(a, warp_rows, s, hub); break;
+        default: launch_rl_ph<VEC, L, 0>(a, warp_rows, s, hub); break;
     }
 }
 

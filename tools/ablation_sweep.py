@@ -10,7 +10,17 @@ rep) for
   fa_unsorted the same kernel on the user's (unsorted) vertex order;
   basic       one thread per row (edges and features sequential), the paper's "Basic";
   edge_atomic one thread per (edge, feature) with a binary search of the destination and atomicAdd
-              (DGL/minigun's strategy, L397-L399).
+              (DGL/minigun's strategy, L397-L399);
+  (r2, F a power of two in 4..128)
+  slot_over   the product's lane mapping (edge slots, 4 gathers in flight per lane) with one warp per row on an
+              oversubscribed grid (the block scheduler balances);
+  slot_pers   the same with a persistent grid (148 x 8 blocks, warps stride over the rows: "persistent threads",
+              L437);
+  slot_dyn    persistent, rows claimed from an atomic counter;
+  slot_hub    oversubscribed, and the rows of degree >= 1024 get a CTA of 8 warps (contiguous slices, warp-order
+              merge) in the same launch (CTA + Warp, L1253);
+  tma_g4      TMA tile::gather4: one lane per warp gathers 4 neighbour rows per cp.async.bulk.tensor into an
+              8-stage shared-memory ring (mbarrier complete_tx), the warp sums them from shared memory.
 Every variant's output is checked against the product kernel's (max-abs-normalised error <= 1e-5).
 Writes gpurun_out/ablation.json and prints a markdown table.  Not product code."""
 import ctypes
@@ -42,6 +52,8 @@ def lib():
     so.abl_basic.argtypes = [I, P, P, P, ctypes.c_int, I, P, P]
     so.abl_edge_atomic.argtypes = [I, I, P, P, P, ctypes.c_int, I, P, P]
     so.abl_fa.argtypes = [I, P, P, P, P, ctypes.c_int, I, P, P]
+    so.abl_slot.argtypes = [I, P, P, P, P, ctypes.c_int, I, P, ctypes.c_int, I, P, P]
+    so.abl_tma.argtypes = [I, P, P, P, P, ctypes.c_int, I, P, P]
     return so
 
 
@@ -73,6 +85,8 @@ def main():
     ip32 = torch.from_numpy(ip.astype(np.int32)).cuda()
     ix32 = torch.from_numpy(ix.astype(np.int32)).cuda()
     flush = torch.empty(64 * 1024 * 1024, device="cuda")
+    counter = torch.zeros(1, dtype=torch.int32, device="cuda")
+    nhub = g.info["fwd_bucket_rows"][0]
     s = torch.cuda.current_stream().cuda_stream
     Fs = [int(a) for a in sys.argv[1:]] or [1, 2, 4, 8, 16, 32, 64, 128, 256, 602]
     rows = []
@@ -91,11 +105,21 @@ def main():
             "edge_atomic": lambda: so.abl_edge_atomic(N, E, ip32.data_ptr(), ix32.data_ptr(), X.data_ptr(), F, ld,
                                                       Y.data_ptr(), s),
         }
+        if F in (4, 8, 16, 32, 64, 128):
+            fp = (fwd["perm"].data_ptr(), fwd["off"].data_ptr(), fwd["nbr"].data_ptr(), X.data_ptr(), F, ld,
+                  Y.data_ptr())
+            runs["slot_over"] = lambda: so.abl_slot(N, *fp, 0, 0, counter.data_ptr(), s)
+            runs["slot_pers"] = lambda: so.abl_slot(N, *fp, 1, 0, counter.data_ptr(), s)
+            runs["slot_dyn"] = lambda: so.abl_slot(N, *fp, 2, 0, counter.data_ptr(), s)
+            runs["slot_hub"] = lambda: so.abl_slot(N, *fp, 0, nhub, counter.data_ptr(), s)
+            runs["tma_g4"] = lambda: so.abl_tma(N, *fp, s)
         L.seastar_gcn_fwd(g.handle, X, F, ld, None, None, "none", 0.0, None, Y0, None, None)
         ref = Y0[:, :F].double()
         den = ref.abs().max().item()
         row = {"F": F}
         for name, fn in runs.items():
+            rc = fn()
+            assert not rc, (name, F, rc)
             ms = timed(fn, flush, 5)
             err = ((Y[:, :F].double() - ref).abs().max().item() / den) if name != "seastar" else 0.0
             assert err <= 1e-5, (name, F, err)
@@ -107,11 +131,12 @@ def main():
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     json.dump({"graph": {"N": N, "E": E}, "rows": rows}, open(os.path.join(ROOT, "gpurun_out", "ablation.json"), "w"),
               indent=1)
-    names = ["seastar", "fa_sorted", "fa_unsorted", "basic", "edge_atomic"]
+    names = ["seastar", "fa_sorted", "fa_unsorted", "basic", "edge_atomic", "slot_over", "slot_pers", "slot_dyn",
+             "slot_hub", "tma_g4"]
     print("| F | " + " | ".join(f"{n} ms" for n in names) + " | seastar G edges/s | seastar alg. GB/s |")
     print("|---" * (len(names) + 3) + "|")
     for r in rows:
-        print(f"| {r['F']} | " + " | ".join(f"{r[n]:.3f}" for n in names) +
+        print(f"| {r['F']} | " + " | ".join(f"{r[n]:.3f}" if n in r else "-" for n in names) +
               f" | {E / (r['seastar'] / 1e3) / 1e9:.1f} | {r['alg_GBps_seastar']:.0f} |")
 
 
