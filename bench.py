@@ -122,11 +122,11 @@ def inputs_sha(w) -> str:
         a = w.get(k)
         if a is not None:
             h.update(k.encode())
-            h.update(memoryview(np.ascontiguousarray(a)).cast("B"))
+            h.update(np.ascontiguousarray(a).tobytes())
     for m in ("gcn", "gat", "appnp", "rgcn", "rgcnb"):
         for k, a in sorted((w.get(m) or {}).items()):
             h.update(f"{m}.{k}".encode())
-            h.update(memoryview(np.ascontiguousarray(a)).cast("B"))
+            h.update(np.ascontiguousarray(a).tobytes())
     return h.hexdigest()
 
 
