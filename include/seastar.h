@@ -318,7 +318,16 @@ size_t seastar_gat_attn_proj_bwd_workspace(int64_t M, int32_t H, int32_t F);
  *   X_all [N,F_in] ld ldx ; W [R,F_in,F_out] ; norm_user [E] by user edge id, or NULL = the
  *   graph's 1/c_{v,r} (requires SEASTAR_GRAPH_RGCN_NORM) ; Y_loc [n_loc,F_out] ld ldy.
  *   F_in, F_out <= 64.
- *   Two paths, chosen by shape (both deterministic, no atomics):
+ *   Three paths, chosen by shape (all deterministic; no floating-point atomics):
+ *   - default when F_in, F_out <= 16 (every R-GCN layer of the BASELINE configs; rgcn_tile.cu): edge-balanced
+ *     tiles of 512 edges in row order; each tile's gathered rows are staged in shared memory, its edges grouped by
+ *     type with a shared-memory counting sort, every edge's product norm_e X_all[src(e)] W[type(e)] computed with
+ *     the W[type] column held in registers across a type run, then each row sums its products in row order
+ *     ((type, eid) order); a row cut by tile borders is summed over its tiles in tile order.  W is resident in
+ *     shared memory ([R][16][round4(F_in)] fp32, persistent CTAs) when R * 64 * round4(F_in) + 82 KB fits in
+ *     227 KB, else read through L1/L2 (one tile per CTA).  workspace: seastar_rgcn_fwd_workspace() bytes
+ *     (dev, caller-owned: 128 B per tile, contents undefined on return); INVALID_ARGUMENT if it is smaller.
+ *     SEASTAR_RGCN_ROWS=1 selects the one-pass path below instead.
  *   - opt-in (environment SEASTAR_RGCN_TWOPHASE=1), F_in, F_out <= 16 and R * F_in * round4(F_out) * 4 <=
  *     200 KB (two-phase; slower than the one pass on the AM shape, kept for the r2 measurements): the edges are visited in
  *     type-major order, a lane per edge, with W staged in shared memory (the 32 edges of a warp share their
@@ -326,11 +335,12 @@ size_t seastar_gat_attn_proj_bwd_workspace(int64_t M, int32_t H, int32_t F);
  *     of `workspace` in row order, and each row sums its slots in (type, eid) order.  workspace:
  *     seastar_rgcn_fwd_workspace() bytes (dev, caller-owned, contents undefined on return); INVALID_ARGUMENT
  *     if it is smaller.
- *   - otherwise (one pass, the default; PAPER.md L473-L475 as written): every row walks its type-sorted edges and flushes
+ *   - otherwise (one pass; PAPER.md L473-L475 as written): every row walks its type-sorted edges and flushes
  *     each run through W[r] staged in shared memory (stride S floats per W[r]: the smallest stride
  *     >= F_in * round4(F_out) that is 16 mod 32 if R * S * 4 <= 219 KB, else the dense F_in * round4(F_out));
  *     needs R * S * 4 <= 227 KB - 256 B, and <= 219 KB when some row has degree >= 1024 (the hub CTAs keep an
  *     8 KB reduction buffer); UNSUPPORTED beyond.  seastar_rgcn_fwd_workspace() returns 0 (workspace may be NULL).
+ *   The workspace of seastar_rgcn_fwd_workspace() covers the path the library will take for this shape.
  */
 seastar_status seastar_rgcn_fwd(seastar_graph g, const float* X_all, int64_t F_in, int64_t ldx, const float* W,
                                 int64_t F_out, const float* norm_user, const float* bias, seastar_act act,
@@ -341,8 +351,10 @@ size_t seastar_rgcn_fwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out);
  *   dX_loc[u] = sum_{type runs r of out(u)} (sum_{e in run} norm_e dA_all[dst(e),:]) W[r]^T
  *     -- source-major over the type-sorted reverse CSR (§6.3.4 L461 + §6.3.5);
  *   dW[r] = sum_{owned v} g_{v,r}^T dA_all[v,:],  g_{v,r} = sum_{e in in(v), type r} norm_e X_all[src(e),:]
- *     -- over a type-major view of the forward edges built at graph_create; one warp owns a dW_r
- *     partial in registers per task, partials are reduced per type in task order (deterministic).
+ *     -- over a type-major view of the forward edges built at graph_create, cut into tasks of one type; per task
+ *     (F_in, F_out <= 16) the rows X_all[src] and dA_all[dst] are staged in shared memory and every warp keeps its
+ *     dW_r partial in registers, summing the per-edge outer products norm_e X_all[src]^T dA_all[dst]; partials
+ *     are reduced per type in task order (deterministic).
  *   X_all [N,F_in] ld ldx (the forward's gathered input) ; dA_all [N,F_out] ld ldd (gathered) ;
  *   dX_loc [n_loc,F_in] ld ldx or NULL ; dW [R,F_in,F_out] or NULL (overwritten; this rank's partial
  *   when partitioned).  ldx, ldd multiples of 4; F_in*F_out <= 1024.
@@ -353,8 +365,8 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
                                 const float* norm_user, const float* Yact_loc, seastar_act act, float* dX_loc,
                                 float* dW, void* workspace, size_t ws_bytes, seastar_stream stream);
 /* (Yact_loc [n_loc,F_in] ld ldx or NULL: dX_loc is multiplied by act'(Yact_loc), fusing the input
- *  layer's activation backward; act is ignored when Yact_loc is NULL.  dX takes the two-phase path of
- *  seastar_rgcn_fwd over the reverse edges when F_in, F_out <= 16; the workspace covers both uses.) */
+ *  layer's activation backward; act is ignored when Yact_loc is NULL.  dX takes the path seastar_rgcn_fwd would
+ *  take over the reverse edges (tile by default for F_in, F_out <= 16); the workspace covers dX and dW.) */
 size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out);
 
 /* ------------------------------------------------------------------------------------------ */

@@ -60,6 +60,7 @@ struct IndexSet {
     int64_t bucket_rows[SEASTAR_NUM_BUCKETS] = {0, 0, 0, 0};
     int64_t max_deg = 0;
     int64_t pow2_rows[kPow2Classes] = {};   // rows with degree >= 2^(kPow2Lo + k) (rows are degree-sorted)
+    int32_t* tile_row = nullptr;   // typed graphs: [2 n_tiles] first / last row of each kRgcnTileEdges-edge tile
 };
 
 // Type-major view of the FWD edges for the R-GCN weight gradient: edges sorted by (type, dst row,

@@ -13,6 +13,7 @@
 #include <vector>
 
 #include "common.cuh"
+#include "rgcn_tile.cuh"
 
 namespace seastar {
 
@@ -265,6 +266,26 @@ __global__ void k_pow2_rows(int64_t n, const int32_t* __restrict__ off, long lon
 }
 
 // degree buckets over degree-sorted rows: out[i] = #rows with deg >= threshold[i]; out[4] = max degree
+// R-GCN edge-balanced tiles (rgcn_tile.cu): tile_row[2t] / [2t+1] = the first / last row with an edge in tile t =
+// [t * kRgcnTileEdges, min((t + 1) * kRgcnTileEdges, E)) (rows with edges come first: rows are degree-sorted)
+__global__ void k_tile_rows(int64_t n, const int32_t* __restrict__ off, int32_t* __restrict__ tr) {
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (r >= n) return;
+    const int64_t b = off[r], e = off[r + 1], E = off[n];
+    if (b == e) return;
+    const int64_t tb = b / kRgcnTileEdges, te = (e - 1) / kRgcnTileEdges;
+    if (b % kRgcnTileEdges == 0 || r == 0) tr[2 * tb] = (int32_t)r;        // first row of tile tb
+    for (int64_t t = tb + 1; t <= te; ++t) tr[2 * t] = (int32_t)r;         // the row continues into tile t
+    for (int64_t t = tb; t < te; ++t) tr[2 * t + 1] = (int32_t)r;          // ... and covers tile t's last edge
+    const int64_t end_te = (te + 1) * kRgcnTileEdges < E ? (te + 1) * kRgcnTileEdges : E;
+    if (e == end_te) tr[2 * te + 1] = (int32_t)r;
+}
+
+static seastar_status tile_rows(int64_t n, const int32_t* off, int32_t* tr, cudaStream_t s) {
+    if (n > 0) k_tile_rows<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(n, off, tr);
+    return check_launch("k_tile_rows");
+}
+
 __global__ void k_buckets(int64_t n, const int32_t* __restrict__ off, long long* __restrict__ out) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
@@ -570,6 +591,10 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
         want(&g->rev.pos, Er, true);
         want(&g->rev.type, Er, etypes != nullptr);
         want(&g->rev.norm, Er, want_norm);
+        const int64_t fwd_tiles = (Ef + kRgcnTileEdges - 1) / kRgcnTileEdges;
+        const int64_t rev_tiles = (Er + kRgcnTileEdges - 1) / kRgcnTileEdges;
+        want(&g->fwd.tile_row, 2 * fwd_tiles + 2, etypes != nullptr);
+        want(&g->rev.tile_row, 2 * rev_tiles + 2, etypes != nullptr);
         want(&g->lsf.off, N + 1, part);
         want(&g->lsf.eid, Er, part);
         want(&g->fsplit.nbr, Ef, part);
@@ -626,6 +651,7 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
 
         // ---- a1: forward CSR ----------------------------------------------------------------------
         CKS(sort_rows(t, n_loc, row_begin, indptr, nullptr, g->indeg_loc, g->fwd.perm, g->fwd.off));
+        if (g->fwd.tile_row) CKS(tile_rows(n_loc, g->fwd.off, g->fwd.tile_row, s));
         if (!etypes) {
             if (n_loc > 0) {
                 k_fill_fwd<<<8 * num_sms(), 256, 0, s>>>(n_loc, g->fwd.perm, g->fwd.off, indptr, indices, nullptr,
@@ -652,6 +678,7 @@ seastar_status seastar_graph_create(int64_t N, int64_t E, const int64_t* indptr,
 
         // ---- a2: reverse CSR ----------------------------------------------------------------------
         CKS(sort_rows(t, n_loc, row_begin, nullptr, outdeg, g->outdeg_loc, g->rev.perm, g->rev.off));
+        if (g->rev.tile_row) CKS(tile_rows(n_loc, g->rev.off, g->rev.tile_row, s));
         int32_t *inv_rev, *sel_eid;
         if (t.alloc(&inv_rev, n_loc + 1) || t.alloc(&sel_eid, Er + 1))
             return fail(cuda_status(cudaErrorMemoryAllocation, "temps(rev)"));

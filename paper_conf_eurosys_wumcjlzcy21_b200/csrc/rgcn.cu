@@ -17,6 +17,7 @@
 #include <type_traits>
 
 #include "common.cuh"
+#include "rgcn_tile.cuh"
 
 namespace seastar {
 
@@ -768,6 +769,20 @@ static seastar_status launch_rows_L(const IndexSet& x, RgcnRowArgs a, cudaStream
     }
 }
 
+// the edge-balanced tile path (rgcn_tile.cu) from the one-pass argument block
+static RgcnTileArgs tile_args(const IndexSet& x, const RgcnRowArgs& a) {
+    RgcnTileArgs t{};
+    t.perm = x.perm; t.off = x.off; t.nbr = a.nbr; t.typ = a.typ; t.norm = a.norm; t.eid = a.eid;
+    t.norm_user = a.norm_user; t.tile_row = x.tile_row; t.n_rows = x.n_rows; t.n_edges = x.n_edges; t.vbase = a.vbase;
+    t.table = a.table; t.ldt = a.ldt; t.W = a.W; t.R = a.R; t.Fg = a.Fg; t.Fo = a.Fo; t.transpose = a.transpose;
+    t.out = a.out; t.ldo = a.ldo; t.bias = a.bias; t.act = a.act; t.Yact = a.Yact;
+    return t;
+}
+
+static bool use_tile(const EdgeMajor& em, const IndexSet& x, int R, int64_t Fg, int64_t Fo) {
+    return x.tile_row != nullptr && !two_phase(em, R, Fg, Fo) && rgcn_tile_ok(R, Fg, Fo);
+}
+
 }  // namespace seastar
 
 using namespace seastar;
@@ -775,8 +790,9 @@ using namespace seastar;
 extern "C" {
 
 size_t seastar_rgcn_fwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out) {
-    if (!g || !two_phase(g->fem, g->R, F_in, F_out)) return 0;
-    return em_ws_bytes(g->fem, F_out);
+    if (!g) return 0;
+    if (two_phase(g->fem, g->R, F_in, F_out)) return em_ws_bytes(g->fem, F_out);
+    return use_tile(g->fem, g->fwd, g->R, F_in, F_out) ? rgcn_tile_ws_bytes(g->fwd.n_edges) : 0;
 }
 
 seastar_status seastar_rgcn_fwd(seastar_graph g, const float* X_all, int64_t F_in, int64_t ldx, const float* W,
@@ -801,7 +817,9 @@ seastar_status seastar_rgcn_fwd(seastar_graph g, const float* X_all, int64_t F_i
     SS_ARG(need == 0 || (workspace && ws_bytes >= need), "rgcn_fwd: workspace too small (%zu < %zu bytes)", ws_bytes,
            need);
     ScopedL2Window win(X_all, (size_t)g->N * ldx * sizeof(float));
-    if (need) return launch_two_phase(g->fwd, g->fem, a, workspace, to_stream(stream));
+    if (two_phase(g->fem, g->R, F_in, F_out)) return launch_two_phase(g->fwd, g->fem, a, workspace, to_stream(stream));
+    if (use_tile(g->fem, g->fwd, g->R, F_in, F_out))
+        return rgcn_tile_launch(tile_args(g->fwd, a), g->fwd.bucket_rows[2], workspace, to_stream(stream));
     return launch_rows_L(g->fwd, a, to_stream(stream));
 }
 
@@ -809,7 +827,9 @@ size_t seastar_rgcn_bwd_workspace(seastar_graph g, int64_t F_in, int64_t F_out) 
     if (!g) return 0;
     // dW task partials and (two-phase dX) the per-segment products: used one after the other
     const size_t dw = (size_t)(g->tm.n_tasks + 1) * (size_t)(F_in * F_out) * sizeof(float) + 256;
-    const size_t dx = two_phase(g->rem, g->R, F_out, F_in) ? em_ws_bytes(g->rem, F_in) : 0;
+    const size_t dx = two_phase(g->rem, g->R, F_out, F_in)  ? em_ws_bytes(g->rem, F_in)
+                      : use_tile(g->rem, g->rev, g->R, F_out, F_in) ? rgcn_tile_ws_bytes(g->rev.n_edges)
+                                                            : 0;
     return dw > dx ? dw : dx;
 }
 
@@ -829,7 +849,7 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
     SS_ARG(!dW || (workspace && ws_bytes >= seastar_rgcn_bwd_workspace(g, F_in, F_out)),
            "rgcn_bwd: workspace too small");
     // argument checks stay before any launch: the two-phase dX needs the workspace as well
-    SS_ARG(!dX_loc || !two_phase(g->rem, g->R, F_out, F_in) ||
+    SS_ARG(!dX_loc || (!two_phase(g->rem, g->R, F_out, F_in) && !use_tile(g->rem, g->rev, g->R, F_out, F_in)) ||
            (workspace && ws_bytes >= seastar_rgcn_bwd_workspace(g, F_in, F_out)), "rgcn_bwd: workspace too small");
     SS_TRY(check_device());
     cudaStream_t s = to_stream(stream);
@@ -844,6 +864,8 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
         if (two_phase(g->rem, g->R, F_out, F_in)) {
             SS_ARG(workspace && ws_bytes >= seastar_rgcn_bwd_workspace(g, F_in, F_out), "rgcn_bwd: workspace too small");
             SS_TRY(launch_two_phase(g->rev, g->rem, a, workspace, s));
+        } else if (use_tile(g->rem, g->rev, g->R, F_out, F_in)) {
+            SS_TRY(rgcn_tile_launch(tile_args(g->rev, a), g->rev.bucket_rows[2], workspace, s));
         } else {
             SS_TRY(launch_rows_L(g->rev, a, s));
         }
@@ -895,7 +917,14 @@ seastar_status seastar_rgcn_bwd(seastar_graph g, const float* X_all, int64_t F_i
         case 3: RGCN_DWG(LL, 3); break;  \
         default: RGCN_DWG(LL, 4); break; \
     }
-            if (F_in <= 16 && F_out <= 16) {
+            const char* dwg = getenv("SEASTAR_RGCN_DWG");   // A/B: the r2 register-walk dW kernel
+            if (F_in <= 16 && F_out <= 16 && !(dwg && dwg[0] == '1')) {
+                RgcnDwTileArgs t{};
+                t.src = d.src; t.dst = d.dst; t.eid = d.eid; t.norm = d.norm; t.norm_user = d.norm_user;
+                t.run_off = d.run_off; t.task_run = d.task_run; t.n_tasks = d.n_tasks;
+                t.X = d.X; t.ldx = d.ldx; t.dA = d.dA; t.ldd = d.ldd; t.Fin = d.Fin; t.Fout = d.Fout; t.part = d.part;
+                SS_TRY(rgcn_dw_tile_launch(t, s));
+            } else if (F_in <= 16 && F_out <= 16) {
                 switch (pow2_ceil((int)((F_in + 1) / 2))) {   // lanes per group: 2 input features per lane
                     case 1: RGCN_DWG_L(1); break;
                     case 2: RGCN_DWG_L(2); break;

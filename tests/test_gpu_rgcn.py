@@ -82,23 +82,31 @@ def test_rgcn_bwd(env, Fin, Fout):
 
 
 @pytest.fixture
-def onepass(request, monkeypatch):
-    """The one-pass kernels (default) when True, the opt-in two-phase path (SEASTAR_RGCN_TWOPHASE=1) when False."""
-    if request.param:
-        monkeypatch.delenv("SEASTAR_RGCN_TWOPHASE", raising=False)
-    else:
+def path(request, monkeypatch):
+    """The R-GCN forward / dX formulation: "tile" (default: edge-balanced tiles with a CTA-local type grouping,
+    rgcn_tile.cu, persistent CTAs with W resident in shared memory), "standalone" (SEASTAR_RGCN_TILE_STANDALONE=1:
+    one tile per CTA, W through L1/L2), "rows" (SEASTAR_RGCN_ROWS=1: the one-pass row kernel, W_r in shared memory per type run) or
+    "twophase" (SEASTAR_RGCN_TWOPHASE=1: lane-per-edge products in type-major order + per-row sums)."""
+    monkeypatch.delenv("SEASTAR_RGCN_TWOPHASE", raising=False)
+    monkeypatch.delenv("SEASTAR_RGCN_ROWS", raising=False)
+    monkeypatch.delenv("SEASTAR_RGCN_TILE_STANDALONE", raising=False)
+    if request.param == "standalone":
+        monkeypatch.setenv("SEASTAR_RGCN_TILE_STANDALONE", "1")
+    if request.param == "rows":
+        monkeypatch.setenv("SEASTAR_RGCN_ROWS", "1")
+    elif request.param == "twophase":
         monkeypatch.setenv("SEASTAR_RGCN_TWOPHASE", "1")
     return request.param
 
 
-@pytest.mark.parametrize("onepass", [False, True], indirect=True)
+@pytest.mark.parametrize("path", ["tile", "standalone", "rows", "twophase"], indirect=True)
 @pytest.mark.parametrize("Fin,Fout", [(16, 16), (16, 11), (3, 7)])
-def test_rgcn_two_phase_and_one_pass(env, onepass, Fin, Fout):
-    """Both R-GCN paths (one pass with W_r in shared memory per type run; opt-in two-phase lane-per-edge products in
-    type-major order + per-row sums) against the oracle, forward and dX, with a hub row of 1,500 typed in-edges."""
+def test_rgcn_paths(env, path, Fin, Fout):
+    """Every R-GCN formulation against the oracle, forward and dX, with a hub row of 1,500 typed in-edges (two tile
+    borders inside it) and rows without in-edges."""
     torch, L, g, N, R = env["torch"], env["L"], env["g"], env["N"], env["R"]
     ws_f = L.seastar_rgcn_fwd_workspace(g.handle, Fin, Fout)
-    assert (ws_f == 0) == onepass
+    assert (ws_f == 0) == (path == "rows")
     ldx, ldy = (Fin + 3) // 4 * 4, (Fout + 3) // 4 * 4
     X, W, b = rnd(21, (N, Fin)), rnd(22, (R, Fin, Fout)), rnd(23, (Fout,))
     Y = torch.full((N, ldy), float("nan"), device="cuda")
@@ -114,6 +122,47 @@ def test_rgcn_two_phase_and_one_pass(env, onepass, Fin, Fout):
                        dev(env, W), None, None, "none", dX, None, ws, ws_b)
     rdX, _ = oracle.rgcn_bwd(env["ip"], env["ix"], env["et"], X, W, dA, need_dW=False)
     assert rel_err(dX.cpu().numpy()[:, :Fin], rdX) <= TOL
+
+
+@pytest.mark.parametrize("degs", [
+    [1024, 1024, 512, 512, 256, 256, 256, 256],          # rows ending exactly on 1,024-edge borders
+    [512, 512, 256, 256, 128, 128, 128, 128],             # ... on 512-edge borders (the default tile)
+    [3000, 1025, 1023, 7, 1, 1, 1],                       # a row over three tiles, rows cut by every border
+    [5000],                                               # one row, five tiles
+    [1] * 2500,                                           # a row per edge: a whole tile of rows
+    [40] * 300,                                           # rows cut by most borders, several tiles per CTA
+])
+def test_rgcn_tile_borders(degs):
+    """Edge-balanced tiles (512 edges by default, RGCN_TILE_EDGES): rows cut by tile borders are summed over their tiles in tile order; rows
+    without edges get the epilogue of 0.  Forward, dX (over the out-degrees) and dW against the oracle."""
+    import torch
+    from paper_conf_eurosys_wumcjlzcy21_b200 import _lib as L
+    from paper_conf_eurosys_wumcjlzcy21_b200.graph import Graph
+    R, Fin, Fout = 9, 16, 11
+    N = max(len(degs) + 5, 64)
+    rng = np.random.default_rng(sum(degs) + len(degs))
+    dst = np.repeat(np.arange(len(degs)), degs)
+    src = rng.integers(0, N, dst.size)
+    et = rng.integers(0, R, dst.size)
+    ip, ix, et = synth.csr_from_edges(N, src, dst, et)
+    g = Graph(ip, ix, et, num_etypes=R, rgcn_norm=True)
+    ldx, ldy = 16, 12
+    X, W, b = rnd(41, (N, Fin)), rnd(42, (R, Fin, Fout)), rnd(43, (Fout,))
+    Y = torch.full((N, ldy), float("nan"), device="cuda")
+    L.seastar_rgcn_fwd(g.handle, torch.from_numpy(X).cuda(), Fin, ldx, torch.from_numpy(W).cuda(), Fout, None,
+                       torch.from_numpy(b).cuda(), "relu", Y, ldy)
+    ref = oracle.act_fwd("relu", oracle.rgcn_fwd(ip, ix, et, X, W) + b)
+    assert rel_err(Y.cpu().numpy()[:, :Fout], ref) <= TOL
+    dA = rnd(44, (N, Fout))
+    dX = torch.full((N, ldx), float("nan"), device="cuda")
+    dW = torch.empty((R, Fin, Fout), device="cuda")
+    ws_b = L.seastar_rgcn_bwd_workspace(g.handle, Fin, Fout)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device="cuda")
+    L.seastar_rgcn_bwd(g.handle, torch.from_numpy(X).cuda(), Fin, ldx, torch.from_numpy(padded(dA, ldy)).cuda(), Fout,
+                       ldy, torch.from_numpy(W).cuda(), None, None, "none", dX, dW, ws, ws_b)
+    rdX, rdW = oracle.rgcn_bwd(ip, ix, et, X, W, dA)
+    assert rel_err(dX.cpu().numpy()[:, :Fin], rdX) <= TOL
+    assert rel_err(dW.cpu().numpy(), rdW) <= TOL
 
 
 def test_rgcn_fwd_workspace_required(env, monkeypatch):
