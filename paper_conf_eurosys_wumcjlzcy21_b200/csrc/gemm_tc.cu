@@ -86,9 +86,28 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
                  : "memory");
 }
 
+// A operand in TMEM (lane = row, 8 consecutive 32-bit columns per K step), B from shared memory
+__device__ __forceinline__ void mma_tf32_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n}" ::"r"(tmem_d), "r"(tmem_a), "l"(db), "r"(idesc),
+        "r"(acc));
+}
+// 16 consecutive 32-bit columns of this thread's TMEM lane (warp quarter addressing as tcgen05.ld)
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(taddr),
+        "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+        "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+        : "memory");
+}
+
 // Add TMEM slot (j & 1) -- the finished accumulation segment j -- into the fp32 register accumulators
 // of this thread's row (lane quarter q4), in column order, then hand the slot back to the MMA issuer.
-template <int NP>
+// NA accumulators per slot (k_gemm_tc2 keeps the three 3xTF32 products in separate accumulators, so consecutive
+// MMAs never depend on each other): they are summed in a fixed order before the register add.
+template <int NP, int NA = 1>
 __device__ __forceinline__ void drain_segment(uint32_t tmem, int j, int q4, uint64_t* seg_done, uint64_t* slot_free,
                                               float (&racc)[NP]) {
     const int slot = j & 1;
@@ -96,15 +115,21 @@ __device__ __forceinline__ void drain_segment(uint32_t tmem, int j, int q4, uint
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 #pragma unroll
     for (int c0 = 0; c0 < NP; c0 += 16) {
-        uint32_t v[16];
-        asm volatile(
-            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
-            : "r"(tmem + ((uint32_t)(q4 * 32) << 16) + (uint32_t)(slot * NP + c0)));
-        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+        float t[16];
 #pragma unroll
-        for (int q = 0; q < 16; ++q) racc[c0 + q] += __uint_as_float(v[q]);
+        for (int ai = 0; ai < NA; ++ai) {
+            uint32_t v[16];
+            asm volatile(
+                "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                  "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+                : "r"(tmem + ((uint32_t)(q4 * 32) << 16) + (uint32_t)((slot * NA + ai) * NP + c0)));
+            asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+            for (int q = 0; q < 16; ++q) t[q] = ai == 0 ? __uint_as_float(v[q]) : t[q] + __uint_as_float(v[q]);
+        }
+#pragma unroll
+        for (int q = 0; q < 16; ++q) racc[c0 + q] += t[q];
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     mbar_arrive(&slot_free[slot]);
@@ -279,6 +304,250 @@ __global__ void __launch_bounds__(192, TcCfg<NP>::CTAS) k_gemm_tc(const __grid_c
     }
 }
 
+// ------------------------------------------------------------------------------------------------
+// k_gemm_tc2: the same product, restructured for HBM streaming.  k_gemm_tc splits X in place,
+// so a stage's TMA could only be re-armed after the MMAs had consumed it, and the two stages per CTA kept too little
+// of X in flight (0.27 ms for Reddit 602 -> 64, ~1/3 of the HBM bound).  Here:
+//   * persistent CTAs (one per SM) loop over 128-row tiles, so the X stream never drains between tiles;
+//   * a deep ring of raw X tiles (NR x 16 KB, TMA) is decoupled from the operands: the split warps read their
+//     rows, write X_hi / X_lo straight into TMEM (tcgen05.st; the MMAs take A from TMEM), and release the raw stage,
+//     so the producer runs up to NR chunks ahead and shared memory carries no hi/lo copies and no A reads by the MMAs
+//     (the 3xTF32 operand traffic that bounded k_gemm_tc);
+//   * the W_hi | W_lo chunks stream through their own ring (WS stages, bulk copies by a dedicated warp), so their
+//     L2 latency never sits between a split and its MMAs;
+//   * the epilogue writes 128-bit rows.
+// Warp 0: X producer (TMA).  Warp 1: TMEM owner and MMA issuer.  Warps 2-5: split, segment drains, epilogue.
+// Warp 6: W producer.
+// ------------------------------------------------------------------------------------------------
+template <int NP>
+struct Tc2Cfg {
+    static constexpr int BM = 128, BK = 32;
+    static constexpr uint32_t RAW_BYTES = BM * BK * 4;                  // 16 KB
+    static constexpr uint32_t A_BYTES = BM * BK * 4;
+    static constexpr uint32_t B_BYTES = NP * BK * 4;
+    static constexpr uint32_t W_BYTES = 2 * B_BYTES;                    // W_hi | W_lo of one K chunk
+    // A stages in TMEM: the split of chunk c waits for the MMAs of chunk c - NH, so NH sets how many
+    // commit -> mbarrier round trips are in flight (2 stages: 0.2 ms for Reddit 602 -> 16, latency-bound)
+#ifndef TC2_NH
+#define TC2_NH 6
+#endif
+#ifndef TC2_CTAS
+#define TC2_CTAS 2   // measured (Reddit 602 -> 16 / 64): 1 CTA 0.20 / 0.30 ms, 2 CTAs 0.128 / 0.203 ms
+#endif
+    static constexpr int CTAS = (TC2_CTAS == 2 && NP <= 64) ? 2 : 1;       // co-resident CTAs per SM
+#ifndef TC2_NA
+#define TC2_NA 1     // 3: the three products in separate accumulators (measured: no gain)
+#endif
+    static constexpr int NA = (TC2_NA == 3 && 6 * NP + 2 * 64 <= 512 / CTAS) ? 3 : 1;   // accumulators per slot
+    static constexpr int NH_FIT = (512 / CTAS - 2 * NA * NP) / 64;
+    static constexpr int NH = NH_FIT < TC2_NH ? NH_FIT : TC2_NH, WS = 4;   // A stages (TMEM), W stages (smem)
+    static constexpr size_t BUDGET = (228 * 1024) / CTAS - 1024 /*reserved*/ - 1024 /*align*/ - 512 /*barriers*/;
+    static constexpr int NR_FIT = (int)((BUDGET - WS * W_BYTES) / RAW_BYTES);
+    static constexpr int NR = NR_FIT > 12 ? 12 : NR_FIT;
+    static constexpr int SEG = TC_SEG;
+    // TMEM: two accumulator slots [0, 2 NP), then NH A stages of 64 columns (X_hi: 32, X_lo: 32)
+    static constexpr uint32_t A_COL0 = 2 * NA * NP;
+    static constexpr uint32_t COLS_USED = 2 * NA * NP + NH * 64;
+    static constexpr uint32_t TMEM_COLS = COLS_USED <= 64 ? 64 : (COLS_USED <= 128 ? 128 : (COLS_USED <= 256 ? 256 : 512));
+    static constexpr size_t SMEM = (size_t)NR * RAW_BYTES + (size_t)WS * W_BYTES + 1024 + 512;
+    static_assert(NH >= 2 && NR >= 2, "k_gemm_tc2 does not fit");
+};
+
+template <int NP>
+__global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid_constant__ CUtensorMap tmX, const TcArgs a) {
+    using C = Tc2Cfg<NP>;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* raw_base = smem;
+    uint8_t* w_base = raw_base + (size_t)C::NR * C::RAW_BYTES;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(w_base + (size_t)C::WS * C::W_BYTES);
+    uint64_t* raw_full = bars;                       // [NR] TMA landed
+    uint64_t* raw_empty = raw_full + C::NR;          // [NR] split warps done reading (128 arrivals)
+    uint64_t* split_full = raw_empty + C::NR;        // [NH] hi/lo written (128 arrivals)
+    uint64_t* hl_empty = split_full + C::NH;         // [NH] MMAs done reading
+    uint64_t* w_full = hl_empty + C::NH;             // [WS] W chunk landed
+    uint64_t* w_empty = w_full + C::WS;              // [WS] MMAs done reading
+    uint64_t* seg_done = w_empty + C::WS;            // [2]
+    uint64_t* slot_free = seg_done + 2;              // [2] (128 arrivals)
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(slot_free + 2);
+    auto RAW = [&](int r) { return raw_base + (size_t)r * C::RAW_BYTES; };
+    auto B_hi = [&](int w) { return w_base + (size_t)w * C::W_BYTES; };
+    auto B_lo = [&](int w) { return w_base + (size_t)w * C::W_BYTES + C::B_BYTES; };
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nk = (int)((a.K + C::BK - 1) / C::BK);
+    const int nseg = (nk + C::SEG - 1) / C::SEG;
+    const int64_t tiles = (a.M + C::BM - 1) / C::BM;
+
+    if (threadIdx.x == 0) {
+        for (int r = 0; r < C::NR; ++r) {
+            mbar_init(&raw_full[r], 1);
+            mbar_init(&raw_empty[r], 128);
+        }
+        for (int h = 0; h < C::NH; ++h) {
+            mbar_init(&split_full[h], 128);
+            mbar_init(&hl_empty[h], 1);
+        }
+        for (int w = 0; w < C::WS; ++w) {
+            mbar_init(&w_full[w], 1);
+            mbar_init(&w_empty[w], 1);
+        }
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(&seg_done[b], 1);
+            mbar_init(&slot_free[b], 128);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(C::TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0) {
+        // ---------------- X producer: raw tiles, up to NR chunks ahead ----------------
+        if (lane == 0) {
+            int c = 0;
+            for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                for (int kc = 0; kc < nk; ++kc, ++c) {
+                    const int r = c % C::NR;
+                    if (c >= C::NR) mbar_wait(&raw_empty[r], ((c / C::NR) - 1) & 1);
+                    mbar_expect_tx(&raw_full[r], C::RAW_BYTES);
+                    tma_load_2d(RAW(r), &tmX, kc * C::BK, (int)(tile * C::BM), &raw_full[r]);
+                }
+            }
+        }
+    } else if (warp == 6) {
+        // ---------------- W producer: pre-split W_hi | W_lo chunks, up to WS chunks ahead ----------------
+        if (lane == 0) {
+            int c = 0;
+            for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                for (int kc = 0; kc < nk; ++kc, ++c) {
+                    const int w = c % C::WS;
+                    if (c >= C::WS) mbar_wait(&w_empty[w], ((c / C::WS) - 1) & 1);
+                    mbar_expect_tx(&w_full[w], C::W_BYTES);
+                    bulk_copy(B_hi(w), a.Wsplit + (size_t)kc * C::W_BYTES / sizeof(float), C::W_BYTES, &w_full[w]);
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ---------------- MMA issuer ----------------
+        const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NP >> 3) << 17) | ((128u >> 4) << 24);
+        int c = 0, J = 0;
+        for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x, J += nseg) {
+            for (int kc = 0; kc < nk; ++kc, ++c) {
+                const int h = c % C::NH, w = c % C::WS;
+                const int j = J + kc / C::SEG, slot = j & 1;
+                const bool first = (kc % C::SEG) == 0;
+                if (first && j >= 2) mbar_wait(&slot_free[slot], ((j >> 1) - 1) & 1);   // segment j-2 drained
+                mbar_wait(&split_full[h], (c / C::NH) & 1);
+                mbar_wait(&w_full[w], (c / C::WS) & 1);
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                if (lane == 0) {
+                    const uint32_t ah = tmem + C::A_COL0 + (uint32_t)h * 64, al = ah + 32;   // A in TMEM (K-major)
+                    const uint64_t bh = smem_desc_k128(B_hi(w)), bl = smem_desc_k128(B_lo(w));
+                    const uint32_t d0 = tmem + (uint32_t)(slot * C::NA * NP);
+                    const uint32_t d1 = d0 + (C::NA > 1 ? NP : 0), d2 = d0 + (C::NA > 1 ? 2 * NP : 0);
+#pragma unroll
+                    for (int ks = 0; ks < C::BK / 8; ++ks) {
+                        const uint64_t adv = (uint64_t)((ks * 8 * 4) >> 4);
+                        const uint32_t init = (!first || ks > 0) ? 1u : 0u;
+                        mma_tf32_ts(d0, al + ks * 8, bh + adv, idesc, init);
+                        mma_tf32_ts(d1, ah + ks * 8, bl + adv, idesc, C::NA > 1 ? init : 1u);
+                        mma_tf32_ts(d2, ah + ks * 8, bh + adv, idesc, C::NA > 1 ? init : 1u);
+                    }
+                    mma_commit(&hl_empty[h]);
+                    mma_commit(&w_empty[w]);
+                    if ((kc % C::SEG) == C::SEG - 1 || kc == nk - 1) mma_commit(&seg_done[slot]);
+                }
+                __syncwarp();
+            }
+        }
+    } else {
+        // ---------------- split, segment drains, epilogue (warps 2-5) ----------------
+        const int t = threadIdx.x - 64;
+        const int q4 = warp & 3;
+        float racc[NP];
+#pragma unroll
+        for (int j = 0; j < NP; ++j) racc[j] = 0.f;
+        int c = 0, J = 0;
+        for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x, J += nseg) {
+            for (int kc = 0; kc < nk; ++kc, ++c) {
+                const int r = c % C::NR, h = c % C::NH;
+                mbar_wait(&raw_full[r], (c / C::NR) & 1);
+                // this thread's row (TMEM lane) of the 128B-swizzled raw tile: chunk q of row rr sits at
+                // rr * 128 + ((q ^ (rr & 7)) * 16) (8 consecutive rows hit 8 different bank groups)
+                const int rr = q4 * 32 + lane;
+                const uint8_t* prow = RAW(r) + rr * 128;
+                float4 xv[8];
+#pragma unroll
+                for (int q = 0; q < 8; ++q) xv[q] = *reinterpret_cast<const float4*>(prow + ((q ^ (rr & 7)) << 4));
+                mbar_arrive(&raw_empty[r]);                   // the raw stage can be refilled now
+                if (c >= C::NH) mbar_wait(&hl_empty[h], ((c / C::NH) - 1) & 1);   // A stage h is free
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                const uint32_t ta = tmem + ((uint32_t)(q4 * 32) << 16) + C::A_COL0 + (uint32_t)h * 64;
+#pragma unroll
+                for (int half = 0; half < 2; ++half) {
+                    uint32_t hv[16], lv[16];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const float4 x = xv[4 * half + q];
+                        const float xs[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) {
+                            const float hh = rna_tf32(xs[u]);
+                            hv[4 * q + u] = __float_as_uint(hh);
+                            lv[4 * q + u] = __float_as_uint(xs[u] - hh);
+                        }
+                    }
+                    tmem_st16(ta + half * 16, hv);
+                    tmem_st16(ta + 32 + half * 16, lv);
+                }
+                asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+                asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+                mbar_arrive(&split_full[h]);
+                if (((kc % C::SEG) == C::SEG - 1 || kc == nk - 1) && kc / C::SEG >= 1)
+                    drain_segment<NP, C::NA>(tmem, J + kc / C::SEG - 1, q4, seg_done, slot_free, racc);
+            }
+            if (nk > 0) drain_segment<NP, C::NA>(tmem, J + nseg - 1, q4, seg_done, slot_free, racc);
+            // epilogue: bias, activation, row scale; 128-bit stores when the rows allow it
+            const int64_t gm = tile * C::BM + q4 * 32 + lane;
+            if (gm < a.M) {
+                const float rs = a.row_scale ? __ldg(a.row_scale + gm) : 1.f;
+                float* y = a.Y + gm * a.ldy;
+                const bool vec = (a.ldy & 3) == 0 && aligned16(a.Y);
+#pragma unroll
+                for (int j = 0; j < NP; j += 4) {
+                    float z[4];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        z[q] = rs * act_apply(a.act, racc[j + q] + ((a.bias && j + q < a.N) ? __ldg(a.bias + j + q) : 0.f));
+                    if (vec && j + 4 <= a.N) {
+                        *reinterpret_cast<float4*>(y + j) = make_float4(z[0], z[1], z[2], z[3]);
+                    } else {
+#pragma unroll
+                        for (int q = 0; q < 4; ++q)
+                            if (j + q < a.N) y[j + q] = z[q];
+                    }
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < NP; ++j) racc[j] = 0.f;
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 1) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C::TMEM_COLS));
+    }
+}
+
 // W [K, N] -> per 32-wide K chunk: W_hi = rna_tf32(W) and W_lo = W - W_hi as NP x 32 K-major tiles in the
 // 128B-swizzled layout the UMMA descriptor expects (element (n, k) at n*128 + ((k/4 ^ n%8)*16 | (k%4)*4))
 __global__ void k_split_w(const float* __restrict__ W, int64_t K, int64_t N, int NP, float* __restrict__ out) {
@@ -320,6 +589,19 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 
 template <int NP>
 static seastar_status launch_tc_np(const CUtensorMap& tm, const TcArgs& a, cudaStream_t s) {
+    // NP <= 64 (every BASELINE transform): k_gemm_tc2; wider outputs and SEASTAR_TC_V1=1 (A/B): k_gemm_tc
+    if constexpr (NP <= 64) {
+        const char* v1 = getenv("SEASTAR_TC_V1");
+        if (!(v1 && v1[0] == '1')) {
+            using C2 = Tc2Cfg<NP>;
+            SS_CUDA(cudaFuncSetAttribute(k_gemm_tc2<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C2::SMEM));
+            const int64_t tiles = (a.M + C2::BM - 1) / C2::BM;
+            const int64_t slots = (int64_t)C2::CTAS * num_sms();
+            const unsigned grid = (unsigned)(tiles < slots ? tiles : slots);
+            k_gemm_tc2<NP><<<grid, 224, C2::SMEM, s>>>(tm, a);
+            return check_launch("k_gemm_tc2");
+        }
+    }
     using C = TcCfg<NP>;
     // set per call: the attribute is per device, and setting it is a cheap host-side call
     SS_CUDA(cudaFuncSetAttribute(k_gemm_tc<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
