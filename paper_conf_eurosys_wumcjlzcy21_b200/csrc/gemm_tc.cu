@@ -835,10 +835,202 @@ __global__ void __launch_bounds__(192, TcTnCfg<NP32>::CTAS)
     }
 }
 
+// ------------------------------------------------------------------------------------------------
+// k_gemm_tc_tn2: dW = X^T dY with the same restructuring as k_gemm_tc2.  A = X^T (M' = 128 features k of the tile,
+// K' = rows m) is K-major when each TMEM lane k holds consecutive rows m: the split warps read column k of a raw
+// X tile ([32 m][128 k], plain row-major TMA box, lane-consecutive words: conflict-free), write X_hi / X_lo into
+// TMEM, and the MMAs take A from there.  B = dY^T stays an MN-major shared-memory operand (SWIZZLE_128B_ATOM_32B,
+// split in place into a B stage).  Raw stages (X tile + dY tile) are released right after the split, so TMA runs
+// NR chunks ahead; 2 CTAs per SM.  Per-split partials [nsplit][K][N] as before (reduced in split order).
+// ------------------------------------------------------------------------------------------------
+template <int NP32>
+struct TcTn2Cfg {
+    static constexpr int BM = 128, BR = 32;                   // k tile, rows per chunk
+    static constexpr int CTAS = 2;
+    static constexpr uint32_t X_BYTES = BR * BM * 4;           // 16 KB raw X tile
+    static constexpr uint32_t Y_BYTES = NP32 * BR * 4;         // 4 KB per 32 columns (4 KB-aligned boxes)
+    static constexpr uint32_t RAW_BYTES = X_BYTES + Y_BYTES;
+    static constexpr uint32_t B_BYTES = NP32 * BR * 4;
+    static constexpr int NH = (256 - 2 * NP32) / 64 > 3 ? 3 : (256 - 2 * NP32) / 64;   // A stages (TMEM) = B stages
+    static constexpr size_t BUDGET = (228 * 1024) / CTAS - 1024 - 1024 - 256;
+    static constexpr int NR_FIT = (int)((BUDGET - (size_t)NH * 2 * B_BYTES) / RAW_BYTES);
+    static constexpr int NR = NR_FIT > 8 ? 8 : NR_FIT;
+    static constexpr int SEG = TC_TN_SEG;
+    static constexpr uint32_t A_COL0 = 2 * NP32;
+    static constexpr uint32_t TMEM_COLS = 256;
+    static constexpr size_t SMEM = (size_t)NR * RAW_BYTES + (size_t)NH * 2 * B_BYTES + 1024 + 256;
+    static_assert(NH >= 2 && NR >= 2, "k_gemm_tc_tn2 does not fit");
+};
+
+template <int NP32>
+__global__ void __launch_bounds__(192, TcTn2Cfg<NP32>::CTAS)
+    k_gemm_tc_tn2(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmY, const TcTnArgs a) {
+    using C = TcTn2Cfg<NP32>;
+    constexpr int NB = NP32 / 32;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* raw_base = smem;
+    uint8_t* b_base = raw_base + (size_t)C::NR * C::RAW_BYTES;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(b_base + (size_t)C::NH * 2 * C::B_BYTES);
+    uint64_t* raw_full = bars;                   // [NR]
+    uint64_t* raw_empty = raw_full + C::NR;      // [NR] (128 arrivals)
+    uint64_t* split_full = raw_empty + C::NR;    // [NH] (128 arrivals)
+    uint64_t* hl_empty = split_full + C::NH;     // [NH]
+    uint64_t* seg_done = hl_empty + C::NH;       // [2]
+    uint64_t* slot_free = seg_done + 2;          // [2] (128 arrivals)
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(slot_free + 2);
+    auto RX = [&](int r) { return raw_base + (size_t)r * C::RAW_BYTES; };
+    auto RY = [&](int r) { return raw_base + (size_t)r * C::RAW_BYTES + C::X_BYTES; };
+    auto B_hi = [&](int h) { return b_base + (size_t)h * 2 * C::B_BYTES; };
+    auto B_lo = [&](int h) { return b_base + (size_t)h * 2 * C::B_BYTES + C::B_BYTES; };
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int k0 = blockIdx.x * C::BM;
+    const int64_t r0 = (int64_t)blockIdx.y * a.rows_per_split;
+    const int64_t r1 = min(a.M, r0 + a.rows_per_split);
+    const int nch = (int)((r1 - r0 + C::BR - 1) / C::BR);
+
+    if (threadIdx.x == 0) {
+        for (int r = 0; r < C::NR; ++r) {
+            mbar_init(&raw_full[r], 1);
+            mbar_init(&raw_empty[r], 128);
+        }
+        for (int h = 0; h < C::NH; ++h) {
+            mbar_init(&split_full[h], 128);
+            mbar_init(&hl_empty[h], 1);
+        }
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(&seg_done[b], 1);
+            mbar_init(&slot_free[b], 128);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(C::TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            for (int c = 0; c < nch; ++c) {
+                const int r = c % C::NR;
+                if (c >= C::NR) mbar_wait(&raw_empty[r], ((c / C::NR) - 1) & 1);
+                mbar_expect_tx(&raw_full[r], C::X_BYTES + C::Y_BYTES);
+                const int m = (int)(r0 + (int64_t)c * C::BR);
+                tma_load_2d(RX(r), &tmX, k0, m, &raw_full[r]);
+#pragma unroll
+                for (int j = 0; j < NB; ++j) tma_load_2d(RY(r) + j * 4096, &tmY, 32 * j, m, &raw_full[r]);
+            }
+        }
+    } else if (warp == 1) {
+        // D f32, A/B tf32, A K-major (TMEM), B MN-major (bit 16), N = NP32, M = 128
+        const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 16) | ((uint32_t)(NP32 >> 3) << 17) |
+                               ((128u >> 4) << 24);
+        for (int c = 0; c < nch; ++c) {
+            const int h = c % C::NH;
+            const int j = c / C::SEG, slot = j & 1;
+            const bool first = (c % C::SEG) == 0;
+            if (first && j >= 2) mbar_wait(&slot_free[slot], ((j >> 1) - 1) & 1);
+            mbar_wait(&split_full[h], (c / C::NH) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            if (lane == 0) {
+                const uint32_t d = tmem + (uint32_t)(slot * NP32);
+                const uint32_t ah = tmem + C::A_COL0 + (uint32_t)h * 64, al = ah + 32;
+#pragma unroll
+                for (int ks = 0; ks < C::BR / 8; ++ks) {
+                    const uint64_t bh = smem_desc_mn32b(B_hi(h) + ks * 1024, 4096);
+                    const uint64_t bl = smem_desc_mn32b(B_lo(h) + ks * 1024, 4096);
+                    mma_tf32_ts(d, al + ks * 8, bh, idesc, (!first || ks > 0) ? 1u : 0u);
+                    mma_tf32_ts(d, ah + ks * 8, bl, idesc, 1u);
+                    mma_tf32_ts(d, ah + ks * 8, bh, idesc, 1u);
+                }
+                mma_commit(&hl_empty[h]);
+                if ((c % C::SEG) == C::SEG - 1 || c == nch - 1) mma_commit(&seg_done[slot]);
+            }
+            __syncwarp();
+        }
+    } else {
+        const int t = threadIdx.x - 64;
+        const int q4 = warp & 3;
+        const int kk = q4 * 32 + lane;                  // this thread's TMEM lane = feature k0 + kk
+        float racc[NP32];
+#pragma unroll
+        for (int j = 0; j < NP32; ++j) racc[j] = 0.f;
+        for (int c = 0; c < nch; ++c) {
+            const int r = c % C::NR, h = c % C::NH;
+            mbar_wait(&raw_full[r], (c / C::NR) & 1);
+            const float* px = reinterpret_cast<const float*>(RX(r)) + kk;
+            float xc[32];
+#pragma unroll
+            for (int m = 0; m < 32; ++m) xc[m] = px[m * 128];     // column kk of the [32 m][128 k] tile
+            const float4* qy = reinterpret_cast<const float4*>(RY(r));
+            float4 yv[NB * 2];
+#pragma unroll
+            for (int q = 0; q < NB * 2; ++q) yv[q] = qy[q * 128 + t];
+            mbar_arrive(&raw_empty[r]);
+            if (c >= C::NH) mbar_wait(&hl_empty[h], ((c / C::NH) - 1) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            const uint32_t ta = tmem + ((uint32_t)(q4 * 32) << 16) + C::A_COL0 + (uint32_t)h * 64;
+#pragma unroll
+            for (int half = 0; half < 2; ++half) {
+                uint32_t hv[16], lv[16];
+#pragma unroll
+                for (int u = 0; u < 16; ++u) {
+                    const float x = xc[16 * half + u];
+                    const float hh = rna_tf32(x);
+                    hv[u] = __float_as_uint(hh);
+                    lv[u] = __float_as_uint(x - hh);
+                }
+                tmem_st16(ta + half * 16, hv);
+                tmem_st16(ta + 32 + half * 16, lv);
+            }
+            float4* bh = reinterpret_cast<float4*>(B_hi(h));
+            float4* bl = reinterpret_cast<float4*>(B_lo(h));
+#pragma unroll
+            for (int q = 0; q < NB * 2; ++q) {                    // layout-preserving split of the dY tile
+                const float4 x = yv[q];
+                const float4 hh = make_float4(rna_tf32(x.x), rna_tf32(x.y), rna_tf32(x.z), rna_tf32(x.w));
+                bh[q * 128 + t] = hh;
+                bl[q * 128 + t] = make_float4(x.x - hh.x, x.y - hh.y, x.z - hh.z, x.w - hh.w);
+            }
+            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+            asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive(&split_full[h]);
+            if (((c % C::SEG) == C::SEG - 1 || c == nch - 1) && c / C::SEG >= 1)
+                drain_segment<NP32>(tmem, c / C::SEG - 1, q4, seg_done, slot_free, racc);
+        }
+        if (nch > 0) drain_segment<NP32>(tmem, (nch - 1) / C::SEG, q4, seg_done, slot_free, racc);
+        const int64_t gk = k0 + kk;
+        if (gk < a.K) {
+            float* prow = a.part + ((int64_t)blockIdx.y * a.K + gk) * a.N;
+#pragma unroll
+            for (int j = 0; j < NP32; ++j)
+                if (j < a.N) prow[j] = racc[j];
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 1) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C::TMEM_COLS));
+    }
+}
+
 // row splits (multiples of 32 rows) so that ktiles x nsplit fills ~4 waves of 2 CTAs per SM
+#ifndef TCTN_CTAS_PER_SM
+#define TCTN_CTAS_PER_SM 4   // CTAs per SM the row splits aim for (measured on Reddit 602 x 64: 8 -> 0.237 ms, 4 -> 0.205, 2 -> 0.252)
+#endif
 static void tc_tn_geometry(int64_t M, int64_t K, int64_t& ktiles, int64_t& nsplit, int64_t& rows_per_split) {
     ktiles = (K + 127) / 128;
-    int64_t want = (8 * num_sms() + ktiles - 1) / ktiles;
+    int64_t want = (TCTN_CTAS_PER_SM * num_sms() + ktiles - 1) / ktiles;
     int64_t max_split = (M + 255) / 256;
     nsplit = want < max_split ? want : max_split;
     if (nsplit < 1) nsplit = 1;
@@ -852,6 +1044,15 @@ size_t linear_bwd_weight_tc_part_bytes(int64_t M, int64_t K, int64_t N) {
     int64_t kt, ns, rps;
     tc_tn_geometry(M > 0 ? M : 1, K, kt, ns, rps);
     return (size_t)ns * K * N * sizeof(float);
+}
+
+template <int NP32>
+static seastar_status launch_tc_tn2(const CUtensorMap& tx, const CUtensorMap& ty, const TcTnArgs& a, dim3 grid,
+                                    cudaStream_t s) {
+    using C = TcTn2Cfg<NP32>;
+    SS_CUDA(cudaFuncSetAttribute(k_gemm_tc_tn2<NP32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
+    k_gemm_tc_tn2<NP32><<<grid, 192, C::SMEM, s>>>(tx, ty, a);
+    return check_launch("k_gemm_tc_tn2");
 }
 
 template <int NP32>
@@ -899,6 +1100,19 @@ seastar_status linear_bwd_weight_tc(const float* X, int64_t M, int64_t K, int64_
     TcTnArgs a{M, K, N, rps, part};
     *nsplit_out = ns;
     const dim3 grid((unsigned)kt, (unsigned)ns);
+    const char* v1 = getenv("SEASTAR_TC_V1");   // A/B: the r1/r2 in-place-split kernel
+    if (!(v1 && v1[0] == '1')) {
+        // k_gemm_tc_tn2: X as plain [32 rows][128 features] boxes (each split thread reads one feature column)
+        CUtensorMap tx2;
+        cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)M};
+        cuuint64_t strides[1] = {(cuuint64_t)ldx * sizeof(float)};
+        cuuint32_t box[2] = {128, 32};
+        cuuint32_t estr[2] = {1, 1};
+        if (enc(&tx2, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(X), dims, strides, box, estr,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS)
+            return N <= 32 ? launch_tc_tn2<32>(tx2, ty, a, grid, s) : launch_tc_tn2<64>(tx2, ty, a, grid, s);
+    }
     return N <= 32 ? launch_tc_tn<32>(tx, ty, a, grid, s) : launch_tc_tn<64>(tx, ty, a, grid, s);
 }
 
