@@ -487,7 +487,6 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
                 float4 xv[8];
 #pragma unroll
                 for (int q = 0; q < 8; ++q) xv[q] = *reinterpret_cast<const float4*>(prow + ((q ^ (rr & 7)) << 4));
-                mbar_arrive(&raw_empty[r]);                   // the raw stage can be refilled now
                 if (c >= C::NH) mbar_wait(&hl_empty[h], ((c / C::NH) - 1) & 1);   // A stage h is free
                 asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
                 const uint32_t ta = tmem + ((uint32_t)(q4 * 32) << 16) + C::A_COL0 + (uint32_t)h * 64;
@@ -511,6 +510,7 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
                 asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
                 asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
                 mbar_arrive(&split_full[h]);
+                mbar_arrive(&raw_empty[r]);                   // after the raw values were consumed (see k_gemm_tc_tn2)
                 if (((kc % C::SEG) == C::SEG - 1 || kc == nk - 1) && kc / C::SEG >= 1)
                     drain_segment<NP, C::NA>(tmem, J + kc / C::SEG - 1, q4, seg_done, slot_free, racc);
             }
@@ -974,7 +974,6 @@ __global__ void __launch_bounds__(192, TcTn2Cfg<NP32>::CTAS)
             float4 yv[NB * 2];
 #pragma unroll
             for (int q = 0; q < NB * 2; ++q) yv[q] = qy[q * 128 + t];
-            mbar_arrive(&raw_empty[r]);
             if (c >= C::NH) mbar_wait(&hl_empty[h], ((c / C::NH) - 1) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
             const uint32_t ta = tmem + ((uint32_t)(q4 * 32) << 16) + C::A_COL0 + (uint32_t)h * 64;
@@ -1004,6 +1003,9 @@ __global__ void __launch_bounds__(192, TcTn2Cfg<NP32>::CTAS)
             asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             mbar_arrive(&split_full[h]);
+            // the raw stage is released only after its values were consumed (the TMA refill is an async-proxy write;
+            // arriving right after issuing the loads let refills race with loads still in flight at large M)
+            mbar_arrive(&raw_empty[r]);
             if (((c % C::SEG) == C::SEG - 1 || c == nch - 1) && c / C::SEG >= 1)
                 drain_segment<NP32>(tmem, c / C::SEG - 1, q4, seg_done, slot_free, racc);
         }

@@ -43,7 +43,8 @@ def test_linear_fwd(env, M, K, N):
 
 
 TC_SHAPES = [(128, 32, 16), (1000, 602, 16), (5003, 602, 64), (777, 64, 41), (3001, 1433, 70), (300, 8710, 8),
-             (2048, 100, 128), (129, 33, 1)]
+             (2048, 100, 128), (129, 33, 1),
+             (60000, 602, 64)]   # many chunks per CTA: the raw-tile ring wraps many times (r2: a WAR race showed here)
 
 
 @pytest.mark.parametrize("M,K,N", TC_SHAPES)
@@ -134,7 +135,8 @@ def test_colsum_axpby_adam(env):
 
 
 TC_TN_SHAPES = [(256, 32, 1), (1000, 602, 16), (5003, 602, 64), (3001, 64, 41), (300, 8710, 8), (4099, 100, 33),
-                (20000, 128, 32), (233, 602, 16), (2000, 64, 70), (3000, 100, 130), (300, 40, 200)]
+                (20000, 128, 32), (233, 602, 16), (2000, 64, 70), (3000, 100, 130), (300, 40, 200),
+                (60000, 602, 64), (60000, 602, 32)]   # >= 16 chunks per CTA (r2: the raw-ring WAR race of tc_tn2)
 
 
 @pytest.mark.parametrize("M,K,N", TC_TN_SHAPES)
