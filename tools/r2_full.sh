@@ -9,4 +9,5 @@ for w in cora_gcn corafull_gat physics_appnp am_rgcn aifb_rgcnb mutag_rgcnb bgs_
   timeout 300 python bench.py --workload $w > gpurun_out/$T/bench_$w.json 2> gpurun_out/$T/bench_$w.err
   python -c "import json;d=json.load(open('gpurun_out/$T/bench_$w.json'));print('$w', round(d['ms_per_step'],4), round(d['e2e']['ms_per_step'],4), round(d['cpu_baseline']['value']/1e6,3))"
 done
-bash tools/sanitize.sh gpurun_out/$T
+# compute-sanitizer is closed on this pool (gpurun refuses it); r2 logs: profiles/r2/r2full1/sanitize_*.log
+# bash tools/sanitize.sh gpurun_out/$T
