@@ -27,7 +27,12 @@ struct TcArgs {
     const float* Wsplit;            // [nk][W_hi tile | W_lo tile], each NP x 32 K-major, 128B-swizzled
     float* Y; int64_t ldy;
     const float* bias; const float* row_scale; int act;
+    int ksplit = 1;                 // k_gemm_tc2: K splits per tile (partials in part, then k_splitk_reduce)
+    float* part = nullptr;          // [ksplit][M][NP]
 };
+constexpr int kSplitKMax = 8;
+// K splits are used only while the row tiles cannot fill two CTAs per SM
+static int64_t splitk_max_rows() { return 2 * (int64_t)num_sms() * 128; }
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -376,8 +381,12 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nk = (int)((a.K + C::BK - 1) / C::BK);
-    const int nseg = (nk + C::SEG - 1) / C::SEG;
-    const int64_t tiles = (a.M + C::BM - 1) / C::BM;
+    const int tiles = (int)((a.M + C::BM - 1) / C::BM);
+    // work item = (128-row tile, K split): split s of a tile covers chunks [s nk / S, (s + 1) nk / S)
+    const int S = a.ksplit;
+    const int items = tiles * S;
+    auto k_lo = [&](int it) { return (it % S) * nk / S; };
+    auto k_hi = [&](int it) { return (it % S + 1) * nk / S; };
 
     if (threadIdx.x == 0) {
         for (int r = 0; r < C::NR; ++r) {
@@ -413,12 +422,13 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
         // ---------------- X producer: raw tiles, up to NR chunks ahead ----------------
         if (lane == 0) {
             int c = 0;
-            for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
-                for (int kc = 0; kc < nk; ++kc, ++c) {
+            for (int it = blockIdx.x; it < items; it += gridDim.x) {
+                const int tile = it / S;
+                for (int kc = k_lo(it); kc < k_hi(it); ++kc, ++c) {
                     const int r = c % C::NR;
                     if (c >= C::NR) mbar_wait(&raw_empty[r], ((c / C::NR) - 1) & 1);
                     mbar_expect_tx(&raw_full[r], C::RAW_BYTES);
-                    tma_load_2d(RAW(r), &tmX, kc * C::BK, (int)(tile * C::BM), &raw_full[r]);
+                    tma_load_2d(RAW(r), &tmX, kc * C::BK, tile * C::BM, &raw_full[r]);
                 }
             }
         }
@@ -426,8 +436,8 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
         // ---------------- W producer: pre-split W_hi | W_lo chunks, up to WS chunks ahead ----------------
         if (lane == 0) {
             int c = 0;
-            for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
-                for (int kc = 0; kc < nk; ++kc, ++c) {
+            for (int it = blockIdx.x; it < items; it += gridDim.x) {
+                for (int kc = k_lo(it); kc < k_hi(it); ++kc, ++c) {
                     const int w = c % C::WS;
                     if (c >= C::WS) mbar_wait(&w_empty[w], ((c / C::WS) - 1) & 1);
                     mbar_expect_tx(&w_full[w], C::W_BYTES);
@@ -439,11 +449,12 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
         // ---------------- MMA issuer ----------------
         const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NP >> 3) << 17) | ((128u >> 4) << 24);
         int c = 0, J = 0;
-        for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x, J += nseg) {
-            for (int kc = 0; kc < nk; ++kc, ++c) {
+        for (int it = blockIdx.x; it < items; it += gridDim.x) {
+            const int kc0 = k_lo(it), kc1 = k_hi(it);
+            for (int kc = kc0; kc < kc1; ++kc, ++c) {
                 const int h = c % C::NH, w = c % C::WS;
-                const int j = J + kc / C::SEG, slot = j & 1;
-                const bool first = (kc % C::SEG) == 0;
+                const int j = J + (kc - kc0) / C::SEG, slot = j & 1;
+                const bool first = ((kc - kc0) % C::SEG) == 0;
                 if (first && j >= 2) mbar_wait(&slot_free[slot], ((j >> 1) - 1) & 1);   // segment j-2 drained
                 mbar_wait(&split_full[h], (c / C::NH) & 1);
                 mbar_wait(&w_full[w], (c / C::WS) & 1);
@@ -463,10 +474,11 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
                     }
                     mma_commit(&hl_empty[h]);
                     mma_commit(&w_empty[w]);
-                    if ((kc % C::SEG) == C::SEG - 1 || kc == nk - 1) mma_commit(&seg_done[slot]);
+                    if (((kc - kc0) % C::SEG) == C::SEG - 1 || kc == kc1 - 1) mma_commit(&seg_done[slot]);
                 }
                 __syncwarp();
             }
+            J += (kc1 - kc0 + C::SEG - 1) / C::SEG;
         }
     } else {
         // ---------------- split, segment drains, epilogue (warps 2-5) ----------------
@@ -476,8 +488,11 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
 #pragma unroll
         for (int j = 0; j < NP; ++j) racc[j] = 0.f;
         int c = 0, J = 0;
-        for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x, J += nseg) {
-            for (int kc = 0; kc < nk; ++kc, ++c) {
+        for (int it = blockIdx.x; it < items; it += gridDim.x) {
+            const int tile = it / S;
+            const int kc0 = k_lo(it), kc1 = k_hi(it);
+            const int nseg = (kc1 - kc0 + C::SEG - 1) / C::SEG;
+            for (int kc = kc0; kc < kc1; ++kc, ++c) {
                 const int r = c % C::NR, h = c % C::NH;
                 mbar_wait(&raw_full[r], (c / C::NR) & 1);
                 // this thread's row (TMEM lane) of the 128B-swizzled raw tile: chunk q of row rr sits at
@@ -511,13 +526,20 @@ __global__ void __launch_bounds__(224, Tc2Cfg<NP>::CTAS) k_gemm_tc2(const __grid
                 asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
                 mbar_arrive(&split_full[h]);
                 mbar_arrive(&raw_empty[r]);                   // after the raw values were consumed (see k_gemm_tc_tn2)
-                if (((kc % C::SEG) == C::SEG - 1 || kc == nk - 1) && kc / C::SEG >= 1)
-                    drain_segment<NP, C::NA>(tmem, J + kc / C::SEG - 1, q4, seg_done, slot_free, racc);
+                if ((((kc - kc0) % C::SEG) == C::SEG - 1 || kc == kc1 - 1) && (kc - kc0) / C::SEG >= 1)
+                    drain_segment<NP, C::NA>(tmem, J + (kc - kc0) / C::SEG - 1, q4, seg_done, slot_free, racc);
             }
-            if (nk > 0) drain_segment<NP, C::NA>(tmem, J + nseg - 1, q4, seg_done, slot_free, racc);
+            if (nseg > 0) drain_segment<NP, C::NA>(tmem, J + nseg - 1, q4, seg_done, slot_free, racc);
+            J += nseg;
+            const int64_t gm = (int64_t)tile * C::BM + q4 * 32 + lane;
+            if (S > 1 && gm < a.M) {
+                // K split: the raw partial row (no epilogue) -> part[s][gm][0 .. NP); k_splitk_reduce finishes it
+                float4* pp = reinterpret_cast<float4*>(a.part + ((it % S) * a.M + gm) * NP);
+#pragma unroll
+                for (int j = 0; j < NP; j += 4) pp[j / 4] = make_float4(racc[j], racc[j + 1], racc[j + 2], racc[j + 3]);
+            }
             // epilogue: bias, activation, row scale; 128-bit stores when the rows allow it
-            const int64_t gm = tile * C::BM + q4 * 32 + lane;
-            if (gm < a.M) {
+            if (S == 1 && gm < a.M) {
                 const float rs = a.row_scale ? __ldg(a.row_scale + gm) : 1.f;
                 float* y = a.Y + gm * a.ldy;
                 const bool vec = (a.ldy & 3) == 0 && aligned16(a.Y);
@@ -567,10 +589,17 @@ __global__ void k_split_w(const float* __restrict__ W, int64_t K, int64_t N, int
     }
 }
 
-size_t linear_fwd_tc_workspace(int64_t K, int64_t N) {
+static size_t wsplit_bytes(int64_t K, int64_t N) {
     const int64_t np = (N + 15) / 16 * 16;
-    return (size_t)((K + 31) / 32) * 2 * np * 32 * sizeof(float) + 256;
+    return ((size_t)((K + 31) / 32) * 2 * np * 32 * sizeof(float) + 255) & ~size_t(255);
 }
+// + room for the K-split partials of k_gemm_tc2 (K >= 1024, N <= 64: the long-K transforms)
+static size_t splitk_part_bytes(int64_t K, int64_t N) {
+    if (K < 1024 || N > 64) return 0;
+    const int64_t np = (N + 15) / 16 * 16;
+    return (size_t)kSplitKMax * (size_t)splitk_max_rows() * (size_t)np * sizeof(float);
+}
+size_t linear_fwd_tc_workspace(int64_t K, int64_t N) { return wsplit_bytes(K, N) + splitk_part_bytes(K, N) + 256; }
 
 // ------------------------------------------------------------------------------------------------
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
@@ -587,6 +616,48 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
     return fn;
 }
 
+// K-split finish: Y[m, j] = row_scale[m] * act(sum_s part[s][m][j] + bias[j]), splits summed in order
+template <int NP>
+__global__ void __launch_bounds__(256) k_splitk_reduce(const float* __restrict__ part, int S, int64_t M, int N,
+                                                       const float* __restrict__ bias, const float* __restrict__ row_scale,
+                                                       int act, float* __restrict__ Y, int64_t ldy) {
+    constexpr int Q = NP / 4;
+    const int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (idx >= M * Q) return;
+    const int64_t m = idx / Q;
+    const int q = (int)(idx % Q);
+    float4 z = __ldcs(reinterpret_cast<const float4*>(part + m * NP) + q);
+    for (int sp = 1; sp < S; ++sp) {
+        const float4 v = __ldcs(reinterpret_cast<const float4*>(part + ((int64_t)sp * M + m) * NP) + q);
+        z.x += v.x; z.y += v.y; z.z += v.z; z.w += v.w;
+    }
+    const float rs = row_scale ? __ldg(row_scale + m) : 1.f;
+    const float zz[4] = {z.x, z.y, z.z, z.w};
+    float* y = Y + m * ldy + 4 * q;
+    float o[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) o[u] = rs * act_apply(act, zz[u] + ((bias && 4 * q + u < N) ? __ldg(bias + 4 * q + u) : 0.f));
+    if (4 * q + 4 <= N && (ldy & 3) == 0 && aligned16(Y)) {
+        *reinterpret_cast<float4*>(y) = make_float4(o[0], o[1], o[2], o[3]);
+    } else {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            if (4 * q + u < N) y[u] = o[u];
+    }
+}
+
+// K splits for k_gemm_tc2 when the row tiles alone cannot fill the grid (CoraFull / Physics / Cora: few rows, long K):
+// the split count minimising (waves of work items) x (chunks per item)
+static int choose_ksplit(int64_t tiles, int nk, int64_t slots) {
+    int best = 1;
+    int64_t best_cost = nk;
+    for (int S = 2; S <= kSplitKMax; S *= 2) {
+        if (nk < 4 * S) break;
+        const int64_t cost = ((tiles * S + slots - 1) / slots) * ((nk + S - 1) / S) + 2;   // + the reduce pass
+        if (cost < best_cost) { best_cost = cost; best = S; }
+    }
+    return best;
+}
 template <int NP>
 static seastar_status launch_tc_np(const CUtensorMap& tm, const TcArgs& a, cudaStream_t s) {
     // NP <= 64 (every BASELINE transform): k_gemm_tc2; wider outputs and SEASTAR_TC_V1=1 (A/B): k_gemm_tc
@@ -597,9 +668,19 @@ static seastar_status launch_tc_np(const CUtensorMap& tm, const TcArgs& a, cudaS
             SS_CUDA(cudaFuncSetAttribute(k_gemm_tc2<NP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C2::SMEM));
             const int64_t tiles = (a.M + C2::BM - 1) / C2::BM;
             const int64_t slots = (int64_t)C2::CTAS * num_sms();
-            const unsigned grid = (unsigned)(tiles < slots ? tiles : slots);
-            k_gemm_tc2<NP><<<grid, 224, C2::SMEM, s>>>(tm, a);
-            return check_launch("k_gemm_tc2");
+            TcArgs b = a;
+            b.ksplit = (a.part && a.M <= splitk_max_rows()) ? choose_ksplit(tiles, (int)((a.K + 31) / 32), slots) : 1;
+            const int64_t items = tiles * b.ksplit;
+            const unsigned grid = (unsigned)(items < slots ? items : slots);
+            k_gemm_tc2<NP><<<grid, 224, C2::SMEM, s>>>(tm, b);
+            SS_TRY(check_launch("k_gemm_tc2"));
+            if (b.ksplit > 1) {
+                const int64_t n = a.M * (NP / 4);
+                k_splitk_reduce<NP><<<(unsigned)((n + 255) / 256), 256, 0, s>>>(b.part, b.ksplit, a.M, (int)a.N, a.bias,
+                                                                             a.row_scale, a.act, a.Y, a.ldy);
+                SS_TRY(check_launch("k_splitk_reduce"));
+            }
+            return SEASTAR_OK;
         }
     }
     using C = TcCfg<NP>;
@@ -636,6 +717,7 @@ seastar_status linear_fwd_tc(const float* X, int64_t M, int64_t K, int64_t ldx, 
         SS_TRY(check_launch("k_split_w"));
     }
     TcArgs a{M, K, N, wsplit, Y, ldy, bias, row_scale, act};
+    if (splitk_part_bytes(K, N)) a.part = reinterpret_cast<float*>(static_cast<char*>(ws) + wsplit_bytes(K, N));
     switch (np) {
         case 16: return launch_tc_np<16>(tm, a, s);
         case 32: return launch_tc_np<32>(tm, a, s);

@@ -44,7 +44,8 @@ def test_linear_fwd(env, M, K, N):
 
 TC_SHAPES = [(128, 32, 16), (1000, 602, 16), (5003, 602, 64), (777, 64, 41), (3001, 1433, 70), (300, 8710, 8),
              (2048, 100, 128), (129, 33, 1),
-             (60000, 602, 64)]   # many chunks per CTA: the raw-tile ring wraps many times (r2: a WAR race showed here)
+             (60000, 602, 64),   # many chunks per CTA: the raw-tile ring wraps many times (r2: a WAR race showed here)
+             (5000, 2048, 64), (19793, 8710, 64), (2708, 1433, 16)]   # K splits (few row tiles, long K)
 
 
 @pytest.mark.parametrize("M,K,N", TC_SHAPES)
