@@ -45,7 +45,7 @@ inline cudaStream_t to_stream(seastar_stream s) { return reinterpret_cast<cudaSt
 // ----------------------------------------------------------------------------------------------
 // the graph handle (all index arrays are int32 on the device; E < 2^31 is validated at create)
 // ----------------------------------------------------------------------------------------------
-constexpr int kPow2Lo = 6, kPow2Classes = 11;   // degree thresholds 64 .. 65536 for the long-row split
+constexpr int kPow2Lo = 2, kPow2Classes = 15;   // degree thresholds 4 .. 65536 (long-row split, medium-row class)
 
 struct IndexSet {
     int32_t* perm = nullptr;   // row -> vertex id            [n_rows]   (nullptr for LSF: identity)

@@ -24,6 +24,11 @@
 
 namespace seastar {
 
+#ifndef H1_MID_CLASS
+#define H1_MID_CLASS 1   // single-head GAT rows with degree >= 2^(kPow2Lo + H1_MID_CLASS) = 8 take 16-lane row groups
+#endif
+constexpr int kH1MidClass = H1_MID_CLASS;
+
 // lane geometry of the chunked kernels: chunk `chunk` covers floats [chunk*VEC, chunk*VEC+VEC)
 // of a row of W = H*F floats; with VEC = 4 every chunk lies inside one head (F % 4 == 0 or H == 1)
 template <int VEC>
@@ -736,7 +741,7 @@ seastar_status seastar_gat_fwd(seastar_graph g, const float* T_all, const float*
     SS_ARG(!attn_drop || (attn_drop->p >= 0.f && attn_drop->p < 1.f), "gat_fwd: need 0 <= attn_drop->p < 1");
     set_drop(a, attn_drop, g->fwd.eid);
     if (!a.deid && launch_gat_fwd_hpl(a, long_rows(g->fwd), s)) return check_launch("k_gat_fwd_hpl");
-    if (!a.deid && launch_gat_fwd_h1(a, long_rows(g->fwd), g->fwd.bucket_rows[1], g->fwd.n_rows, s))
+    if (!a.deid && launch_gat_fwd_h1(a, long_rows(g->fwd), g->fwd.bucket_rows[1], g->fwd.pow2_rows[kH1MidClass], g->fwd.n_rows, s))
         return check_launch("k_gat_fwd_h1");
     const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_all) && aligned16(A_loc) &&
                       aligned16(Y_loc);
@@ -810,7 +815,7 @@ seastar_status seastar_gat_bwd(seastar_graph g, const float* T_loc, const float*
     SS_ARG(!attn_drop || (attn_drop->p >= 0.f && attn_drop->p < 1.f), "gat_bwd: need 0 <= attn_drop->p < 1");
     set_drop(a, attn_drop, g->rev.eid);
     if (!a.deid && launch_gat_bwd_hpl(a, long_rows(g->rev), s)) return check_launch("k_gat_bwd_hpl");
-    if (!a.deid && launch_gat_bwd_h1(a, long_rows(g->rev), g->rev.bucket_rows[1], g->rev.n_rows, false, s))
+    if (!a.deid && launch_gat_bwd_h1(a, long_rows(g->rev), g->rev.bucket_rows[1], g->rev.pow2_rows[kH1MidClass], g->rev.n_rows, false, s))
         return check_launch("k_gat_bwd_h1");
     const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_loc) && aligned16(D_all) &&
                       aligned16(dT_loc);
@@ -842,7 +847,7 @@ seastar_status seastar_gat_der(seastar_graph g, const float* T_all, const float*
     SS_ARG(!attn_drop || (attn_drop->p >= 0.f && attn_drop->p < 1.f), "gat_der: need 0 <= attn_drop->p < 1");
     set_drop(a, attn_drop, g->fwd.eid);
     if (!a.deid && launch_gat_der_hpl(a, s)) return check_launch("k_gat_der_hpl");
-    if (!a.deid && launch_gat_bwd_h1(a, long_rows(g->fwd), g->fwd.bucket_rows[1], g->fwd.n_rows, true, s))
+    if (!a.deid && launch_gat_bwd_h1(a, long_rows(g->fwd), g->fwd.bucket_rows[1], g->fwd.pow2_rows[kH1MidClass], g->fwd.n_rows, true, s))
         return check_launch("k_gat_der_h1");
     const bool vec4 = (ldt % 4 == 0) && (H == 1 || F % 4 == 0) && aligned16(T_all) && aligned16(D_loc);
     const int VEC = vec4 ? 4 : 1;

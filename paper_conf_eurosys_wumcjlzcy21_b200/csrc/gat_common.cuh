@@ -82,8 +82,10 @@ inline int64_t el_stride(const float* T, const float* el, int H, int F, int64_t 
 bool launch_gat_fwd_hpl(const GatFwdArgs& a, int64_t hub, cudaStream_t s);
 bool launch_gat_bwd_hpl(const GatBwdArgs& a, int64_t hub, cudaStream_t s);
 bool launch_gat_der_hpl(const GatBwdArgs& a, cudaStream_t s);
-bool launch_gat_fwd_h1(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t n_rows, cudaStream_t s);
-bool launch_gat_bwd_h1(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t n_rows, bool der, cudaStream_t s);
+// mid: rows with degree >= 8 (IndexSet::pow2_rows[0]); rows [split, mid) take 16-lane row groups
+bool launch_gat_fwd_h1(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t mid, int64_t n_rows, cudaStream_t s);
+bool launch_gat_bwd_h1(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t mid, int64_t n_rows, bool der,
+                       cudaStream_t s);
 
 // head-per-lane geometry: H | 32, every head row is whole float4s held by one lane
 inline int hpl_f4(int H, int F, int64_t ldt, bool aligned) {

@@ -376,46 +376,58 @@ __global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdA
 // ---------------------------------------------------------------------------------------------
 constexpr int kHubWarpsH1 = 8;      // warps per hub row (degree >= 1024)
 
-template <typename Args, typename LH, typename LW, typename LS>
-static void h1_buckets(const Args& a, int64_t hub, int64_t split, int64_t n_rows, LH lh, LW lw, LS ls) {
-    Args hi = a, lo = a;
+// degree classes: [0, split) warp rows (degree >= 32; the first `hub` of them long rows with a CTA each),
+// [split, mid) 16-lane row groups (8 <= degree < 32: 16 / L edges in flight per row instead of one slot of 4 lanes --
+// the small graphs' latency-bound class, r2), [mid, n_rows) 4-lane row groups
+template <typename Args, typename LH, typename LW, typename LM, typename LS>
+static void h1_buckets(const Args& a, int64_t hub, int64_t split, int64_t mid, int64_t n_rows, LH lh, LW lw, LM lm,
+                       LS ls) {
+    Args hi = a, md = a, lo = a;
+    mid = std::min<int64_t>(std::max<int64_t>(mid, split), n_rows);
     hi.row_begin = 0; hi.row_end = split;
     hi.nlong = std::min<int64_t>(hub, split);
-    lo.row_begin = split; lo.row_end = n_rows;
+    md.row_begin = split; md.row_end = mid; md.nlong = 0;
+    lo.row_begin = mid; lo.row_end = n_rows;
     lo.nlong = 0;
     if (split > 0) {
         const unsigned g = (unsigned)(hi.nlong + (split - hi.nlong + 7) / 8);
         if (hi.nlong > 0) lh(hi, g);                                        // long rows + warp rows, one launch
         else lw(hi, g);
     }
-    if (n_rows > split) ls(lo, (unsigned)((n_rows - split + 63) / 64));   // RL = 4: 64 rows per block
+    if (mid > split) lm(md, (unsigned)((mid - split + 15) / 16));          // RL = 16: 16 rows per block
+    if (n_rows > mid) ls(lo, (unsigned)((n_rows - mid + 63) / 64));       // RL = 4: 64 rows per block
 }
 
 template <int VPL, int L>
-static void fwd_h1_run(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t n, cudaStream_t s) {
+static void fwd_h1_run(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t mid, int64_t n, cudaStream_t s) {
     if (a.B)
-        h1_buckets(a, hub, split, n,
+        h1_buckets(a, hub, split, mid, n,
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 32, true, kHubWarpsH1>, dim3(g), dim3(32 * kHubWarpsH1), 0, s, x); },
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 32, true>, dim3(g), dim3(256), 0, s, x); },
+                   [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 16, true>, dim3(g), dim3(256), 0, s, x); },
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 4, true>, dim3(g), dim3(256), 0, s, x); });
     else
-        h1_buckets(a, hub, split, n,
+        h1_buckets(a, hub, split, mid, n,
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 32, false, kHubWarpsH1>, dim3(g), dim3(32 * kHubWarpsH1), 0, s, x); },
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 32, false>, dim3(g), dim3(256), 0, s, x); },
+                   [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 16, false>, dim3(g), dim3(256), 0, s, x); },
                    [&](const GatFwdArgs& x, unsigned g) { launch_k(k_gat_fwd_h1<VPL, L, 4, false>, dim3(g), dim3(256), 0, s, x); });
 }
 
 template <int VPL, int L>
-static void bwd_h1_run(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t n, bool der, cudaStream_t s) {
+static void bwd_h1_run(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t mid, int64_t n, bool der,
+                       cudaStream_t s) {
     if (der)
-        h1_buckets(a, hub, split, n,
+        h1_buckets(a, hub, split, mid, n,
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 32, true, kHubWarpsH1>, dim3(g), dim3(32 * kHubWarpsH1), 0, s, x); },
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 32, true>, dim3(g), dim3(256), 0, s, x); },
+                   [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 16, true>, dim3(g), dim3(256), 0, s, x); },
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 4, true>, dim3(g), dim3(256), 0, s, x); });
     else
-        h1_buckets(a, hub, split, n,
+        h1_buckets(a, hub, split, mid, n,
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 32, false, kHubWarpsH1>, dim3(g), dim3(32 * kHubWarpsH1), 0, s, x); },
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 32, false>, dim3(g), dim3(256), 0, s, x); },
+                   [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 16, false>, dim3(g), dim3(256), 0, s, x); },
                    [&](const GatBwdArgs& x, unsigned g) { launch_k(k_gat_bwd_h1<VPL, L, 4, false>, dim3(g), dim3(256), 0, s, x); });
 }
 
@@ -441,18 +453,19 @@ static void bwd_h1_run(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t 
         default: RUN<8, 4>(__VA_ARGS__); break;                                   \
     }
 
-bool launch_gat_fwd_h1(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t n_rows, cudaStream_t s) {
+bool launch_gat_fwd_h1(const GatFwdArgs& a, int64_t hub, int64_t split, int64_t mid, int64_t n_rows, cudaStream_t s) {
     int vpl = 0, L = 0;
     if (!h1_geometry(a.H, a.F, a.ld, aligned16(a.T) && aligned16(a.A) && aligned16(a.Y), vpl, L)) return false;
-    SS_H1_DISPATCH(fwd_h1_run, vpl, L, a, hub, split, n_rows, s)
+    SS_H1_DISPATCH(fwd_h1_run, vpl, L, a, hub, split, mid, n_rows, s)
     return true;
 }
 
-bool launch_gat_bwd_h1(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t n_rows, bool der, cudaStream_t s) {
+bool launch_gat_bwd_h1(const GatBwdArgs& a, int64_t hub, int64_t split, int64_t mid, int64_t n_rows, bool der,
+                       cudaStream_t s) {
     int vpl = 0, L = 0;
     const bool al = der ? aligned16(a.T) && aligned16(a.D) : aligned16(a.T) && aligned16(a.D) && aligned16(a.dT);
     if (!h1_geometry(a.H, a.F, a.ldt, al, vpl, L)) return false;
-    SS_H1_DISPATCH(bwd_h1_run, vpl, L, a, hub, split, n_rows, der, s)
+    SS_H1_DISPATCH(bwd_h1_run, vpl, L, a, hub, split, mid, n_rows, der, s)
     return true;
 }
 
