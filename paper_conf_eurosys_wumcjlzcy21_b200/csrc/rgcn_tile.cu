@@ -175,10 +175,9 @@ __device__ __forceinline__ void process_tile(const RgcnTileArgs& a, const TileBu
         order[atomicAdd(&hist[t], 1)] = ((uint32_t)t << 16) | (uint32_t)i;
     }
     __syncthreads();
-    // products: the two half-warps take alternate pairs of positions of the warp's stretch of the type-major order;
-    // lane (j, e) keeps column j of W'_t (all 4 FG4 gathered features) for its half-warp's current type t, reloaded
-    // only when the type changes, and computes output j of two edges per step from the staged rows (broadcast
-    // reads; four independent FMA chains per edge).  order[] packs (type << 16 | slot).
+    // products: lane (j, e) keeps column j of W'_t (all 4 FG4 gathered features) for its half-warp's current type t,
+    // reloaded only when the type changes, and computes output j of its half-warp's edges from the staged rows
+    // (broadcast reads; four independent FMA chains per edge).  order[] packs (type << 16 | slot).
     {
         constexpr int KP = 4 * FG4;
         const int j = lane & 15, e = lane >> 4;
@@ -212,31 +211,46 @@ __device__ __forceinline__ void process_tile(const RgcnTileArgs& a, const TileBu
             }
             return (m[0] + m[1]) + (m[2] + m[3]);
         };
-        for (int pb = p0; pb < p1; pb += 4) {                // warp-uniform trip count
-            const int pA = pb + e, pB = pb + 2 + e;
-            const bool liveA = pA < p1, liveB = pB < p1;
-            const uint32_t oA = liveA ? order[pA] : 0u, oB = liveB ? order[pB] : 0u;
-            const int iA = (int)(oA & 0xffffu), iB = (int)(oB & 0xffffu);
-            float4 xA[FG4], xB[FG4];
+        // each half-warp walks its own contiguous half of the stretch, UE edges per step (their rows' loads all in
+        // flight before the FMAs); both halves step together (warp-uniform trip count and branch: a step takes the
+        // fast path when every live edge of both halves has its half's current type)
+        constexpr int UE = 4;
+        const int pm = p0 + (p1 - p0 + 1) / 2;
+        const int q0 = e ? pm : p0, q1 = e ? p1 : pm;
+        const int steps = (pm - p0 + UE - 1) / UE;           // the first half is the longer one
+        for (int st = 0; st < steps; ++st) {                 // warp-uniform trip count
+            const int pb = q0 + st * UE;
+            uint32_t o[UE];
+            float4 x[UE][FG4];
 #pragma unroll
-            for (int q = 0; q < FG4; ++q) {
-                xA[q] = b.slot[iA * SW4 + q];
-                xB[q] = b.slot[iB * SW4 + q];
+            for (int u = 0; u < UE; ++u) {
+                o[u] = pb + u < q1 ? order[pb + u] : 0xffffffffu;
+                const int i = o[u] != 0xffffffffu ? (int)(o[u] & 0xffffu) : 0;
+#pragma unroll
+                for (int q = 0; q < FG4; ++q) x[u][q] = b.slot[i * SW4 + q];
             }
-            float mA = 0.f, mB = 0.f;
-            if (liveA) {
-                if ((int)(oA >> 16) != cur) reload((int)(oA >> 16));   // half-warp-uniform
-                mA = dot(xA);
+            bool same = true;
+#pragma unroll
+            for (int u = 0; u < UE; ++u) same &= (o[u] == 0xffffffffu) || (int)(o[u] >> 16) == cur;
+            float m[UE];
+            if (__all_sync(FULL, same)) {                    // warp-uniform
+#pragma unroll
+                for (int u = 0; u < UE; ++u) m[u] = dot(x[u]);
+            } else {
+#pragma unroll
+                for (int u = 0; u < UE; ++u) {
+                    if (o[u] != 0xffffffffu && (int)(o[u] >> 16) != cur) reload((int)(o[u] >> 16));
+                    m[u] = dot(x[u]);
+                }
             }
-            if (liveB) {
-                if ((int)(oB >> 16) != cur) reload((int)(oB >> 16));
-                mB = dot(xB);
-            }
-            const float nA = b.snorm[iA], nB = b.snorm[iB];
+            float nrm[UE];
+#pragma unroll
+            for (int u = 0; u < UE; ++u) nrm[u] = o[u] != 0xffffffffu ? b.snorm[o[u] & 0xffffu] : 0.f;
             __syncwarp();                                    // every lane's reads of its rows before the writes
             if (j < 4 * FO4) {
-                if (liveA) reinterpret_cast<float*>(b.slot + iA * SW4)[j] = mA * nA;
-                if (liveB) reinterpret_cast<float*>(b.slot + iB * SW4)[j] = mB * nB;
+#pragma unroll
+                for (int u = 0; u < UE; ++u)
+                    if (o[u] != 0xffffffffu) reinterpret_cast<float*>(b.slot + (o[u] & 0xffffu) * SW4)[j] = m[u] * nrm[u];
             }
         }
     }
