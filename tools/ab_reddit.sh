@@ -1,0 +1,9 @@
+# Reddit step: A/B of library variants (variants/libseastar_X.so; needs variants/ on the box), per-kernel timers
+LIB=paper_conf_eurosys_wumcjlzcy21_b200/libseastar.so
+cp $LIB /tmp/libseastar_orig.so
+trap 'cp /tmp/libseastar_orig.so $LIB' EXIT
+for v in base "$@" base; do
+  if [ $v != base ]; then cp variants/libseastar_$v.so $LIB; else cp /tmp/libseastar_orig.so $LIB; fi
+  timeout 300 python bench.py --no-cpu-baseline --no-e2e --steps 20 > /tmp/b.json 2>/dev/null
+  python -c "import json;d=json.load(open('/tmp/b.json'));print('$v', round(d['ms_per_step'],4), {k:round(v['ms'],4) for k,v in d['kernels'].items()})"
+done
