@@ -46,17 +46,18 @@ struct AggArgs {
     int phase; const int32_t* lcnt; const float* tloc; int64_t ldloc; float* part; int64_t ldp;
 };
 
-// minimum resident blocks (0: compiler's choice, 48 registers at F = 16).  Measured on Reddit: forcing 6 blocks
-// (40 registers) speeds the plain-sum sweep at F = 32 / 64 (1.12 / 2.00 -> 1.01 / 1.88 ms) but slows the GCN
-// training aggregation with its fused epilogue (0.68 -> 0.73 ms), so the default leaves it to the compiler
+// minimum resident blocks.  Measured on Reddit (r1/r2): with one index chunk per iteration, forcing 6 blocks (40
+// registers) sped the plain-sum sweep at F = 32 / 64 (1.12 / 2.00 -> 1.01 / 1.88 ms) but slowed the GCN training
+// aggregation (0.68 -> 0.73 ms).  r2 (second session): two index chunks per iteration for warp rows (AGG_NB4 = 2,
+// 64 edges' gathers in flight per warp: the kernel is bound by bytes in flight, long-scoreboard stalls) at 4 blocks
+// per SM (64 registers): GCN aggregation 0.68 -> 0.61 ms; NB = 2 at the compiler's 66 registers 0.79 ms, at 5 blocks
+// (spills) 0.78 ms, NB = 3 at 4 blocks 0.78 ms (tools/ab_reddit.sh)
 #ifndef AGG_MB
-#define AGG_MB 0
+#define AGG_MB 4
 #endif
-#if AGG_MB > 0
-#define AGG_BOUNDS __launch_bounds__(256, AGG_MB)
-#else
-#define AGG_BOUNDS __launch_bounds__(256)
-#endif
+// (applied to the two-chunk warp-row instances only: the other classes keep the compiler's choice -- at 4 blocks the
+// APPNP propagation on the Physics shape lost 10 %)
+#define AGG_BOUNDS __launch_bounds__(256, (AGG_MB > 0 && L >= 4 && NB >= 2) ? AGG_MB : 1)
 // WPR > 1 (RL = 32, WPR = the block's warps): the launch's first a.nlong blocks each own one long row (long_rows():
 // degree above a quarter of one SM's share of the launch) -- warp w walks the w-th contiguous slice of the row's
 // edges, and the warps' partial sums are added in warp order through shared memory before warp 0 runs the epilogue
@@ -245,6 +246,9 @@ __global__ void AGG_BOUNDS k_aggregate(const AggArgs a) {
 }
 
 constexpr int kHubWarps = 8;       // warps per hub row (degree >= 1024: >= 128 edges per warp)
+#ifndef AGG_NB4
+#define AGG_NB4 2                  // index chunks per iteration for warp rows with L >= 4 (see AGG_MB)
+#endif
 
 template <int VEC, int L, int PH>
 static void launch_rl_ph(AggArgs a, bool warp_rows, cudaStream_t s, bool hub) {
@@ -253,7 +257,7 @@ static void launch_rl_ph(AggArgs a, bool warp_rows, cudaStream_t s, bool hub) {
     constexpr int threads = 256;
     if (hub) {                                   // long rows (a CTA each) + warp rows in one launch
         static_assert(32 * kHubWarps == threads, "hub CTAs are the launch's 256-thread blocks");
-        constexpr int NBW = L >= 4 ? 1 : 4 / L;
+        constexpr int NBW = L >= 4 ? AGG_NB4 : 4 / L;
         const unsigned grid = (unsigned)(a.nlong + (rows - a.nlong + kHubWarps - 1) / kHubWarps);
         if (a.deid) launch_k(k_aggregate<VEC, L, 32, NBW, true, kHubWarps, PH>, dim3(grid), dim3(threads), 0, s, a);
         else launch_k(k_aggregate<VEC, L, 32, NBW, false, kHubWarps, PH>, dim3(grid), dim3(threads), 0, s, a);
@@ -265,7 +269,7 @@ static void launch_rl_ph(AggArgs a, bool warp_rows, cudaStream_t s, bool hub) {
         // buys more memory-level parallelism than deeper per-lane batches
         // narrow rows (L < 4 chunk lanes, F <= 8) take 4/L index chunks per iteration so every lane still has
         // 4 gathers in flight: F = 8 0.75 -> 0.50 ms, F = 1..4 0.54 -> 0.46 ms on Reddit (tools/ab_gcn.sh)
-        constexpr int NBW = L >= 4 ? 1 : 4 / L;
+        constexpr int NBW = L >= 4 ? AGG_NB4 : 4 / L;
         if (a.deid) launch_k(k_aggregate<VEC, L, 32, NBW, true, 1, PH>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
         else launch_k(k_aggregate<VEC, L, 32, NBW, false, 1, PH>, dim3((unsigned)blocks), dim3(threads), 0, s, a);
     } else {
