@@ -14,7 +14,13 @@ namespace seastar {
 #define GAT_H1_UBMAX 4
 #endif
 template <int VPL>
-constexpr int h1_ub() { return (VPL <= 2 ? 4 : 2) < GAT_H1_UBMAX ? (VPL <= 2 ? 4 : 2) : GAT_H1_UBMAX; }
+#ifndef GAT_H1_UB3
+#define GAT_H1_UB3 2        // edges per slot per batch at VPL = 3 (Reddit's F = 41 layer; A/B knob)
+#endif
+constexpr int h1_ub() {
+    return (VPL <= 2 ? 4 : (VPL == 3 ? GAT_H1_UB3 : 2)) < GAT_H1_UBMAX ? (VPL <= 2 ? 4 : (VPL == 3 ? GAT_H1_UB3 : 2))
+                                                                      : GAT_H1_UBMAX;
+}
 
 // load the lane's chunks of a row; chunks at or past W are zero (never loaded).  Columns inside
 // the last partial chunk are loaded as stored (row padding): callers either zero the matching
@@ -34,7 +40,10 @@ __device__ __forceinline__ float4 mask_tail(float4 x, int nv) {
 // of the row's edges, slices merged in warp order by the online-softmax merge through shared memory; later blocks
 // own 8 warp rows (as k_gat_fwd_hpl)
 template <int VPL, int L, int RL, bool SB, int WPR = 1>
-__global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs a) {
+#ifndef GAT_MB_FWD_H1
+#define GAT_MB_FWD_H1 GAT_MB_FWD
+#endif
+__global__ void __launch_bounds__(256, GAT_MB_FWD_H1) k_gat_fwd_h1(const GatFwdArgs a) {
     static_assert(WPR == 1 || RL == 32, "hub rows take whole warps");
     constexpr int NV = 4 * VPL, S = RL / L;
     constexpr int UE = h1_ub<VPL>() < L ? h1_ub<VPL>() : L;   // edges per slot per batch
@@ -218,11 +227,21 @@ __global__ void __launch_bounds__(256, GAT_MB_FWD) k_gat_fwd_h1(const GatFwdArgs
 #ifndef GAT_H1_BWD_UBMAX
 #define GAT_H1_BWD_UBMAX 4
 #endif
+// VPL = 3 (Reddit's F = 41 layer): 4 edges per slot per batch at 2 blocks per SM (124 registers) -- measured
+// (tools/ab_reddit.sh): layer-2 backward 1.905 -> 1.833 ms; the forward keeps 2 edges at 3 blocks (4 edges: 2.00 ->
+// 2.44 ms at 2 blocks, spills at 3)
+#ifndef GAT_H1_BWD_UB3
+#define GAT_H1_BWD_UB3 4
+#endif
+#ifndef GAT_MB_BWD_H1_V3
+#define GAT_MB_BWD_H1_V3 2
+#endif
 template <int VPL, int L, int RL, bool DER, int WPR = 1>
-__global__ void __launch_bounds__(256, GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdArgs a) {
+__global__ void __launch_bounds__(256, VPL == 3 ? GAT_MB_BWD_H1_V3 : GAT_MB_BWD_H1) k_gat_bwd_h1(const GatBwdArgs a) {
     static_assert(WPR == 1 || RL == 32, "hub rows take whole warps");
     constexpr int NV = 4 * VPL, S = RL / L;
-    constexpr int UB0 = h1_ub<VPL>() < GAT_H1_BWD_UBMAX ? h1_ub<VPL>() : GAT_H1_BWD_UBMAX;
+    constexpr int UBV = VPL == 3 ? GAT_H1_BWD_UB3 : h1_ub<VPL>();
+    constexpr int UB0 = UBV < GAT_H1_BWD_UBMAX ? UBV : GAT_H1_BWD_UBMAX;
     constexpr int UE = UB0 < L ? UB0 : L;
     constexpr int NB = L / UE;
     const int lane = threadIdx.x & 31;
