@@ -34,7 +34,11 @@ constexpr int kTileThreads = 256;    // standalone tile kernel (W read through L
 #ifndef RGCN_TILE_PT
 #define RGCN_TILE_PT 512
 #endif
-constexpr int kTilePThreads = RGCN_TILE_PT;   // persistent tile kernel (one CTA per SM, W resident in shared memory)
+constexpr int kTilePThreads = RGCN_TILE_PT;
+#ifndef RGCN_W_SWIZZLE
+#define RGCN_W_SWIZZLE 1
+#endif
+constexpr bool kRgcnWSwizzle = RGCN_W_SWIZZLE;   // bank-conflict-free W' column reloads (FG4 = 4)   // persistent tile kernel (one CTA per SM, W resident in shared memory)
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
     const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
@@ -192,7 +196,7 @@ __device__ __forceinline__ void process_tile(const RgcnTileArgs& a, const TileBu
                 const float4* wc = reinterpret_cast<const float4*>(Ws + (t * 16 + j) * KP);
 #pragma unroll
                 for (int q = 0; q < FG4; ++q) {
-                    const float4 v = wc[q];
+                    const float4 v = wc[(FG4 == 4 && kRgcnWSwizzle) ? (q + (j >> 1)) & 3 : q];
                     w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
                 }
             } else {
@@ -373,7 +377,10 @@ __global__ void __launch_bounds__(kTilePThreads, 1) k_rgcn_tile_p(const RgcnTile
     }
     for (int idx = tid; idx < a.R * 16 * 4 * FG4; idx += NT) {      // W'_r as [R][16 (j)][4 FG4 (k)]
         const int k = idx % (4 * FG4), j = (idx / (4 * FG4)) & 15, r = idx / (64 * FG4);
-        Ws[idx] = (j < a.Fo && k < a.Fg) ? w_prime(a, r, k, j) : 0.f;
+        // FG4 = 4: chunk q of column j sits at chunk (q + j / 2) % 4, so the 8 lanes of a reload's quarter-warp hit 8
+        // different 16-byte bank groups (column stride 64 B: unswizzled, lanes j and j + 2 collide)
+        const int pk = (FG4 == 4 && kRgcnWSwizzle) ? ((((k >> 2) + (j >> 1)) & 3) << 2) | (k & 3) : k;
+        Ws[idx - k + pk] = (j < a.Fo && k < a.Fg) ? w_prime(a, r, k, j) : 0.f;
     }
     for (int it = 0; t < n_tiles; ++it, t += G) {
         const TileBuf& cur = (it & 1) ? buf1 : buf0;
