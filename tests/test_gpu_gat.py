@@ -42,7 +42,8 @@ def run_fwd(env, g, N, H, F, ld, T, el, er, b, act, slope=0.2, save_B=False):
 
 # covers: head-per-lane (H | 32, F % 4 == 0), single-head multi-chunk (H = 1, VPL 1..8), generic chunked
 CASES = [(1, 3), (1, 4), (1, 16), (1, 33), (1, 41), (1, 70), (1, 128), (2, 3), (2, 4), (8, 8), (4, 16), (8, 4),
-         (3, 5), (2, 32), (16, 4)]
+         (3, 5), (2, 32), (16, 4),
+         (8, 32), (16, 16), (32, 8)]   # rows of 256 floats: head-per-lane kernels (the chunked ones stop at 128)
 
 
 @pytest.mark.parametrize("H,F", CASES)
